@@ -1,0 +1,178 @@
+/*
+ * oracle.c -- TEST INFRASTRUCTURE ONLY (see oracle.h).  Plain C, fp64, no
+ * blocking / fusion / reordering beyond what the paper's algorithms state.
+ * Compiled with -O2 -ffp-contract=off (no FMA contraction, no fast-math).
+ */
+#include "oracle.h"
+
+#include <math.h>
+#include <stddef.h>
+#include <string.h>
+
+/* ------------------------------------------------------------ SpMM ------ */
+/* Algorithm 1. */
+int oracle_spmm(int64_t i0, int64_t i1, const int32_t *row_ind, const int32_t *col_ind,
+                const float *val, int64_t K, const float *A, int64_t lda, int64_t r0,
+                int64_t nrows, double *O, double *T) {
+  if (i0 < 0 || i1 < i0 || K < 1 || lda < K || nrows < 0) return -1;
+  memset(O, 0, sizeof(double) * (size_t)(nrows * K));
+  if (T) memset(T, 0, sizeof(double) * (size_t)(nrows * K));
+  for (int64_t i = i0; i < i1; ++i) {                       /* line 1 */
+    int64_t r = row_ind[i], c = col_ind[i];                 /* line 2 */
+    double v = val ? (double)val[i] : 1.0;
+    if (r < r0 || r >= r0 + nrows || c < 0) return -1;
+    double *o = O + (r - r0) * K;
+    const float *a = A + c * lda;
+    for (int64_t k = 0; k < K; ++k) {                       /* line 3 */
+      double term = v * (double)a[k];
+      o[k] += term;                                         /* line 4 */
+      if (T) T[(r - r0) * K + k] += fabs(term);
+    }
+  }
+  return 0;
+}
+
+/* ----------------------------------------------------------- SDDMM ------ */
+/* Algorithm 2. */
+int oracle_sddmm(int64_t i0, int64_t i1, const int32_t *row_ind, const int32_t *col_ind,
+                 const float *val, int64_t K, const float *A1, int64_t lda1,
+                 const float *A2T, int64_t lda2, double *out, double *T) {
+  if (i0 < 0 || i1 < i0 || K < 1 || lda1 < K || lda2 < K) return -1;
+  for (int64_t i = i0; i < i1; ++i) {                       /* line 1 */
+    int64_t r = row_ind[i], c = col_ind[i];                 /* line 2 */
+    double v = val ? (double)val[i] : 1.0;
+    if (r < 0 || c < 0) return -1;
+    const float *a1 = A1 + r * lda1;
+    const float *a2 = A2T + c * lda2;                       /* A2[k][c] = A2T[c][k] */
+    double acc = 0.0, tabs = 0.0;
+    for (int64_t k = 0; k < K; ++k) {                       /* line 3 */
+      double term = (double)a1[k] * (double)a2[k];
+      acc += term;                                          /* line 4 */
+      tabs += fabs(term);
+    }
+    out[i - i0] = acc * v;                                  /* line 6 */
+    if (T) T[i - i0] = fabs(v) * tabs;
+  }
+  return 0;
+}
+
+/* ------------------------------------------------------------ plan ------ */
+/* NnzPerWarp candidate set. */
+static const int32_t kCandidates[6] = {8, 32, 64, 128, 256, 512};
+
+static int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+/* Right-hand side of InEq. (5) in integer form: the number of thread
+ * blocks launched when every chunk of C nnz is cut into S K-slices, each slice
+ * is one lane group's work item, G groups share a warp, WPB warps a block. */
+static int64_t blocks_for(int64_t nnz, int64_t C, int64_t S, int64_t G, int64_t WPB) {
+  int64_t chunks = cdiv(nnz, C);
+  int64_t items = chunks * S;
+  int64_t warps = cdiv(items, G);
+  return cdiv(warps, WPB);
+}
+
+int oracle_plan(int64_t nnz, const int32_t *row_ind, int32_t K, int32_t alpha,
+                int32_t warps_per_block, int32_t force_chunk, int32_t force_vw,
+                int32_t num_sms, int32_t active_blocks_per_sm, oracle_plan_info_t *info,
+                int32_t *row_first, int32_t *row_last, uint8_t *flags) {
+  if (nnz < 0 || K < 1 || alpha < 1 || warps_per_block < 1 || num_sms < 1 ||
+      active_blocks_per_sm < 1 || force_chunk < 0 || !info)
+    return -1;
+  /* step 1: feature vector width from K alone (or forced) */
+  int32_t vw;
+  if (force_vw > 0) {
+    if (!(force_vw == 1 || force_vw == 2 || force_vw == 4 || force_vw == 8)) return -1;
+    if (K % force_vw != 0) return -1;
+    vw = force_vw;
+  } else if (K % 8 == 0 && K >= 256) {
+    vw = 8;
+  } else if (K % 4 == 0) {
+    vw = 4;
+  } else if (K % 2 == 0) {
+    vw = 2;
+  } else {
+    vw = 1;
+  }
+  /* step 2: lanes per chunk-slice, slices, groups per warp */
+  int64_t need = cdiv(K, vw);
+  int32_t L = 1;
+  while (L < need && L < 32) L *= 2;
+  int32_t S = (int32_t)cdiv(K, (int64_t)L * vw);
+  int32_t G = 32 / L;
+  /* step 3: FullWaveSize = NumSM x ActiveblocksPerSM (Eqs. 3-4) */
+  int64_t FW = (int64_t)num_sms * active_blocks_per_sm;
+  /* steps 4-5: largest candidate satisfying InEq. (5), else 8 */
+  int32_t C = 8;
+  for (int j = 0; j < 6; ++j) {
+    if (blocks_for(nnz, kCandidates[j], S, G, warps_per_block) >= (int64_t)alpha * FW)
+      C = kCandidates[j];
+  }
+  if (force_chunk > 0) C = force_chunk;
+  /* step 6: sparse-load vector width (HVMA) */
+  int32_t vws = 1;
+  if (C >= 128 && C % 4 == 0) vws = 4;
+  else if (C >= 64 && C % 2 == 0) vws = 2;
+  /* step 7: chunks (Algo 3 lines 2-3: warp_start = id x NnzPerWarp, end clamped) */
+  int64_t nch = nnz > 0 ? cdiv(nnz, C) : 0;
+  info->chunk = C;
+  info->vw_feat = vw;
+  info->vw_sparse = vws;
+  info->lanes = L;
+  info->slices = S;
+  info->groups = G;
+  info->warps_per_block = warps_per_block;
+  info->active_blocks_per_sm = active_blocks_per_sm;
+  info->num_sms = num_sms;
+  info->alpha = alpha;
+  info->K = K;
+  info->nnz = nnz;
+  info->num_chunks = nch;
+  info->num_blocks = nnz > 0 ? blocks_for(nnz, C, S, G, warps_per_block) : 0;
+  for (int64_t c = 0; c < nch; ++c) {
+    int64_t s = c * C;
+    int64_t e = s + C < nnz ? s + C : nnz;
+    if (row_first) row_first[c] = row_ind[s];
+    if (row_last) row_last[c] = row_ind[e - 1];
+    if (flags) {
+      uint8_t f = 0;
+      if (s > 0 && row_ind[s - 1] == row_ind[s]) f |= 1;      /* head continues */
+      if (e < nnz && row_ind[e] == row_ind[e - 1]) f |= 2;    /* tail continues */
+      flags[c] = f;
+    }
+  }
+  return 0;
+}
+
+/* ---------------------------------------------------------- shards ------ */
+int oracle_shard_rows(const int32_t *row_ptr, int64_t M, int32_t P, int64_t *bounds) {
+  if (!row_ptr || M < 0 || P < 1 || !bounds) return -1;
+  int64_t base = row_ptr[0];
+  int64_t nnz = (int64_t)row_ptr[M] - base;
+  bounds[0] = 0;
+  for (int32_t p = 1; p < P; ++p) {
+    int64_t t = (int64_t)p * nnz / P;
+    int64_t lo = 0, hi = M; /* first r in [0, M] with row_ptr[r] - base >= t */
+    while (lo < hi) {
+      int64_t mid = lo + (hi - lo) / 2;
+      if ((int64_t)row_ptr[mid] - base >= t) hi = mid; else lo = mid + 1;
+    }
+    bounds[p] = lo < bounds[p - 1] ? bounds[p - 1] : lo;
+  }
+  bounds[P] = M;
+  return 0;
+}
+
+int oracle_shard_edges(int64_t nnz, int32_t P, int64_t *bounds) {
+  if (nnz < 0 || P < 1 || !bounds) return -1;
+  for (int32_t p = 0; p <= P; ++p) bounds[p] = (int64_t)p * nnz / P;
+  return 0;
+}
+
+int oracle_csr_to_coo(const int32_t *row_ptr, int64_t M, int32_t *row_ind) {
+  if (!row_ptr || M < 0) return -1;
+  int64_t base = row_ptr[0];
+  for (int64_t r = 0; r < M; ++r)
+    for (int64_t i = row_ptr[r]; i < row_ptr[r + 1]; ++i) row_ind[i - base] = (int32_t)r;
+  return 0;
+}
