@@ -1,0 +1,512 @@
+#!/usr/bin/env python
+"""Benchmark of the hot path (plan + SpMM + SDDMM) on B200.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                    [--workload C4|C5|C2|C1] [--K 32,64,128,256] [--xmode replicate|allgather]
+
+A step = one pass of the whole hot path over the workload: for every K in --K, the
+DTP plan (GPU plan kernel), SpMM (O = S X) and SDDMM (out = v * <X_r, X_c>, A1 = A2T =
+X as in GNN use).  BASELINE.json metric: "SpMM/SDDMM GB/s & GFLOP/s vs HBM roofline
+at K=32-256, 1/2/4/8 B200", quoted on the Reddit-shaped graph (configs[3] = C4).
+
+value = algorithmic bytes of all kernels of the step (SURVEY.md §8(d) byte model,
+DESIGN.md "Measurement") / device time, whole job (sum over ranks / max-over-ranks
+time).  Inputs are resident in HBM; L2 is flushed (256 MiB write) between timed
+steps, outside the timed events.  Multi-GPU (torchrun): SpMM rows and SDDMM edges are
+nnz-balanced shards (gnn_shard_rows / gnn_shard_edges); X replicated (default) or
+NCCL all-gathered inside the step (--xmode allgather).  Strong scaling: the graph is
+fixed, N GPUs split it.
+
+--impl reference runs the fp64 CPU oracle (the only "reference" this paper has) as
+it stands on a bounded sample of the same workload, on rank 0 only.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "SpMM/SDDMM GB/s & GFLOP/s vs HBM roofline at K=32–256, 1/2/4/8 B200"
+WORKLOAD_DESC = {
+    "C4": "Reddit-shaped synthetic power-law graph (N=232,965, nnz=114,848,857, self-looped, "
+          "50 planted communities, GCN values)",
+    "C5": "ogbn-products-shaped synthetic power-law graph (N=2,449,029, nnz=126,167,053, "
+          "500 planted communities, GCN values)",
+    "C2": "Cora/PubMed-shaped synthetic GCN graph (N=20,000, nnz=100,000)",
+    "C1": "tiny synthetic power-law graph (N=1,000, nnz=10,000)",
+}
+
+
+# ------------------------------------------------------------- byte model ---
+def spmm_bytes(nnz, M, K):
+    """Per nnz: 12 B sparse (row, col, val) + 4K B gathered feature row; per output
+    row 4K B written."""
+    return nnz * (12 + 4 * K) + 4 * K * M
+
+
+def sddmm_bytes(nnz, M, K):
+    """Per nnz: 12 B sparse + 4 B out + 4K B gathered A2T row; per row 4K B of A1."""
+    return nnz * (16 + 4 * K) + 4 * K * M
+
+
+def plan_bytes(nch):
+    return nch * (16 + 9)
+
+
+def spmm_flops(nnz, K):
+    return 2 * nnz * K
+
+
+def sddmm_flops(nnz, K):
+    return (2 * K + 1) * nnz
+
+
+def hbm_compulsory(nnz, M, N, K, kind):
+    if kind == "spmm":
+        return 12 * nnz + 4 * K * (N + M)
+    return 16 * nnz + 4 * K * (M + N)
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d.get("hbm_gbs", 6650.0)), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+def load_ncu_traffic():
+    """DRAM bytes per launch from the committed `ncu --set full` summary, if any."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(p):
+        try:
+            return json.load(open(p))
+        except Exception:
+            return {}
+    return {}
+
+
+# ----------------------------------------------------------------- clocks ---
+class ClockSampler:
+    def __init__(self, device_index):
+        self.proc = None
+        self.path = None
+        self.dev = device_index
+
+    def start(self):
+        try:
+            fd, self.path = tempfile.mkstemp(suffix=".csv")
+            os.close(fd)
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.dev),
+                 "--query-gpu=clocks.sm,clocks.max.sm,power.draw,"
+                 "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+                 "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return None
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        rows = []
+        for line in open(self.path):
+            f = [x.strip() for x in line.split(",")]
+            if len(f) >= 7:
+                try:
+                    rows.append((float(f[0]), float(f[1]), f[3:7]))
+                except ValueError:
+                    pass
+        os.unlink(self.path)
+        if not rows:
+            return None
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for _, _, r in rows for i in range(4) if r[i] == "Active"})
+        return {"sm_mhz": statistics.median(r[0] for r in rows),
+                "sm_max_mhz": max(r[1] for r in rows), "reasons": reasons,
+                "samples": len(rows)}
+
+
+# ------------------------------------------------------------- workload -----
+def build_graph(name):
+    from gen import configs
+    if name in configs.CONFIGS:
+        return configs.make_graph(name)
+    raise SystemExit(f"unknown workload {name}")
+
+
+def parse_ks(s, name):
+    from gen import configs
+    if s:
+        return [int(x) for x in s.split(",")]
+    return configs.CONFIGS[name]["K"]
+
+
+# ------------------------------------------------------------ our impl ------
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+
+    import gen
+    import paper_conf_ipps_fanwc23_b200 as gs
+    from gen import configs
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        ncores = os.cpu_count() or 1
+        os.environ.setdefault("OMP_NUM_THREADS", str(max(1, ncores // world)))
+    dev = torch.device("cuda", local if world > 1 else 0)
+    torch.cuda.set_device(dev)
+    gs.lib()
+
+    name = args.workload
+    Ks = parse_ks(args.K, name)
+    t0 = time.time()
+    g = build_graph(name)
+    gen_s = time.time() - t0
+    P, p = world, rank
+    rb = gs.shard_rows(g.row_ptr, P)
+    eb = gs.shard_edges(g.nnz, P)
+    r0, r1 = int(rb[p]), int(rb[p + 1])
+    e0, e1 = int(g.row_ptr[r0]), int(g.row_ptr[r1])
+    f0, f1 = int(eb[p]), int(eb[p + 1])
+
+    full = gs.DeviceGraph.from_arrays(g.M, g.N, g.row_ind, g.col_ind, g.val, g.row_ptr, device=dev)
+    spg = full.shard(r0, r1, e0, e1) if P > 1 else full
+    sdg = gs.DeviceGraph(g.M, g.N, full.row_ind[f0:f1], full.col_ind[f0:f1],
+                         full.val[f0:f1]) if P > 1 else full
+    # X: replicated (generated on every rank: deterministic) or all-gathered
+    blk = -(-g.N // P)
+    X, Xown = {}, {}
+    for K in Ks:
+        if args.xmode == "allgather" and P > 1:
+            own = gen.features(configs.FEATURE_SEED[name] * 16, min(blk, max(0, g.N - p * blk)),
+                               K, row0=p * blk)
+            buf = torch.zeros((blk, K), dtype=torch.float32, device=dev)
+            buf[:own.shape[0]] = torch.from_numpy(own).to(dev)
+            Xown[K] = buf
+            X[K] = torch.empty((blk * P, K), dtype=torch.float32, device=dev)
+        else:
+            X[K] = torch.from_numpy(configs.make_features(name, g.N, K)).to(dev)
+    O = {K: torch.empty((spg.M, K), dtype=torch.float32, device=dev) for K in Ks}
+    E = torch.empty(sdg.nnz, dtype=torch.float32, device=dev)
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
+    stream = torch.cuda.current_stream()
+    same = (P == 1)
+
+    launches_per_step = 0
+
+    def step(ev=None):
+        nonlocal launches_per_step
+        n = 0
+        for K in Ks:
+            if args.xmode == "allgather" and P > 1:
+                dist.all_gather_into_tensor(X[K], Xown[K])
+            if ev is not None:
+                ev[K][0].record(stream)
+            pl = gs.plan(spg, K)
+            n += 1
+            if ev is not None:
+                ev[K][1].record(stream)
+            gs.spmm(pl, spg, X[K], out=O[K])
+            n += 2 if spg.nnz else 0
+            if ev is not None:
+                ev[K][2].record(stream)
+            pl2 = pl if same else gs.plan(sdg, K)
+            n += 0 if same else 1
+            gs.sddmm(pl2, sdg, X[K], X[K], out=E)
+            n += 1 if sdg.nnz else 0
+            if ev is not None:
+                ev[K][3].record(stream)
+        launches_per_step = n
+
+    # warm-up
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+
+    ev = [{K: [torch.cuda.Event(enable_timing=True) for _ in range(4)] for K in Ks}
+          for _ in range(args.steps)]
+    clk = ClockSampler(dev.index)
+    clk.start()
+    time.sleep(0.3)
+    step_ms = []
+    for s in range(args.steps):
+        flush.fill_(float(s))  # L2 flush between timed steps (outside the events)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        step(ev[s])
+        torch.cuda.synchronize()
+    clocks = clk.stop()
+    per = {K: {"plan": [], "spmm": [], "sddmm": []} for K in Ks}
+    for s in range(args.steps):
+        tot = 0.0
+        for K in Ks:
+            e = ev[s][K]
+            a, b, c = e[0].elapsed_time(e[1]), e[1].elapsed_time(e[2]), e[2].elapsed_time(e[3])
+            per[K]["plan"].append(a)
+            per[K]["spmm"].append(b)
+            per[K]["sddmm"].append(c)
+            tot += a + b + c
+        step_ms.append(tot)
+    my_ms = float(sum(step_ms))
+
+    # bytes / flops of this rank's kernels
+    my_bytes = 0
+    my_flops = 0
+    detail = {}
+    for K in Ks:
+        b_sp = spmm_bytes(spg.nnz, spg.M, K)
+        b_sd = sddmm_bytes(sdg.nnz, g.M, K) if not same else sddmm_bytes(spg.nnz, spg.M, K)
+        info = gs.plan(spg, K).info()
+        b_pl = plan_bytes(info["num_chunks"])
+        my_bytes += b_sp + b_sd + b_pl
+        my_flops += spmm_flops(spg.nnz, K) + sddmm_flops(sdg.nnz, K)
+        t_sp = statistics.mean(per[K]["spmm"])
+        t_sd = statistics.mean(per[K]["sddmm"])
+        t_pl = statistics.mean(per[K]["plan"])
+        detail[f"K{K}"] = {
+            "chunk": info["chunk"], "vw_feat": info["vw_feat"], "lanes": info["lanes"],
+            "active_blocks_per_sm": info["active_blocks_per_sm"],
+            "plan_ms": round(t_pl, 4), "spmm_ms": round(t_sp, 4), "sddmm_ms": round(t_sd, 4),
+            "spmm_GBps": round(b_sp / t_sp / 1e6, 1), "sddmm_GBps": round(b_sd / t_sd / 1e6, 1),
+            "spmm_GFLOPs": round(spmm_flops(spg.nnz, K) / t_sp / 1e6, 1),
+            "sddmm_GFLOPs": round(sddmm_flops(sdg.nnz, K) / t_sd / 1e6, 1),
+            "spmm_hbm_compulsory_GBps": round(hbm_compulsory(spg.nnz, spg.M, g.N, K, "spmm")
+                                              / t_sp / 1e6, 1),
+        }
+
+    # aggregate over ranks: sum of work, max of time
+    if world > 1:
+        t = torch.tensor([my_ms, float(my_bytes), float(my_flops)], dtype=torch.float64,
+                         device=dev)
+        mx = t.clone()
+        dist.all_reduce(mx, op=dist.ReduceOp.MAX)
+        sm = t.clone()
+        dist.all_reduce(sm, op=dist.ReduceOp.SUM)
+        tot_ms, tot_bytes, tot_flops = float(mx[0]), float(sm[1]), float(sm[2])
+    else:
+        tot_ms, tot_bytes, tot_flops = my_ms, float(my_bytes), float(my_flops)
+    tot_bytes *= args.steps
+    tot_flops *= args.steps
+    value = tot_bytes / (tot_ms * 1e-3) / 1e9
+
+    # dominant kernel (largest share of this rank's step time) -> roofline
+    shares = {(K, kind): statistics.mean(per[K][kind]) for K in Ks for kind in ("spmm", "sddmm")}
+    (dK, dkind), dms = max(shares.items(), key=lambda kv: kv[1])
+    dbytes = spmm_bytes(spg.nnz, spg.M, dK) if dkind == "spmm" else sddmm_bytes(sdg.nnz, g.M, dK)
+    peak, peak_src = load_peaks()
+    achieved = dbytes / (dms * 1e-3) / 1e9
+    traffic = load_ncu_traffic().get(f"{name}:{dkind}:K{dK}")
+    roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                "frac": round(achieved / peak, 4), "traffic": traffic,
+                "kernel": f"{dkind} K={dK} ({name})", "peak_source": peak_src,
+                "algorithmic_bytes_per_launch": int(dbytes),
+                "share_of_step": round(dms / (my_ms / args.steps), 4),
+                "hbm_compulsory_frac": round(
+                    hbm_compulsory(spg.nnz if dkind == "spmm" else sdg.nnz, spg.M, g.N, dK,
+                                   dkind) / (dms * 1e-3) / 1e9 / peak, 4)}
+
+    # e2e through the public API with host buffers (pinned), rank 0's numbers
+    e2e = run_e2e(args, g, Ks, dev, full if P == 1 else None) if (P == 1 and not args.no_e2e) \
+        else None
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        cpu = cpu_baseline(g, Ks, args.cpu_seconds, name)
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": round(tot_ms / args.steps, 4), "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": f"{name}: {WORKLOAD_DESC.get(name, name)}", "K": Ks,
+                       "nnz": g.nnz, "M": g.M, "N": g.N, "degree": g.degree_stats(),
+                       "step": "per K: plan (GPU plan kernel) + SpMM + SDDMM",
+                       "l2": "flushed between timed steps (256 MiB write, outside events)",
+                       "parallelism": f"rowshard-spmm/edgeshard-sddmm x{world}",
+                       "xmode": args.xmode, "graph_gen_s": round(gen_s, 1)},
+            "gflops": round(tot_flops / (tot_ms * 1e-3) / 1e9, 1),
+            "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+            "gpu_launches": launches_per_step * args.steps, "clocks": clocks,
+            "kernels": detail,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def run_e2e(args, g, Ks, dev, full):
+    """Same metric end to end through the public API: every step copies the graph
+    arrays and X from pinned host memory, runs plan + SpMM + SDDMM, and copies O and the
+    SDDMM output back to pinned host memory; all inside the CUDA-event timed region."""
+    import torch
+
+    import paper_conf_ipps_fanwc23_b200 as gs
+    from gen import configs
+
+    pin = lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory()
+    h_ri, h_ci, h_v = pin(g.row_ind), pin(g.col_ind), pin(g.val)
+    h_X = {K: pin(configs.make_features(args.workload, g.N, K)) for K in Ks}
+    h_O = {K: torch.empty((g.M, K), dtype=torch.float32).pin_memory() for K in Ks}
+    h_E = torch.empty(g.nnz, dtype=torch.float32).pin_memory()
+    d_ri = torch.empty_like(h_ri, device=dev)
+    d_ci = torch.empty_like(h_ci, device=dev)
+    d_v = torch.empty_like(h_v, device=dev)
+    d_X = {K: torch.empty_like(h_X[K], device=dev) for K in Ks}
+    d_O = {K: torch.empty((g.M, K), dtype=torch.float32, device=dev) for K in Ks}
+    d_E = torch.empty(g.nnz, dtype=torch.float32, device=dev)
+    dg = gs.DeviceGraph(g.M, g.N, d_ri, d_ci, d_v)
+    h2d = 12 * g.nnz + sum(4 * g.N * K for K in Ks)
+    d2h = sum(4 * g.M * K for K in Ks) + 4 * g.nnz * len(Ks)
+
+    def step():
+        d_ri.copy_(h_ri, non_blocking=True)
+        d_ci.copy_(h_ci, non_blocking=True)
+        d_v.copy_(h_v, non_blocking=True)
+        for K in Ks:
+            d_X[K].copy_(h_X[K], non_blocking=True)
+            p = gs.plan(dg, K)
+            gs.spmm(p, dg, d_X[K], out=d_O[K])
+            gs.sddmm(p, dg, d_X[K], d_X[K], out=d_E)
+            h_O[K].copy_(d_O[K], non_blocking=True)
+            h_E.copy_(d_E, non_blocking=True)
+
+    for _ in range(max(1, min(args.warmup, 2))):
+        step()
+    torch.cuda.synchronize()
+    steps = max(1, min(args.steps, 5))
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record()
+    for _ in range(steps):
+        step()
+    b.record()
+    torch.cuda.synchronize()
+    ms = a.elapsed_time(b) / steps
+    nbytes = sum(spmm_bytes(g.nnz, g.M, K) + sddmm_bytes(g.nnz, g.M, K) for K in Ks)
+    return {"value": round(nbytes / (ms * 1e-3) / 1e9, 2), "unit": "GB/s",
+            "ms_per_step": round(ms, 3), "h2d_bytes_per_step": int(h2d),
+            "d2h_bytes_per_step": int(d2h), "steps": steps}
+
+
+# --------------------------------------------------------- CPU baseline -----
+def oracle_sample(g, Ks, budget_s, name):
+    """Time the oracle (as it stands, single-threaded fp64 C) on a bounded contiguous
+    row sample of the workload: rows [0, r) with r grown until the run costs about
+    budget_s seconds.  Returns (GB/s by the same byte model, description, seconds)."""
+    import oracle
+    from gen import configs
+    X = {K: configs.make_features(name, g.N, K) for K in Ks}
+    # calibrate on a small sample
+    rows = max(1, min(g.M, 64))
+    while True:
+        e = int(g.row_ptr[rows])
+        t0 = time.perf_counter()
+        nbytes = 0
+        for K in Ks:
+            oracle.spmm(g.row_ind, g.col_ind, g.val, X[K], i0=0, i1=e, r0=0, nrows=rows)
+            oracle.sddmm(g.row_ind, g.col_ind, g.val, X[K], X[K], i0=0, i1=e)
+            nbytes += spmm_bytes(e, rows, K) + sddmm_bytes(e, rows, K)
+        dt = time.perf_counter() - t0
+        if dt >= budget_s or rows >= g.M:
+            return nbytes / dt / 1e9, f"rows [0,{rows}) = {e} nnz of {g.nnz}, K={Ks}", dt
+        grow = min(8.0, max(1.5, budget_s / max(dt, 1e-3)))
+        rows = min(g.M, int(rows * grow) + 1)
+
+
+def cpu_baseline(g, Ks, budget_s, name):
+    gbps, sample, dt = oracle_sample(g, Ks, budget_s, name)
+    return {"value": round(gbps, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+            "sample": sample, "seconds": round(dt, 2),
+            "cpu": _cpu_model()}
+
+
+def _cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return "unknown"
+
+
+def run_reference(args):
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    name = args.workload
+    Ks = parse_ks(args.K, name)
+    g = build_graph(name)
+    per_step = max(1.0, min(20.0, 60.0 / max(1, args.steps + args.warmup)))
+    for _ in range(args.warmup):
+        oracle_sample(g, Ks, per_step / 4, name)
+    vals, secs, desc = [], 0.0, ""
+    for _ in range(args.steps):
+        v, desc, dt = oracle_sample(g, Ks, per_step, name)
+        vals.append(v)
+        secs += dt
+    value = statistics.mean(vals)
+    line = {"impl": "reference", "metric": METRIC, "value": round(value, 4), "unit": "GB/s",
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": round(secs / args.steps * 1e3, 2), "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": f"{name}: {WORKLOAD_DESC.get(name, name)}", "K": Ks,
+                       "step": "oracle (fp64 C, Algorithms 1-2) SpMM + SDDMM on a bounded "
+                               "row sample per K"},
+            "cpu_baseline": {"value": round(value, 4), "unit": "GB/s", "cores": 1,
+                             "kind": "oracle", "sample": desc, "cpu": _cpu_model()},
+            "e2e": {"value": round(value, 4), "unit": "GB/s", "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--workload", default="C4")
+    ap.add_argument("--K", default="")
+    ap.add_argument("--xmode", default="replicate", choices=["replicate", "allgather"])
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3 and args.impl == "ours":
+        args.warmup = 3
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

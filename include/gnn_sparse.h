@@ -1,0 +1,173 @@
+/*
+ * gnn_sparse.h -- C ABI of libgnnsparse.so, the B200 (sm_100a) hybrid-parallel
+ * SpMM / SDDMM library for GNN message passing.
+ *
+ * Paper: R. Fan, W. Wang, X. Chu, "Fast Sparse GPU Kernels for Accelerated Training
+ * of Graph Neural Networks", IPDPS 2023.  "P:n" below is /root/reference/PAPER.md
+ * line n (the paper text; not needed at run time).
+ *
+ * Conventions for every entry point
+ *   - All array pointers are DEVICE pointers unless the name ends in _host.
+ *   - Sparse input is hybrid CSR/COO (Fig. 2d): row_ind[nnz] is the fully
+ *     decoded, NON-DECREASING row index; col_ind[nnz], val[nnz] (val may be NULL,
+ *     meaning every value is 1).  int32 indices, int64 sizes/offsets (P:295 max nnz
+ *     264M fits int32).  Row r is a destination node, column c a source node
+ *     (Table I).
+ *   - Dense matrices are row-major fp32 with a leading dimension (pitch, in
+ *     elements) >= K ("row-major ... FP32").
+ *   - The caller owns every buffer (graph arrays, features, outputs and the plan
+ *     workspace); the library never allocates device memory.
+ *   - Every call is asynchronous on the given stream (a cudaStream_t; NULL = the
+ *     legacy default stream) and never synchronises the host, except
+ *     gnn_validate().  Launch errors are returned as GNN_ERR_CUDA; faults inside a
+ *     kernel surface at the caller's next synchronisation.
+ *   - Calls return a gnn_status_t; no C++ exception crosses the ABI.  A thread-local
+ *     message for the last failure is available from gnn_last_error().
+ *   - There is no CPU fallback: without a usable sm_100 device every compute entry
+ *     point returns GNN_ERR_CUDA.
+ */
+#ifndef GNN_SPARSE_H
+#define GNN_SPARSE_H
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#if defined(_WIN32)
+#define GNN_API
+#else
+#define GNN_API __attribute__((visibility("default")))
+#endif
+
+typedef enum {
+  GNN_OK = 0,
+  GNN_ERR_INVALID_ARG = 1,   /* NULL pointer, negative size, K < 1, bad option   */
+  GNN_ERR_UNSUPPORTED = 2,   /* alignment/pitch not compatible with the plan's VW */
+  GNN_ERR_CUDA = 3,          /* CUDA runtime / launch error or no sm_100 device   */
+  GNN_ERR_WORKSPACE = 4,     /* workspace too small or misaligned                 */
+  GNN_ERR_INPUT_CHECK = 5    /* gnn_validate found an invalid graph               */
+} gnn_status_t;
+
+typedef void *gnn_stream_t; /* a cudaStream_t */
+
+/* A hybrid CSR/COO adjacency S (M x N) or a row/edge shard of one.
+ * A shard's row_ind holds GLOBAL row ids in [row_base, row_base + M); its
+ * row_ind/col_ind/val pointers are sub-views starting at the shard's first nnz.
+ * Kernels write output row r at O[(r - row_base) * ldo]. */
+typedef struct {
+  int64_t M, N, nnz;
+  const int32_t *row_ptr;  /* [M+1] CSR offsets, read relative to row_ptr[0]; only
+                              used by gnn_validate / gnn_csr_to_coo; may be NULL   */
+  const int32_t *row_ind;  /* [nnz] non-decreasing, in [row_base, row_base + M)     */
+  const int32_t *col_ind;  /* [nnz] in [0, N)                                       */
+  const float *val;        /* [nnz] or NULL (all ones)                              */
+  int64_t row_base;
+} gnn_graph_t;
+
+/* Plan options; zero-initialised fields take defaults. */
+typedef struct {
+  int32_t alpha;           /* InEq. (5) scale factor; default 2             */
+  int32_t warps_per_block; /* WarpsPerBlock; 1..16, default 8               */
+  int32_t force_chunk;     /* 0 = DTP choice; >0 forces NnzPerWarp (ablation/tests) */
+  int32_t force_vw;        /* 0 = from K; 1/2/4/8 forces the feature vector width   */
+  int32_t deterministic;   /* reserved (must be 0 in this version)                  */
+} gnn_plan_opts_t;
+
+/* What the plan decided (all integers; bit-exact with the oracle's plan). */
+typedef struct {
+  int32_t chunk;           /* C*: nnz per work chunk ("NnzPerWarp")    */
+  int32_t vw_feat;         /* feature-row vector width VW (floats per lane)         */
+  int32_t vw_sparse;       /* sparse-array vector width (HVMA): 1, 2 or 4     */
+  int32_t lanes;           /* L: lanes per chunk-slice                              */
+  int32_t slices;          /* S: K-slices per chunk                                 */
+  int32_t groups;          /* G = 32 / L chunk-slices per warp                      */
+  int32_t warps_per_block;
+  int32_t active_blocks_per_sm; /* occupancy API value for the SpMM kernel (Eq. 3)  */
+  int32_t num_sms;         /* NumSM (Eq. 4)                                         */
+  int32_t alpha;
+  int32_t K;
+  int64_t nnz;
+  int64_t num_chunks;      /* ceil(nnz / chunk)                                     */
+  int64_t num_blocks;      /* SpMM grid size (integer form of InEq. (5) RHS)         */
+} gnn_plan_info_t;
+
+typedef struct gnn_plan *gnn_plan_t;
+
+/* ---------------------------------------------------------------- plan ---- */
+/* Bytes of device workspace gnn_plan_create needs for (nnz, K, opts) on the current
+ * device (exact; 0 when nnz == 0).  Returns (size_t)-1 on invalid arguments. */
+GNN_API size_t gnn_plan_workspace_bytes(int64_t nnz, int32_t K, const gnn_plan_opts_t *opts);
+
+/* Dynamic Task Partition + Hierarchical Vectorized Memory Access and the
+ * per-chunk boundary table of the hybrid-parallel strategy (Algo 3 lines
+ * 2-3 P:175-176).  Host part: C* from InEq. (5) over the candidate set
+ * {8,32,64,128,256,512}, scalar integer arithmetic only -- no device read, no sync.
+ * Device part: one launch writing, for every chunk c (nnz [c*C*, min((c+1)*C*, nnz))),
+ *   row_first[c] = row_ind[start], row_last[c] = row_ind[end-1],
+ *   flags[c] = (head row continues from chunk c-1) | (tail row continues into c+1) << 1.
+ * workspace: device memory of gnn_plan_workspace_bytes() bytes, 256-byte aligned,
+ * owned by the caller; it must outlive every use of the plan.  The plan is bound to
+ * (graph arrays, nnz, K, device) and immutable; it may be used concurrently.
+ * opts may be NULL (defaults).  *out receives a host handle (free with
+ * gnn_plan_destroy). */
+GNN_API gnn_status_t gnn_plan_create(const gnn_graph_t *graph, int32_t K,
+                                     const gnn_plan_opts_t *opts, void *workspace,
+                                     size_t ws_bytes, gnn_stream_t stream, gnn_plan_t *out);
+GNN_API gnn_status_t gnn_plan_info(gnn_plan_t plan, gnn_plan_info_t *info);
+/* Device views of the plan's per-chunk arrays (inside the workspace). */
+GNN_API gnn_status_t gnn_plan_arrays(gnn_plan_t plan, const int32_t **row_first,
+                                     const int32_t **row_last, const uint8_t **flags);
+GNN_API void gnn_plan_destroy(gnn_plan_t plan);
+
+/* ------------------------------------------------------------- kernels ---- */
+/* SpMM, O = S A (Algorithm 1), hybrid-parallel (Algorithm 3
+ * P:168-195): O[r - row_base][k] = sum_{i : row_ind[i] = r} val[i] * A[col_ind[i]][k]
+ * for every r in [row_base, row_base + M), k in [0, K).  OVERWRITES O (rows without
+ * nnz become +0).  A: N x K (lda >= K), O: M x K (ldo >= K), fp32 accumulation.
+ * A, O must be 4*vw_feat-byte aligned and lda, ldo multiples of vw_feat, else
+ * GNN_ERR_UNSUPPORTED (re-plan with force_vw).  A and O must not overlap.
+ * Rows split across chunks are combined with vector atomic adds, so the fp32
+ * summation order of such rows is not deterministic (tolerance: DESIGN.md). */
+GNN_API gnn_status_t gnn_spmm(gnn_plan_t plan, const gnn_graph_t *graph, const float *A,
+                              int64_t lda, float *O, int64_t ldo, gnn_stream_t stream);
+
+/* SDDMM, S_O = (A1 A2) (.) S (Algorithm 2), hybrid-parallel
+ * (Algorithm 4): out[i] = val[i] * sum_k A1[row_ind[i] - row_base][k] *
+ * A2T[col_ind[i]][k] for i in [0, nnz).  A1: M x K (destination rows, lda1 >= K);
+ * A2T: N x K, the transpose of Table I's K x N A2 (source rows, lda2 >= K);
+ * out: nnz fp32 in col_ind order, each written exactly once (deterministic).
+ * Same alignment rules as gnn_spmm; uses the same plan. */
+GNN_API gnn_status_t gnn_sddmm(gnn_plan_t plan, const gnn_graph_t *graph, const float *A1,
+                               int64_t lda1, const float *A2T, int64_t lda2, float *out,
+                               gnn_stream_t stream);
+
+/* -------------------------------------------------------------- shards ---- */
+/* nnz-balanced contiguous row shards for P GPUs (HOST arrays; DESIGN.md
+ * "Multi-GPU"): t_p = floor(p * nnz / P), bounds[p] = first r with
+ * row_ptr[r] - row_ptr[0] >= t_p, bounds[0] = 0, bounds[P] = M (monotone).
+ * row_ptr_host: [M+1]; bounds: [P+1]. */
+GNN_API gnn_status_t gnn_shard_rows(const int32_t *row_ptr_host, int64_t M, int32_t P,
+                                    int64_t *bounds);
+/* Equal edge-range shards: bounds[p] = floor(p * nnz / P), [P+1] host array. */
+GNN_API gnn_status_t gnn_shard_edges(int64_t nnz, int32_t P, int64_t *bounds);
+
+/* ------------------------------------------------------------- helpers ---- */
+/* Decode CSR offsets into the hybrid format's RowInd (Fig. 2d):
+ * row_ind[i - row_ptr[0]] = r + row_base for row_ptr[r] <= i < row_ptr[r+1]. */
+GNN_API gnn_status_t gnn_csr_to_coo(const int32_t *row_ptr, int64_t M, int64_t row_base,
+                                    int32_t *row_ind, gnn_stream_t stream);
+/* Debug check of a graph's contents (row_ind non-decreasing and in range, col_ind
+ * in [0,N), row_ptr consistent when given).  SYNCHRONISES the stream.  Returns
+ * GNN_OK or GNN_ERR_INPUT_CHECK (message in gnn_last_error()). */
+GNN_API gnn_status_t gnn_validate(const gnn_graph_t *graph, gnn_stream_t stream);
+/* Thread-local description of the last failure on this thread ("" if none). */
+GNN_API const char *gnn_last_error(void);
+/* Library version string. */
+GNN_API const char *gnn_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* GNN_SPARSE_H */

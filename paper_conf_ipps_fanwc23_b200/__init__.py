@@ -1,0 +1,278 @@
+"""Thin Python binding of libgnnsparse.so (the C ABI in include/gnn_sparse.h).
+
+Hybrid-parallel SpMM / SDDMM for GNN message passing on B200 (sm_100a), after
+Fan, Wang, Chu, IPDPS 2023.  This module only marshals arguments:
+every step of the hot path (plan, SpMM, SDDMM) runs in the library's CUDA kernels.
+PyTorch provides device memory, streams and process groups.  There is no CPU
+fallback: if the shared library or a CUDA device is missing, calls raise.
+
+Names follow the C ABI: ``plan`` (gnn_plan_create), ``spmm`` (gnn_spmm),
+``sddmm`` (gnn_sddmm), ``shard_rows`` / ``shard_edges``, ``csr_to_coo``,
+``validate``.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass, field
+
+import numpy as np
+import torch
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libgnnsparse.so")
+
+__all__ = ["DeviceGraph", "Plan", "PlanOpts", "plan", "spmm", "sddmm", "shard_rows",
+           "shard_edges", "csr_to_coo", "validate", "GnnError", "lib", "LIB_PATH"]
+
+GNN_OK, GNN_ERR_INVALID_ARG, GNN_ERR_UNSUPPORTED, GNN_ERR_CUDA, GNN_ERR_WORKSPACE, \
+    GNN_ERR_INPUT_CHECK = range(6)
+
+
+class GnnError(RuntimeError):
+    def __init__(self, status, msg):
+        super().__init__(f"[gnn status {status}] {msg}")
+        self.status = status
+
+
+class _Graph(ctypes.Structure):
+    _fields_ = [("M", ctypes.c_int64), ("N", ctypes.c_int64), ("nnz", ctypes.c_int64),
+                ("row_ptr", ctypes.c_void_p), ("row_ind", ctypes.c_void_p),
+                ("col_ind", ctypes.c_void_p), ("val", ctypes.c_void_p),
+                ("row_base", ctypes.c_int64)]
+
+
+class PlanOpts(ctypes.Structure):
+    """gnn_plan_opts_t; zero fields take the library defaults (alpha 2, 8 warps/block)."""
+    _fields_ = [("alpha", ctypes.c_int32), ("warps_per_block", ctypes.c_int32),
+                ("force_chunk", ctypes.c_int32), ("force_vw", ctypes.c_int32),
+                ("deterministic", ctypes.c_int32)]
+
+
+class _PlanInfo(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_int32) for n in (
+        "chunk", "vw_feat", "vw_sparse", "lanes", "slices", "groups", "warps_per_block",
+        "active_blocks_per_sm", "num_sms", "alpha", "K")] + [
+        ("nnz", ctypes.c_int64), ("num_chunks", ctypes.c_int64), ("num_blocks", ctypes.c_int64)]
+
+
+EXPORTS = ["gnn_plan_workspace_bytes", "gnn_plan_create", "gnn_plan_info", "gnn_plan_arrays",
+           "gnn_plan_destroy", "gnn_spmm", "gnn_sddmm", "gnn_shard_rows", "gnn_shard_edges",
+           "gnn_csr_to_coo", "gnn_validate", "gnn_last_error", "gnn_version"]
+
+_lib = None
+
+
+def lib():
+    """Load libgnnsparse.so (raises if it has not been built -- no fallback)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} missing: run `make` (or __graft_entry__.build()) first")
+    L = ctypes.CDLL(LIB_PATH)
+    vp, i64, i32, st = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_int
+    P = ctypes.POINTER
+    L.gnn_plan_workspace_bytes.argtypes = [i64, i32, P(PlanOpts)]
+    L.gnn_plan_workspace_bytes.restype = ctypes.c_size_t
+    L.gnn_plan_create.argtypes = [P(_Graph), i32, P(PlanOpts), vp, ctypes.c_size_t, vp, P(vp)]
+    L.gnn_plan_info.argtypes = [vp, P(_PlanInfo)]
+    L.gnn_plan_arrays.argtypes = [vp, P(vp), P(vp), P(vp)]
+    L.gnn_plan_destroy.argtypes = [vp]
+    L.gnn_plan_destroy.restype = None
+    L.gnn_spmm.argtypes = [vp, P(_Graph), vp, i64, vp, i64, vp]
+    L.gnn_sddmm.argtypes = [vp, P(_Graph), vp, i64, vp, i64, vp, vp]
+    L.gnn_shard_rows.argtypes = [vp, i64, i32, vp]
+    L.gnn_shard_edges.argtypes = [i64, i32, vp]
+    L.gnn_csr_to_coo.argtypes = [vp, i64, i64, vp, vp]
+    L.gnn_validate.argtypes = [P(_Graph), vp]
+    L.gnn_last_error.argtypes = []
+    L.gnn_last_error.restype = ctypes.c_char_p
+    L.gnn_version.argtypes = []
+    L.gnn_version.restype = ctypes.c_char_p
+    for f in ("gnn_plan_create", "gnn_plan_info", "gnn_plan_arrays", "gnn_spmm", "gnn_sddmm",
+              "gnn_shard_rows", "gnn_shard_edges", "gnn_csr_to_coo", "gnn_validate"):
+        getattr(L, f).restype = st
+    _lib = L
+    return L
+
+
+def _check(status):
+    if status != GNN_OK:
+        raise GnnError(status, lib().gnn_last_error().decode())
+
+
+def _stream(stream=None):
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return ctypes.c_void_p(stream.cuda_stream)
+
+
+def _ptr(t):
+    return None if t is None else ctypes.c_void_p(t.data_ptr())
+
+
+# ----------------------------------------------------------------- graph ----
+@dataclass
+class DeviceGraph:
+    """Hybrid CSR/COO adjacency resident on a CUDA device.
+    row_ind is the decoded, non-decreasing row index; val None means all ones.
+    A row shard keeps global row ids in [row_base, row_base + M)."""
+    M: int
+    N: int
+    row_ind: torch.Tensor
+    col_ind: torch.Tensor
+    val: torch.Tensor | None = None
+    row_ptr: torch.Tensor | None = None
+    row_base: int = 0
+    _keep: list = field(default_factory=list, repr=False)
+
+    @property
+    def nnz(self) -> int:
+        return int(self.row_ind.numel())
+
+    @staticmethod
+    def from_arrays(M, N, row_ind, col_ind, val=None, row_ptr=None, device="cuda",
+                    row_base=0):
+        def dev(a, dt):
+            if a is None:
+                return None
+            t = torch.as_tensor(np.asarray(a) if not torch.is_tensor(a) else a)
+            return t.to(device=device, dtype=dt).contiguous()
+        return DeviceGraph(int(M), int(N), dev(row_ind, torch.int32), dev(col_ind, torch.int32),
+                           dev(val, torch.float32), dev(row_ptr, torch.int32), int(row_base))
+
+    def shard(self, r0: int, r1: int, e0: int, e1: int) -> "DeviceGraph":
+        """Zero-copy view of rows [r0, r1) whose nnz are [e0, e1) (a row shard)."""
+        return DeviceGraph(r1 - r0, self.N, self.row_ind[e0:e1], self.col_ind[e0:e1],
+                           None if self.val is None else self.val[e0:e1],
+                           None if self.row_ptr is None else self.row_ptr[r0:r1 + 1],
+                           self.row_base + r0)
+
+    def desc(self) -> _Graph:
+        return _Graph(self.M, self.N, self.nnz, _ptr(self.row_ptr), _ptr(self.row_ind),
+                      _ptr(self.col_ind), _ptr(self.val), self.row_base)
+
+
+# ------------------------------------------------------------------ plan ----
+class Plan:
+    """Owns the plan handle and its device workspace (a torch uint8 tensor)."""
+
+    def __init__(self, handle, workspace, graph, K):
+        self._h = handle
+        self.workspace = workspace
+        self.graph = graph
+        self.K = K
+
+    @property
+    def handle(self):
+        return self._h
+
+    def info(self) -> dict:
+        inf = _PlanInfo()
+        _check(lib().gnn_plan_info(self._h, ctypes.byref(inf)))
+        return {n: getattr(inf, n) for n, _ in _PlanInfo._fields_}
+
+    def arrays(self):
+        """(row_first, row_last, flags) as device tensors (views into the workspace)."""
+        rf, rl, fl = ctypes.c_void_p(), ctypes.c_void_p(), ctypes.c_void_p()
+        _check(lib().gnn_plan_arrays(self._h, ctypes.byref(rf), ctypes.byref(rl),
+                                     ctypes.byref(fl)))
+        nch = self.info()["num_chunks"]
+        if nch == 0:
+            z = torch.empty(0, dtype=torch.int32, device=self.workspace.device)
+            return z, z.clone(), torch.empty(0, dtype=torch.uint8, device=z.device)
+        base = self.workspace.data_ptr()
+        ws = self.workspace
+        def view(ptr, nbytes, dt):
+            off = ptr - base
+            return ws[off:off + nbytes].view(dt)
+        return (view(rf.value, 4 * nch, torch.int32), view(rl.value, 4 * nch, torch.int32),
+                view(fl.value, nch, torch.uint8))
+
+    def __del__(self):
+        h, self._h = getattr(self, "_h", None), None
+        if h and _lib is not None:
+            _lib.gnn_plan_destroy(h)
+
+
+def _opts(alpha=0, warps_per_block=0, force_chunk=0, force_vw=0):
+    return PlanOpts(alpha, warps_per_block, force_chunk, force_vw, 0)
+
+
+def plan(graph: DeviceGraph, K: int, alpha: int = 0, warps_per_block: int = 0,
+         force_chunk: int = 0, force_vw: int = 0, stream=None) -> Plan:
+    """gnn_plan_create: DTP/HVMA chunking + the GPU plan kernel (no host sync)."""
+    L = lib()
+    o = _opts(alpha, warps_per_block, force_chunk, force_vw)
+    nbytes = L.gnn_plan_workspace_bytes(graph.nnz, K, ctypes.byref(o))
+    if nbytes == ctypes.c_size_t(-1).value:
+        _check(GNN_ERR_INVALID_ARG)
+    dev = graph.row_ind.device
+    ws = torch.empty(max(int(nbytes), 1), dtype=torch.uint8, device=dev)
+    h = ctypes.c_void_p()
+    g = graph.desc()
+    _check(L.gnn_plan_create(ctypes.byref(g), K, ctypes.byref(o), _ptr(ws), int(nbytes),
+                             _stream(stream), ctypes.byref(h)))
+    return Plan(h, ws, graph, K)
+
+
+def _dense(t, name):
+    if t.dtype != torch.float32 or t.dim() != 2 or t.stride(1) != 1 or not t.is_cuda:
+        raise ValueError(f"{name} must be a CUDA fp32 row-major 2-D tensor")
+    return t
+
+
+def spmm(p: Plan, graph: DeviceGraph, A: torch.Tensor, out: torch.Tensor | None = None,
+         stream=None) -> torch.Tensor:
+    """gnn_spmm: O = S A (overwrites out; returns it)."""
+    K = p.K
+    _dense(A, "A")
+    if out is None:
+        out = torch.empty((graph.M, K), dtype=torch.float32, device=A.device)
+    _dense(out, "out")
+    g = graph.desc()
+    _check(lib().gnn_spmm(p.handle, ctypes.byref(g), _ptr(A), A.stride(0), _ptr(out),
+                          out.stride(0), _stream(stream)))
+    return out
+
+
+def sddmm(p: Plan, graph: DeviceGraph, A1: torch.Tensor, A2T: torch.Tensor,
+          out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """gnn_sddmm: out[i] = val[i] * <A1[row_i], A2T[col_i]> (returns out)."""
+    _dense(A1, "A1")
+    _dense(A2T, "A2T")
+    if out is None:
+        out = torch.empty(graph.nnz, dtype=torch.float32, device=A1.device)
+    g = graph.desc()
+    _check(lib().gnn_sddmm(p.handle, ctypes.byref(g), _ptr(A1), A1.stride(0), _ptr(A2T),
+                           A2T.stride(0), _ptr(out), _stream(stream)))
+    return out
+
+
+# ---------------------------------------------------------------- helpers ---
+def shard_rows(row_ptr, P: int) -> np.ndarray:
+    """gnn_shard_rows on a HOST row_ptr (numpy int32)."""
+    rp = np.ascontiguousarray(row_ptr, dtype=np.int32)
+    b = np.empty(P + 1, np.int64)
+    _check(lib().gnn_shard_rows(rp.ctypes.data, rp.shape[0] - 1, P, b.ctypes.data))
+    return b
+
+
+def shard_edges(nnz: int, P: int) -> np.ndarray:
+    b = np.empty(P + 1, np.int64)
+    _check(lib().gnn_shard_edges(nnz, P, b.ctypes.data))
+    return b
+
+
+def csr_to_coo(row_ptr: torch.Tensor, row_base: int = 0, stream=None) -> torch.Tensor:
+    M = row_ptr.numel() - 1
+    nnz = int(row_ptr[-1].item() - row_ptr[0].item()) if M >= 0 else 0
+    out = torch.empty(nnz, dtype=torch.int32, device=row_ptr.device)
+    _check(lib().gnn_csr_to_coo(_ptr(row_ptr), M, row_base, _ptr(out), _stream(stream)))
+    return out
+
+
+def validate(graph: DeviceGraph, stream=None) -> None:
+    g = graph.desc()
+    _check(lib().gnn_validate(ctypes.byref(g), _stream(stream)))

@@ -1,0 +1,66 @@
+// internal.cuh -- shared internals of libgnnsparse.so (not part of the ABI).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "gnn_sparse.h"
+
+namespace gnn {
+
+// Per-thread error message + status helpers (gnn_last_error()).
+gnn_status_t fail(gnn_status_t st, const char *fmt, ...);
+gnn_status_t cuda_fail(cudaError_t e, const char *what);
+void clear_error();
+
+// Cached per-device properties (queried once per device, no sync).
+struct DeviceInfo {
+  int device;
+  int num_sms;
+  int cc_major, cc_minor;
+};
+gnn_status_t device_info(DeviceInfo *out);
+
+// The plan handle (host struct; arrays live in the caller's workspace).
+struct Plan {
+  gnn_plan_info_t info;
+  int device;
+  const int32_t *row_ind;  // graph arrays the plan was built for
+  int32_t *row_first;
+  int32_t *row_last;
+  uint8_t *flags;
+  int64_t M;
+  int64_t row_base;
+};
+
+// Kernel parameter block shared by the SpMM / SDDMM launchers.
+struct SparseArgs {
+  const int32_t *__restrict__ row_ind;
+  const int32_t *__restrict__ col_ind;
+  const float *__restrict__ val;  // may be null
+  const int32_t *__restrict__ row_first;
+  const int32_t *__restrict__ row_last;
+  const uint8_t *__restrict__ flags;
+  int64_t nnz;
+  int64_t num_chunks;
+  int64_t row_base;
+  int64_t M;
+  int32_t chunk;
+  int32_t K;
+  int32_t slices;
+};
+
+// Occupancy (active blocks / SM) of the SpMM kernel for a feature width/lane count;
+// DTP's ActiveblocksPerSM (Eq. 3) -- defined in spmm.cu.
+int spmm_active_blocks_per_sm(int vw, int lanes, int warps_per_block);
+
+// Shared launcher helpers (spmm.cu).
+gnn_status_t check_common(const Plan *p, const gnn_graph_t *g, const char *who);
+int effective_vws(int vws, const gnn_graph_t *g, const void *extra);
+SparseArgs make_args(const Plan *p, const gnn_graph_t *g);
+
+// Valid warps_per_block range; block size = 32 * wpb <= kMaxThreads.
+constexpr int kMaxThreads = 512;
+
+inline bool aligned(const void *p, size_t a) { return (reinterpret_cast<uintptr_t>(p) % a) == 0; }
+
+}  // namespace gnn

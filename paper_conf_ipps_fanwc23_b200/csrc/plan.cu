@@ -1,0 +1,190 @@
+// plan.cu -- Dynamic Task Partition + HVMA candidate set:
+// host-side choice of the chunk size C* (scalar integer arithmetic, no device
+// reads, no sync) and the device plan kernel that tabulates, per chunk, its first
+// and last row and whether those rows continue into the neighbouring chunks (the
+// node boundaries the hybrid-parallel kernels must respect).
+#include <cuda_runtime.h>
+#include <string.h>
+
+#include <new>
+
+#include "internal.cuh"
+
+namespace gnn {
+
+namespace {
+
+// NnzPerWarp candidate set.
+constexpr int32_t kCand[6] = {8, 32, 64, 128, 256, 512};
+
+inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+inline size_t align256(size_t b) { return (b + 255) & ~size_t(255); }
+
+// InEq. (5) RHS in integer form (DESIGN.md "Plan rule" step 4).
+inline int64_t blocks_for(int64_t nnz, int64_t C, int64_t S, int64_t G, int64_t WPB) {
+  return cdiv(cdiv(cdiv(nnz, C) * S, G), WPB);
+}
+
+gnn_status_t make_info(int64_t nnz, int32_t K, const gnn_plan_opts_t *opts,
+                       gnn_plan_info_t *info) {
+  gnn_plan_opts_t o{};
+  if (opts) o = *opts;
+  const int32_t alpha = o.alpha ? o.alpha : 2;
+  const int32_t wpb = o.warps_per_block ? o.warps_per_block : 8;
+  if (nnz < 0 || nnz >= (int64_t(1) << 31) || K < 1 || alpha < 1 || wpb < 1 ||
+      wpb * 32 > kMaxThreads || o.force_chunk < 0 || o.deterministic != 0)
+    return fail(GNN_ERR_INVALID_ARG,
+                "plan: bad arguments (nnz=%lld K=%d alpha=%d wpb=%d force_chunk=%d det=%d)",
+                (long long)nnz, K, alpha, wpb, o.force_chunk, o.deterministic);
+  // step 1: feature vector width from K alone (or forced)
+  int32_t vw;
+  if (o.force_vw) {
+    if (!(o.force_vw == 1 || o.force_vw == 2 || o.force_vw == 4 || o.force_vw == 8) ||
+        K % o.force_vw)
+      return fail(GNN_ERR_INVALID_ARG, "plan: force_vw=%d invalid for K=%d", o.force_vw, K);
+    vw = o.force_vw;
+  } else if (K % 8 == 0 && K >= 256) {
+    vw = 8;
+  } else if (K % 4 == 0) {
+    vw = 4;
+  } else if (K % 2 == 0) {
+    vw = 2;
+  } else {
+    vw = 1;
+  }
+  // step 2: lanes per chunk-slice, slices, chunk-slices per warp
+  const int64_t need = cdiv(K, vw);
+  int32_t L = 1;
+  while (L < need && L < 32) L *= 2;
+  const int32_t S = (int32_t)cdiv(K, (int64_t)L * vw);
+  const int32_t G = 32 / L;
+  // step 3: FullWaveSize (Eqs. 3-4) from the occupancy of the SpMM kernel
+  DeviceInfo d;
+  if (gnn_status_t st = device_info(&d)) return st;
+  const int32_t abs = spmm_active_blocks_per_sm(vw, L, wpb);
+  if (abs < 1) return fail(GNN_ERR_CUDA, "plan: occupancy query failed (vw=%d L=%d)", vw, L);
+  const int64_t FW = (int64_t)d.num_sms * abs;
+  // steps 4-5: the largest candidate satisfying InEq. (5); none -> 8
+  int32_t C = 8;
+  for (int32_t c : kCand)
+    if (blocks_for(nnz, c, S, G, wpb) >= alpha * FW) C = c;
+  if (o.force_chunk > 0) C = o.force_chunk;
+  // step 6: sparse vector width (HVMA)
+  int32_t vws = 1;
+  if (C >= 128 && C % 4 == 0) vws = 4;
+  else if (C >= 64 && C % 2 == 0) vws = 2;
+  // step 7
+  info->chunk = C;
+  info->vw_feat = vw;
+  info->vw_sparse = vws;
+  info->lanes = L;
+  info->slices = S;
+  info->groups = G;
+  info->warps_per_block = wpb;
+  info->active_blocks_per_sm = abs;
+  info->num_sms = d.num_sms;
+  info->alpha = alpha;
+  info->K = K;
+  info->nnz = nnz;
+  info->num_chunks = nnz > 0 ? cdiv(nnz, C) : 0;
+  info->num_blocks = nnz > 0 ? blocks_for(nnz, C, S, G, wpb) : 0;
+  return GNN_OK;
+}
+
+size_t ws_bytes_for(int64_t nch) {
+  if (nch == 0) return 0;
+  return 2 * align256(sizeof(int32_t) * nch) + align256(nch);
+}
+
+// One thread per chunk: Algo 3 lines 2-3 (warp_start = id * NnzPerWarp, end
+// clamped to NNZ) and the node-boundary flags of the hybrid strategy.
+__global__ void plan_kernel(const int32_t *__restrict__ row_ind, int64_t nnz, int32_t C,
+                            int64_t nch, int32_t *__restrict__ row_first,
+                            int32_t *__restrict__ row_last, uint8_t *__restrict__ flags) {
+  const int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= nch) return;
+  const int64_t s = c * C;
+  const int64_t e = s + C < nnz ? s + C : nnz;
+  const int32_t rf = row_ind[s], rl = row_ind[e - 1];
+  uint8_t f = 0;
+  if (s > 0 && row_ind[s - 1] == rf) f |= 1;
+  if (e < nnz && row_ind[e] == rl) f |= 2;
+  row_first[c] = rf;
+  row_last[c] = rl;
+  flags[c] = f;
+}
+
+}  // namespace
+}  // namespace gnn
+
+using namespace gnn;
+
+extern "C" {
+
+GNN_API size_t gnn_plan_workspace_bytes(int64_t nnz, int32_t K, const gnn_plan_opts_t *opts) {
+  gnn_plan_info_t info;
+  if (make_info(nnz, K, opts, &info) != GNN_OK) return (size_t)-1;
+  return ws_bytes_for(info.num_chunks);
+}
+
+GNN_API gnn_status_t gnn_plan_create(const gnn_graph_t *g, int32_t K,
+                                     const gnn_plan_opts_t *opts, void *workspace,
+                                     size_t ws_bytes, gnn_stream_t stream, gnn_plan_t *out) {
+  if (!out) return fail(GNN_ERR_INVALID_ARG, "gnn_plan_create: out is NULL");
+  *out = nullptr;
+  if (!g || g->M < 0 || g->N < 0 || g->nnz < 0 || g->row_base < 0 ||
+      (g->nnz > 0 && (!g->row_ind || !g->col_ind)))
+    return fail(GNN_ERR_INVALID_ARG, "gnn_plan_create: bad graph descriptor");
+  gnn_plan_info_t info;
+  if (gnn_status_t st = make_info(g->nnz, K, opts, &info)) return st;
+  const int64_t nch = info.num_chunks;
+  const size_t need = ws_bytes_for(nch);
+  if (ws_bytes < need || (need > 0 && (!workspace || !aligned(workspace, 256))))
+    return fail(GNN_ERR_WORKSPACE, "gnn_plan_create: workspace %zu B (need %zu B, 256-B aligned)",
+                ws_bytes, need);
+  Plan *p = new (std::nothrow) Plan();
+  if (!p) return fail(GNN_ERR_INVALID_ARG, "gnn_plan_create: out of host memory");
+  p->info = info;
+  p->row_ind = g->row_ind;
+  p->M = g->M;
+  p->row_base = g->row_base;
+  char *w = (char *)workspace;
+  p->row_first = (int32_t *)w;
+  p->row_last = (int32_t *)(w + align256(sizeof(int32_t) * nch));
+  p->flags = (uint8_t *)(w + 2 * align256(sizeof(int32_t) * nch));
+  DeviceInfo d;
+  device_info(&d);
+  p->device = d.device;
+  if (nch > 0) {
+    const int threads = 256;
+    plan_kernel<<<(unsigned)cdiv(nch, threads), threads, 0, (cudaStream_t)stream>>>(
+        g->row_ind, g->nnz, info.chunk, nch, p->row_first, p->row_last, p->flags);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) {
+      delete p;
+      return cuda_fail(e, "plan kernel launch");
+    }
+  }
+  *out = reinterpret_cast<gnn_plan_t>(p);
+  return GNN_OK;
+}
+
+GNN_API gnn_status_t gnn_plan_info(gnn_plan_t plan, gnn_plan_info_t *info) {
+  if (!plan || !info) return fail(GNN_ERR_INVALID_ARG, "gnn_plan_info: NULL argument");
+  *info = reinterpret_cast<Plan *>(plan)->info;
+  return GNN_OK;
+}
+
+GNN_API gnn_status_t gnn_plan_arrays(gnn_plan_t plan, const int32_t **row_first,
+                                     const int32_t **row_last, const uint8_t **flags) {
+  if (!plan) return fail(GNN_ERR_INVALID_ARG, "gnn_plan_arrays: NULL plan");
+  Plan *p = reinterpret_cast<Plan *>(plan);
+  if (row_first) *row_first = p->row_first;
+  if (row_last) *row_last = p->row_last;
+  if (flags) *flags = p->flags;
+  return GNN_OK;
+}
+
+GNN_API void gnn_plan_destroy(gnn_plan_t plan) { delete reinterpret_cast<Plan *>(plan); }
+
+}  // extern "C"

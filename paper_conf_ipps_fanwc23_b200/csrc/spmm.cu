@@ -1,0 +1,293 @@
+// spmm.cu -- hybrid-parallel SpMM for sm_100a (O = S A; Algorithm 1
+// is the definition, Algorithm 3 P:168-195 the prior-art GPU design).
+//
+// Work decomposition: the plan cuts the nnz into chunks of C*
+// consecutive nonzeros (equal work per unit, hybrid node/edge parallelism).
+// Each (chunk, K-slice) work item is owned by a lane group of L lanes; every lane
+// holds VW consecutive feature columns, so one group gathers L*VW columns of a
+// source row per nonzero with one vector load per lane (128-bit, or 256-bit at
+// VW = 8).  G = 32/L groups share a warp.  Per tile of T = L*vw_sparse nonzeros the
+// group loads (row, col, val) coalesced and vectorised, then broadcasts them
+// nonzero by nonzero with width-L shuffles; U feature rows are in flight per lane
+// before the FMAs consume them.  A row switch ("row-switch procedure")
+// flushes the accumulator: rows wholly inside the chunk get a plain vector store,
+// rows shared with a neighbouring chunk (plan flags) a vector atomic add into a row
+// zeroed beforehand by spmm_prezero_kernel.  Empty rows are written as zeros by the
+// chunk that precedes them, so O is fully overwritten without a memset.
+#include <climits>
+
+#include "device.cuh"
+#include "internal.cuh"
+
+namespace gnn {
+
+template <int VW>
+struct FeatDepth {
+  static constexpr int value = VW == 8 ? 4 : 8;  // feature rows in flight per lane
+};
+
+template <int VW, int L, int VWS>
+struct TileCfg {
+  static constexpr int G = 32 / L;
+  static constexpr int T = L * VWS;  // nonzeros per tile per group
+  static constexpr int U = FeatDepth<VW>::value < T ? FeatDepth<VW>::value : T;
+  static_assert(T % U == 0 && U % VWS == 0, "tile / prefetch shape");
+};
+
+template <int VW, int L, int VWS>
+__global__ void __launch_bounds__(kMaxThreads)
+    spmm_kernel(const SparseArgs a, const float *__restrict__ A, const int64_t lda,
+                float *__restrict__ O, const int64_t ldo) {
+  using Cfg = TileCfg<VW, L, VWS>;
+  constexpr int G = Cfg::G, T = Cfg::T, U = Cfg::U;
+  const int lane = threadIdx.x & 31;
+  const int g = lane / L;
+  const int l = lane & (L - 1);
+  const int64_t item = ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * G + g;
+  const bool item_ok = item < a.num_chunks * a.slices;
+  if (!__any_sync(kFull, item_ok)) return;  // warp-uniform exit
+
+  int64_t c = 0;
+  int s = 0;
+  if (item_ok) {
+    c = item / a.slices;
+    s = (int)(item - c * a.slices);
+  }
+  const int k0 = (s * L + l) * VW;
+  const bool col_ok = item_ok && k0 < a.K;
+  const int64_t cs = c * a.chunk;
+  const int64_t ce = item_ok ? min(cs + (int64_t)a.chunk, a.nnz) : cs;
+  int32_t rf = 0, rl = 0;
+  uint32_t fl = 0;
+  if (item_ok) {
+    rf = a.row_first[c];
+    rl = a.row_last[c];
+    fl = a.flags[c];
+  }
+  const float *__restrict__ Ak = A + k0;
+  float *__restrict__ Ok = O + k0;  // row r at Ok + (r - row_base) * ldo
+
+  // empty rows between the previous chunk's last row and ours are ours to zero
+  if (col_ok) {
+    const int64_t prev = (c == 0) ? a.row_base - 1 : (int64_t)a.row_last[c - 1];
+    for (int64_t r = prev + 1; r < rf; ++r) st_zero<VW>(Ok + (r - a.row_base) * ldo);
+  }
+
+  float acc[VW];
+#pragma unroll
+  for (int v = 0; v < VW; ++v) acc[v] = 0.f;
+  int32_t cur = -1;
+
+  const int ntiles = (a.chunk + T - 1) / T;  // warp-uniform trip count
+  for (int t = 0; t < ntiles; ++t) {
+    const int64_t tb = cs + (int64_t)t * T;
+    const int64_t li = tb + (int64_t)l * VWS;
+    int32_t rr[VWS], cc[VWS];
+    float vv[VWS];
+    ld_sparse_i32<VWS>(a.row_ind, li, ce, 0, rr);
+    ld_sparse_i32<VWS>(a.col_ind, li, ce, 0, cc);
+    ld_sparse_f32<VWS>(a.val, li, ce, vv);
+#pragma unroll 1
+    for (int jj = 0; jj < T; jj += U) {
+      int32_t rj[U], cj[U];
+      float vj[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const int src = (jj + u) / VWS;
+        rj[u] = __shfl_sync(kFull, rr[u % VWS], src, L);
+        cj[u] = __shfl_sync(kFull, cc[u % VWS], src, L);
+        vj[u] = __shfl_sync(kFull, vv[u % VWS], src, L);
+      }
+      float x[U][VW];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        if (col_ok && tb + jj + u < ce) {
+          ld_feat<VW>(Ak + (int64_t)cj[u] * lda, x[u]);
+        } else {
+#pragma unroll
+          for (int v = 0; v < VW; ++v) x[u][v] = 0.f;
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        if (tb + jj + u < ce) {
+          if (rj[u] != cur) {  // row-switch procedure
+            if (cur >= 0 && col_ok) {
+              float *o = Ok + ((int64_t)cur - a.row_base) * ldo;
+              const bool shared = (cur == rf && (fl & 1u)) || (cur == rl && (fl & 2u));
+              if (shared) red_add<VW>(o, acc);
+              else st_vec<VW>(o, acc);
+              for (int64_t r = (int64_t)cur + 1; r < rj[u]; ++r)
+                st_zero<VW>(Ok + (r - a.row_base) * ldo);
+            }
+            cur = rj[u];
+#pragma unroll
+            for (int v = 0; v < VW; ++v) acc[v] = 0.f;
+          }
+#pragma unroll
+          for (int v = 0; v < VW; ++v) acc[v] = fmaf(vj[u], x[u][v], acc[v]);
+        }
+      }
+    }
+  }
+  if (cur >= 0 && col_ok) {
+    float *o = Ok + ((int64_t)cur - a.row_base) * ldo;
+    const bool shared = (cur == rf && (fl & 1u)) || (cur == rl && (fl & 2u));
+    if (shared) red_add<VW>(o, acc);
+    else st_vec<VW>(o, acc);
+  }
+  // trailing empty rows after the last chunk
+  if (col_ok && c == a.num_chunks - 1) {
+    for (int64_t r = (int64_t)rl + 1; r < a.row_base + a.M; ++r)
+      st_zero<VW>(Ok + (r - a.row_base) * ldo);
+  }
+}
+
+// Zero every row shared by several chunks before the atomics land on it: the row
+// is zeroed by the chunk in which it starts (tail flag set, and not a pure
+// continuation of an earlier chunk's row).  One warp per chunk.
+template <int VW>
+__global__ void spmm_prezero_kernel(const SparseArgs a, float *__restrict__ O,
+                                    const int64_t ldo) {
+  const int64_t c = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  if (c >= a.num_chunks) return;
+  const uint32_t fl = a.flags[c];
+  if (!(fl & 2u)) return;
+  const int32_t rf = a.row_first[c], rl = a.row_last[c];
+  if ((fl & 1u) && rf == rl) return;
+  float *o = O + ((int64_t)rl - a.row_base) * ldo;
+  for (int k = lane * VW; k < a.K; k += 32 * VW) st_zero<VW>(o + k);
+}
+
+// ------------------------------------------------------------ dispatch ----
+using SpmmFn = void (*)(const SparseArgs, const float *__restrict__, const int64_t,
+                        float *__restrict__, const int64_t);
+
+template <int VW, int L>
+SpmmFn pick_vws(int vws) {
+  switch (vws) {
+    case 1: return spmm_kernel<VW, L, 1>;
+    case 2: return spmm_kernel<VW, L, 2>;
+    case 4: return spmm_kernel<VW, L, 4>;
+  }
+  return nullptr;
+}
+template <int VW>
+SpmmFn pick_l(int L, int vws) {
+  switch (L) {
+    case 1: return pick_vws<VW, 1>(vws);
+    case 2: return pick_vws<VW, 2>(vws);
+    case 4: return pick_vws<VW, 4>(vws);
+    case 8: return pick_vws<VW, 8>(vws);
+    case 16: return pick_vws<VW, 16>(vws);
+    case 32: return pick_vws<VW, 32>(vws);
+  }
+  return nullptr;
+}
+SpmmFn pick_spmm(int vw, int L, int vws) {
+  switch (vw) {
+    case 1: return pick_l<1>(L, vws);
+    case 2: return pick_l<2>(L, vws);
+    case 4: return pick_l<4>(L, vws);
+    case 8: return pick_l<8>(L, vws);
+  }
+  return nullptr;
+}
+
+int spmm_active_blocks_per_sm(int vw, int lanes, int wpb) {
+  SpmmFn f = pick_spmm(vw, lanes, 1);
+  if (!f) return 0;
+  int n = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, f, wpb * 32, 0) != cudaSuccess) return 0;
+  return n;
+}
+
+// Common argument checks for gnn_spmm / gnn_sddmm.
+gnn_status_t check_common(const Plan *p, const gnn_graph_t *g, const char *who) {
+  if (!p || !g) return fail(GNN_ERR_INVALID_ARG, "%s: NULL plan or graph", who);
+  if (g->nnz != p->info.nnz || g->row_ind != p->row_ind || g->M != p->M ||
+      g->row_base != p->row_base)
+    return fail(GNN_ERR_INVALID_ARG, "%s: graph does not match the plan", who);
+  if (g->nnz > 0 && (!g->row_ind || !g->col_ind))
+    return fail(GNN_ERR_INVALID_ARG, "%s: NULL sparse arrays", who);
+  int dev = -1;
+  cudaGetDevice(&dev);
+  if (dev != p->device)
+    return fail(GNN_ERR_INVALID_ARG, "%s: plan built for device %d, current %d", who, p->device,
+                dev);
+  return GNN_OK;
+}
+
+// Sparse vector width actually usable for these pointers (HVMA needs aligned bases).
+int effective_vws(int vws, const gnn_graph_t *g, const void *extra) {
+  while (vws > 1) {
+    const size_t al = 4u * vws;
+    if (aligned(g->row_ind, al) && aligned(g->col_ind, al) && (!g->val || aligned(g->val, al)) &&
+        (!extra || aligned(extra, al)))
+      break;
+    vws >>= 1;
+  }
+  return vws;
+}
+
+SparseArgs make_args(const Plan *p, const gnn_graph_t *g) {
+  SparseArgs a;
+  a.row_ind = g->row_ind;
+  a.col_ind = g->col_ind;
+  a.val = g->val;
+  a.row_first = p->row_first;
+  a.row_last = p->row_last;
+  a.flags = p->flags;
+  a.nnz = g->nnz;
+  a.num_chunks = p->info.num_chunks;
+  a.row_base = g->row_base;
+  a.M = g->M;
+  a.chunk = p->info.chunk;
+  a.K = p->info.K;
+  a.slices = p->info.slices;
+  return a;
+}
+
+}  // namespace gnn
+
+using namespace gnn;
+
+extern "C" GNN_API gnn_status_t gnn_spmm(gnn_plan_t plan, const gnn_graph_t *g, const float *A,
+                                         int64_t lda, float *O, int64_t ldo,
+                                         gnn_stream_t stream) {
+  const Plan *p = reinterpret_cast<const Plan *>(plan);
+  if (gnn_status_t st = check_common(p, g, "gnn_spmm")) return st;
+  const gnn_plan_info_t &in = p->info;
+  const int K = in.K, VW = in.vw_feat;
+  if (g->M == 0) return GNN_OK;
+  if (!O || ldo < K || (g->nnz > 0 && (!A || lda < K)))
+    return fail(GNN_ERR_INVALID_ARG, "gnn_spmm: bad dense operand (lda=%lld ldo=%lld K=%d)",
+                (long long)lda, (long long)ldo, K);
+  if (!aligned(O, 4u * VW) || ldo % VW || (g->nnz > 0 && (!aligned(A, 4u * VW) || lda % VW)))
+    return fail(GNN_ERR_UNSUPPORTED,
+                "gnn_spmm: A/O must be %d-byte aligned with pitches multiple of %d "
+                "(re-plan with force_vw)", 4 * VW, VW);
+  cudaStream_t s = (cudaStream_t)stream;
+  if (g->nnz == 0) {  // no chunks: O := 0
+    cudaError_t e = cudaMemset2DAsync(O, ldo * sizeof(float), 0, K * sizeof(float), g->M, s);
+    return e == cudaSuccess ? GNN_OK : cuda_fail(e, "gnn_spmm memset");
+  }
+  const int vws = effective_vws(in.vw_sparse, g, nullptr);
+  SpmmFn f = pick_spmm(VW, in.lanes, vws);
+  if (!f) return fail(GNN_ERR_UNSUPPORTED, "gnn_spmm: no kernel for vw=%d L=%d", VW, in.lanes);
+  const SparseArgs a = make_args(p, g);
+  const int threads = in.warps_per_block * 32;
+  {
+    const int64_t blocks = (a.num_chunks * 32 + 255) / 256;
+    switch (VW) {
+      case 1: spmm_prezero_kernel<1><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo); break;
+      case 2: spmm_prezero_kernel<2><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo); break;
+      case 4: spmm_prezero_kernel<4><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo); break;
+      default: spmm_prezero_kernel<8><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo); break;
+    }
+  }
+  f<<<(unsigned)in.num_blocks, threads, 0, s>>>(a, A, lda, O, ldo);
+  cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? GNN_OK : cuda_fail(e, "gnn_spmm launch");
+}

@@ -1,0 +1,171 @@
+// util.cu -- errors, device info, shards, CSR->COO, validation (C ABI).
+#include <cuda_runtime.h>
+#include <stdarg.h>
+#include <stdio.h>
+#include <string.h>
+
+#include <mutex>
+
+#include "internal.cuh"
+
+namespace gnn {
+
+static thread_local char g_err[512] = "";
+
+gnn_status_t fail(gnn_status_t st, const char *fmt, ...) {
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(g_err, sizeof(g_err), fmt, ap);
+  va_end(ap);
+  return st;
+}
+
+gnn_status_t cuda_fail(cudaError_t e, const char *what) {
+  return fail(GNN_ERR_CUDA, "%s: %s (%s)", what, cudaGetErrorName(e), cudaGetErrorString(e));
+}
+
+void clear_error() { g_err[0] = '\0'; }
+
+gnn_status_t device_info(DeviceInfo *out) {
+  static std::mutex mu;
+  static DeviceInfo cache[64];
+  static bool have[64] = {false};
+  int dev = -1;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice (no usable CUDA device)");
+  if (dev < 0 || dev >= 64) return fail(GNN_ERR_CUDA, "device ordinal %d out of range", dev);
+  std::lock_guard<std::mutex> lk(mu);
+  if (!have[dev]) {
+    DeviceInfo d{};
+    d.device = dev;
+    if ((e = cudaDeviceGetAttribute(&d.num_sms, cudaDevAttrMultiProcessorCount, dev)) !=
+        cudaSuccess)
+      return cuda_fail(e, "cudaDeviceGetAttribute(SM count)");
+    cudaDeviceGetAttribute(&d.cc_major, cudaDevAttrComputeCapabilityMajor, dev);
+    cudaDeviceGetAttribute(&d.cc_minor, cudaDevAttrComputeCapabilityMinor, dev);
+    if (d.cc_major != 10 || d.cc_minor != 0)
+      return fail(GNN_ERR_CUDA, "device %d is sm_%d%d; this library is built for sm_100a only",
+                  dev, d.cc_major, d.cc_minor);
+    cache[dev] = d;
+    have[dev] = true;
+  }
+  *out = cache[dev];
+  return GNN_OK;
+}
+
+// ------------------------------------------------------------- kernels ----
+__global__ void csr_to_coo_kernel(const int32_t *__restrict__ row_ptr, int64_t M,
+                                  int64_t row_base, int32_t *__restrict__ row_ind) {
+  // one warp per row: coalesced writes of the row's run
+  const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const int64_t base = row_ptr[0];
+  for (int64_t r = warp; r < M; r += nwarps) {
+    const int64_t b = row_ptr[r] - base, e = row_ptr[r + 1] - base;
+    for (int64_t i = b + lane; i < e; i += 32) row_ind[i] = (int32_t)(r + row_base);
+  }
+}
+
+// err[0]: first offending nnz index (or -1), err[1]: kind
+__global__ void validate_kernel(gnn_graph_t g, unsigned long long *bad) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  const int64_t base = g.row_ptr ? g.row_ptr[0] : 0;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < g.nnz; i += stride) {
+    const int64_t r = g.row_ind[i], c = g.col_ind[i];
+    unsigned long long kind = 0;
+    if (r < g.row_base || r >= g.row_base + g.M) kind = 1;
+    else if (c < 0 || c >= g.N) kind = 2;
+    else if (i > 0 && g.row_ind[i - 1] > r) kind = 3;
+    else if (g.row_ptr && !((int64_t)g.row_ptr[r - g.row_base] - base <= i &&
+                            i < (int64_t)g.row_ptr[r - g.row_base + 1] - base))
+      kind = 4;
+    if (kind) atomicMin(bad, ((unsigned long long)i << 3) | kind);
+  }
+}
+
+}  // namespace gnn
+
+using namespace gnn;
+
+extern "C" {
+
+GNN_API const char *gnn_last_error(void) { return g_err; }
+
+GNN_API const char *gnn_version(void) { return "gnnsparse 0.1 (sm_100a)"; }
+
+GNN_API gnn_status_t gnn_shard_rows(const int32_t *row_ptr_host, int64_t M, int32_t P,
+                                    int64_t *bounds) {
+  if (!row_ptr_host || M < 0 || P < 1 || !bounds)
+    return fail(GNN_ERR_INVALID_ARG, "gnn_shard_rows: bad arguments");
+  const int64_t base = row_ptr_host[0];
+  const int64_t nnz = (int64_t)row_ptr_host[M] - base;
+  bounds[0] = 0;
+  for (int32_t p = 1; p < P; ++p) {
+    const int64_t t = (int64_t)p * nnz / P;
+    // lower_bound over r in [0, M] of row_ptr[r] - base >= t
+    int64_t lo = 0, n = M + 1;
+    while (n > 0) {
+      const int64_t half = n / 2;
+      if ((int64_t)row_ptr_host[lo + half] - base < t) {
+        lo += half + 1;
+        n -= half + 1;
+      } else {
+        n = half;
+      }
+    }
+    bounds[p] = lo > bounds[p - 1] ? lo : bounds[p - 1];
+  }
+  bounds[P] = M;
+  return GNN_OK;
+}
+
+GNN_API gnn_status_t gnn_shard_edges(int64_t nnz, int32_t P, int64_t *bounds) {
+  if (nnz < 0 || P < 1 || !bounds) return fail(GNN_ERR_INVALID_ARG, "gnn_shard_edges: bad arguments");
+  for (int32_t p = 0; p <= P; ++p) bounds[p] = (int64_t)((__int128)p * nnz / P);
+  return GNN_OK;
+}
+
+GNN_API gnn_status_t gnn_csr_to_coo(const int32_t *row_ptr, int64_t M, int64_t row_base,
+                                    int32_t *row_ind, gnn_stream_t stream) {
+  if (M < 0 || (M > 0 && (!row_ptr || !row_ind)))
+    return fail(GNN_ERR_INVALID_ARG, "gnn_csr_to_coo: bad arguments");
+  if (M == 0) return GNN_OK;
+  DeviceInfo d;
+  if (gnn_status_t st = device_info(&d)) return st;
+  const int threads = 256;
+  int64_t blocks = (M * 32 + threads - 1) / threads;
+  const int64_t cap = (int64_t)d.num_sms * 16;
+  if (blocks > cap) blocks = cap;
+  csr_to_coo_kernel<<<(unsigned)blocks, threads, 0, (cudaStream_t)stream>>>(row_ptr, M, row_base,
+                                                                           row_ind);
+  cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? GNN_OK : cuda_fail(e, "csr_to_coo launch");
+}
+
+GNN_API gnn_status_t gnn_validate(const gnn_graph_t *g, gnn_stream_t stream) {
+  if (!g || g->M < 0 || g->N < 0 || g->nnz < 0 ||
+      (g->nnz > 0 && (!g->row_ind || !g->col_ind)))
+    return fail(GNN_ERR_INVALID_ARG, "gnn_validate: bad graph descriptor");
+  if (g->nnz == 0) return GNN_OK;
+  DeviceInfo d;
+  if (gnn_status_t st = device_info(&d)) return st;
+  cudaStream_t s = (cudaStream_t)stream;
+  unsigned long long *bad = nullptr, h = ~0ull;
+  cudaError_t e = cudaMallocAsync((void **)&bad, sizeof(*bad), s);
+  if (e != cudaSuccess) return cuda_fail(e, "gnn_validate alloc");
+  cudaMemcpyAsync(bad, &h, sizeof(h), cudaMemcpyHostToDevice, s);
+  validate_kernel<<<d.num_sms * 8, 256, 0, s>>>(*g, bad);
+  cudaMemcpyAsync(&h, bad, sizeof(h), cudaMemcpyDeviceToHost, s);
+  cudaFreeAsync(bad, s);
+  e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) return cuda_fail(e, "gnn_validate");
+  if (h == ~0ull) return GNN_OK;
+  static const char *kinds[] = {"", "row_ind out of [row_base, row_base+M)",
+                                "col_ind out of [0, N)", "row_ind decreasing",
+                                "row_ptr inconsistent with row_ind"};
+  return fail(GNN_ERR_INPUT_CHECK, "gnn_validate: nnz %lld: %s", (long long)(h >> 3),
+              kinds[h & 7]);
+}
+
+}  // extern "C"

@@ -1,0 +1,322 @@
+"""GPU parity: the CUDA path (through the C ABI) against the fp64 CPU oracle.
+
+Bars (BASELINE.json north_star): plan arrays/info bit-exact; fp32 outputs within
+|err| <= 1e-5 * sum|terms| elementwise (tests/helpers.assert_within); exact where
+the mathematics makes the result exact (one-term sums, integer sums, symmetric pairs,
+sharded SDDMM vs unsharded).
+"""
+import numpy as np
+import pytest
+import torch
+
+import gen
+import oracle
+from gen import configs
+import paper_conf_ipps_fanwc23_b200 as gs
+
+from helpers import assert_within, upload
+
+pytestmark = pytest.mark.gpu
+
+DEV = "cuda"
+
+
+def _x(seed, rows, K, ld=None):
+    X = gen.features(seed, rows, K, ld=ld)
+    return X
+
+
+def check_plan(p, g, K, **kw):
+    info = p.info()
+    ref = oracle.plan(g.row_ind, K, info["num_sms"], info["active_blocks_per_sm"],
+                      alpha=kw.get("alpha", 2) or 2,
+                      warps_per_block=kw.get("warps_per_block", 8) or 8,
+                      force_chunk=kw.get("force_chunk", 0), force_vw=kw.get("force_vw", 0))
+    assert info == ref.info, (info, ref.info)
+    rf, rl, fl = (t.cpu().numpy() for t in p.arrays())
+    assert np.array_equal(rf, ref.row_first)
+    assert np.array_equal(rl, ref.row_last)
+    assert np.array_equal(fl, ref.flags)
+    return info
+
+
+def run_full(g, K, seed=7, check_sddmm=True, with_val=True, ld_pad=0, **kw):
+    """Plan + SpMM + SDDMM on the whole graph, compared with the oracle everywhere."""
+    dg = upload(g, with_val=with_val)
+    p = gs.plan(dg, K, **kw)
+    info = check_plan(p, g, K, **kw)
+    ld = K + ld_pad
+    A = _x(seed, g.N, K, ld=ld)
+    At = torch.from_numpy(A).to(DEV)[:, :K] if ld_pad else torch.from_numpy(A).to(DEV)
+    O = torch.full((g.M, ld), float("nan"), device=DEV)[:, :K] if ld_pad else \
+        torch.full((g.M, K), float("nan"), device=DEV)
+    gs.spmm(p, dg, At, out=O)
+    torch.cuda.synchronize()
+    val = g.val if with_val else None
+    ref, T = oracle.spmm(g.row_ind, g.col_ind, val, np.ascontiguousarray(A[:, :K]), M=g.M)
+    worst = assert_within(O.cpu().numpy(), ref, T, what=f"spmm K={K}")
+    if check_sddmm:
+        A1 = _x(seed + 1, g.M, K)
+        out = gs.sddmm(p, dg, torch.from_numpy(A1).to(DEV), At)
+        torch.cuda.synchronize()
+        r2, T2 = oracle.sddmm(g.row_ind, g.col_ind, val, A1, np.ascontiguousarray(A[:, :K]))
+        assert_within(out.cpu().numpy(), r2, T2, what=f"sddmm K={K}")
+    return info, worst
+
+
+# ------------------------------------------------------- BJ small configs ---
+def test_c1_tiny_powerlaw_k32():
+    g = configs.make_graph("C1")
+    info, _ = run_full(g, 32)
+    assert info["chunk"] == 8  # Eq. 5 infeasible on 148 SMs -> most parallel candidate
+
+
+def test_c2_cora_shaped_k64():
+    g = configs.make_graph("C2")
+    run_full(g, 64)
+
+
+@pytest.mark.parametrize("t", [0, 1, 2])
+def test_c3_sampled_subgraph_k128(t):
+    run_full(configs.make_c3(t), 128)
+
+
+# ------------------------------------------------------ shapes / edge cases --
+@pytest.mark.parametrize("K", [1, 2, 3, 4, 6, 8, 16, 24, 32, 33, 64, 100, 128, 256, 300, 512])
+def test_feature_widths(K):
+    g = gen.powerlaw_graph(3000, 60000, gamma=2.3, n_comm=6, seed=K)
+    run_full(g, K, check_sddmm=K <= 1024)
+
+
+@pytest.mark.parametrize("C", [1, 2, 5, 8, 32, 64, 128, 256, 512, 1000])
+def test_forced_chunk_sizes(C):
+    g = gen.powerlaw_graph(2000, 50000, gamma=2.1, n_comm=4, seed=100 + C)
+    run_full(g, 32, force_chunk=C)
+    run_full(g, 256, force_chunk=C)
+
+
+@pytest.mark.parametrize("vw", [1, 2, 4, 8])
+def test_forced_vector_width(vw):
+    g = gen.powerlaw_graph(2000, 30000, seed=200 + vw)
+    run_full(g, 64, force_vw=vw)
+
+
+@pytest.mark.parametrize("wpb,alpha", [(1, 1), (4, 2), (16, 8)])
+def test_block_shape_and_alpha(wpb, alpha):
+    g = gen.powerlaw_graph(5000, 200000, seed=300 + wpb)
+    run_full(g, 64, warps_per_block=wpb, alpha=alpha)
+
+
+def test_val_none_and_padded_pitch():
+    g = gen.powerlaw_graph(3000, 40000, seed=301)
+    run_full(g, 64, with_val=False)
+    run_full(g, 64, ld_pad=12)
+
+
+def test_empty_rows_rectangular_duplicates():
+    rng = np.random.default_rng(5)
+    M, N, nnz = 777, 333, 9000
+    rows = rng.integers(0, M, nnz)
+    rows = rows[(rows % 7) != 3]  # many empty rows, incl. runs
+    rows = np.concatenate([rows, np.full(3000, 500)])  # one heavy row
+    cols = rng.integers(0, N, rows.size)
+    cols[:20] = cols[0]
+    rows[:20] = rows[0]  # duplicates
+    vals = rng.uniform(0.1, 1, rows.size).astype(np.float32)
+    g = gen.from_coo(M, N, rows, cols, vals)
+    for C in (0, 5, 8, 64, 512):
+        run_full(g, 32, force_chunk=C)
+        run_full(g, 12, force_chunk=C)
+
+
+def test_leading_and_trailing_empty_rows():
+    g = gen.from_coo(50, 10, [10, 10, 11, 30, 30, 30], [1, 2, 3, 4, 5, 6])
+    for C in (0, 1, 2, 4):
+        run_full(g, 8, force_chunk=C)
+
+
+def test_single_hub_row_spans_many_chunks():
+    N = 20000
+    g = gen.from_coo(3, N, np.r_[np.zeros(5), np.ones(N), np.full(5, 2)],
+                     np.r_[np.arange(5), np.arange(N), np.arange(5)],
+                     gen.uniform_values(9, N + 10))
+    for C in (0, 8, 64, 512):
+        run_full(g, 128, force_chunk=C)
+
+
+def test_empty_graph_overwrites_output():
+    g = gen.from_coo(40, 10, [], [])
+    dg = upload(g)
+    p = gs.plan(dg, 16)
+    assert p.info()["num_chunks"] == 0
+    O = torch.full((40, 16), 7.0, device=DEV)
+    gs.spmm(p, dg, torch.zeros((10, 16), device=DEV), out=O)
+    out = gs.sddmm(p, dg, torch.zeros((40, 16), device=DEV), torch.zeros((10, 16), device=DEV))
+    torch.cuda.synchronize()
+    assert (O == 0).all() and out.numel() == 0
+
+
+def test_zero_rows_graph():
+    g = gen.from_coo(0, 10, [], [])
+    dg = upload(g)
+    p = gs.plan(dg, 8)
+    gs.spmm(p, dg, torch.zeros((10, 8), device=DEV), out=torch.empty((0, 8), device=DEV))
+
+
+# ------------------------------------------------------------ exact pins ---
+def test_identity_returns_A_bitwise():
+    N, K = 5000, 64
+    g = gen.from_coo(N, N, np.arange(N), np.arange(N))
+    A = torch.from_numpy(_x(1, N, K)).to(DEV)
+    dg = upload(g)
+    for C in (0, 1, 8, 512):
+        p = gs.plan(dg, K, force_chunk=C)
+        O = gs.spmm(p, dg, A)
+        torch.cuda.synchronize()
+        assert torch.equal(O, A)
+
+
+def test_ones_features_integer_sums_exact():
+    g = gen.powerlaw_graph(4000, 100000, seed=41)
+    g.val = np.random.default_rng(0).integers(1, 4, g.nnz).astype(np.float32)
+    dg = upload(g)
+    p = gs.plan(dg, 32)
+    O = gs.spmm(p, dg, torch.ones((g.N, 32), device=DEV)).cpu().numpy()
+    sums = np.bincount(g.row_ind, weights=g.val.astype(np.float64), minlength=g.M)
+    assert np.array_equal(O.astype(np.float64), np.repeat(sums[:, None], 32, 1))
+
+
+def test_sddmm_pair_symmetry_bitwise_and_self_loop_norm():
+    g = gen.powerlaw_graph(3000, 50000, seed=42, val_mode="ones")
+    dg = upload(g)
+    K = 128
+    X = torch.from_numpy(_x(42, g.N, K)).to(DEV)
+    p = gs.plan(dg, K)
+    out = gs.sddmm(p, dg, X, X).cpu().numpy()
+    key = g.row_ind.astype(np.int64) * g.N + g.col_ind
+    rkey = g.col_ind.astype(np.int64) * g.N + g.row_ind
+    pos = np.searchsorted(key, rkey)
+    assert np.array_equal(out, out[pos])  # (u,v) and (v,u) identical
+    self_ = g.row_ind == g.col_ind
+    Xn = X.cpu().numpy().astype(np.float64)
+    nrm = (Xn ** 2).sum(1)[g.row_ind[self_]]
+    assert np.allclose(out[self_], nrm, rtol=1e-5)
+
+
+def test_fig4_fig5_worked_example():
+    from test_oracle import fig4_matrix
+    g, C, K, w, entries = fig4_matrix()
+    dg = upload(g)
+    p = gs.plan(dg, K, force_chunk=C)
+    rf, rl, fl = (t.cpu().numpy() for t in p.arrays())
+    assert (rf[w], rl[w]) == (3, 4)
+    run_full(g, K, force_chunk=C)
+
+
+# --------------------------------------------------------------- shards ----
+@pytest.mark.parametrize("P", [2, 3, 8])
+def test_virtual_row_and_edge_shards(P):
+    """P shard plans run one after another on one GPU: row-sharded SpMM equals the
+    unsharded result within tolerance, and edge-sharded SDDMM equals it bitwise (each
+    output's dot product is computed in a fixed lane order whatever the chunking)."""
+    g = gen.powerlaw_graph(6000, 300000, gamma=2.2, n_comm=6, seed=60 + P)
+    K = 64
+    A = _x(61, g.N, K)
+    At = torch.from_numpy(A).to(DEV)
+    dg = upload(g)
+    ref, T = oracle.spmm(g.row_ind, g.col_ind, g.val, A, M=g.M)
+    rb = gs.shard_rows(g.row_ptr, P)
+    O = torch.empty((g.M, K), device=DEV)
+    for q in range(P):
+        r0, r1 = int(rb[q]), int(rb[q + 1])
+        e0, e1 = int(g.row_ptr[r0]), int(g.row_ptr[r1])
+        sh = dg.shard(r0, r1, e0, e1)
+        p = gs.plan(sh, K)
+        gs.spmm(p, sh, At, out=O[r0:r1])
+    torch.cuda.synchronize()
+    assert_within(O.cpu().numpy(), ref, T, what="row-sharded spmm")
+    # edge shards for SDDMM
+    full = gs.sddmm(gs.plan(dg, K), dg, At, At)
+    eb = gs.shard_edges(g.nnz, P)
+    out = torch.empty(g.nnz, device=DEV)
+    for q in range(P):
+        e0, e1 = int(eb[q]), int(eb[q + 1])
+        sh = gs.DeviceGraph(g.M, g.N, dg.row_ind[e0:e1], dg.col_ind[e0:e1], dg.val[e0:e1])
+        p = gs.plan(sh, K)
+        gs.sddmm(p, sh, At, At, out=out[e0:e1])
+    torch.cuda.synchronize()
+    assert torch.equal(out, full)  # each output's dot is chunking-independent
+
+
+def test_plan_spmm_sddmm_capture_in_cuda_graph():
+    """No host sync anywhere on the path: plan + SpMM + SDDMM capture into a CUDA graph."""
+    g = configs.make_c3(5)
+    dg = upload(g)
+    K = 128
+    X = torch.from_numpy(_x(5, g.N, K)).to(DEV)
+    O = torch.empty((g.M, K), device=DEV)
+    E = torch.empty(g.nnz, device=DEV)
+    nbytes = gs.lib().gnn_plan_workspace_bytes(g.nnz, K, None)
+    s = torch.cuda.Stream()
+    s.wait_stream(torch.cuda.current_stream())
+    holder = []
+    with torch.cuda.stream(s):
+        gs.plan(dg, K)  # warm-up (occupancy cache) outside capture
+        graph = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(graph, stream=s):
+            p = gs.plan(dg, K)
+            holder.append(p)
+            gs.spmm(p, dg, X, out=O)
+            gs.sddmm(p, dg, X, X, out=E)
+    graph.replay()
+    torch.cuda.synchronize()
+    ref, T = oracle.spmm(g.row_ind, g.col_ind, g.val, X.cpu().numpy(), M=g.M)
+    assert_within(O.cpu().numpy(), ref, T, what="graph-captured spmm")
+    assert nbytes > 0
+
+
+def test_misaligned_subview_falls_back_to_scalar_sparse_loads():
+    g = gen.powerlaw_graph(4000, 200000, seed=77)
+    dg = upload(g)
+    r0 = 1
+    e0 = int(g.row_ptr[r0])
+    assert e0 % 4 != 0
+    sh = dg.shard(r0, g.M, e0, g.nnz)
+    K = 32
+    A = _x(77, g.N, K)
+    p = gs.plan(sh, K)
+    assert p.info()["vw_sparse"] == 4
+    O = gs.spmm(p, sh, torch.from_numpy(A).to(DEV))
+    ref, T = oracle.spmm(g.row_ind, g.col_ind, g.val, A, i0=e0, i1=g.nnz, r0=r0, nrows=g.M - r0)
+    assert_within(O.cpu().numpy(), ref, T, what="misaligned shard")
+
+
+def test_unsupported_alignment_is_reported():
+    g = gen.powerlaw_graph(500, 5000, seed=78)
+    dg = upload(g)
+    p = gs.plan(dg, 32)
+    A = torch.zeros((g.N, 33), device=DEV)[:, 1:]  # 4-byte offset, pitch 33
+    with pytest.raises(gs.GnnError) as e:
+        gs.spmm(p, dg, A)
+    assert e.value.status == gs.GNN_ERR_UNSUPPORTED
+
+
+def test_graph_plan_mismatch_and_validate():
+    g = gen.powerlaw_graph(500, 5000, seed=79)
+    dg = upload(g)
+    p = gs.plan(dg, 32)
+    other = upload(gen.powerlaw_graph(500, 5000, seed=80))
+    with pytest.raises(gs.GnnError):
+        gs.spmm(p, other, torch.zeros((500, 32), device=DEV))
+    gs.validate(dg)
+    bad = gs.DeviceGraph(g.M, g.N, dg.row_ind.flip(0).contiguous(), dg.col_ind, dg.val)
+    with pytest.raises(gs.GnnError) as e:
+        gs.validate(bad)
+    assert e.value.status == gs.GNN_ERR_INPUT_CHECK
+
+
+def test_csr_to_coo_matches_oracle():
+    g = gen.powerlaw_graph(7000, 90000, seed=81)
+    rp = torch.from_numpy(g.row_ptr).to(DEV)
+    ri = gs.csr_to_coo(rp).cpu().numpy()
+    assert np.array_equal(ri, oracle.csr_to_coo(g.row_ptr))
