@@ -163,9 +163,9 @@ def run_ours(args):
     import torch
     import torch.distributed as dist
 
-    import gen
     import paper_conf_ipps_fanwc23_b200 as gs
     from gen import configs
+    from paper_conf_ipps_fanwc23_b200 import dist as gdist
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -185,27 +185,17 @@ def run_ours(args):
     g = build_graph(name)
     gen_s = time.time() - t0
     P, p = world, rank
-    rb = gs.shard_rows(g.row_ptr, P)
-    eb = gs.shard_edges(g.nnz, P)
-    r0, r1 = int(rb[p]), int(rb[p + 1])
-    e0, e1 = int(g.row_ptr[r0]), int(g.row_ptr[r1])
-    f0, f1 = int(eb[p]), int(eb[p + 1])
-
+    spec = gdist.shard_spec(g.row_ptr, g.N, rank, world)
     full = gs.DeviceGraph.from_arrays(g.M, g.N, g.row_ind, g.col_ind, g.val, g.row_ptr, device=dev)
-    spg = full.shard(r0, r1, e0, e1) if P > 1 else full
-    sdg = gs.DeviceGraph(g.M, g.N, full.row_ind[f0:f1], full.col_ind[f0:f1],
-                         full.val[f0:f1]) if P > 1 else full
+    spg, sdg = gdist.local_graphs(full, spec)
     # X: replicated (generated on every rank: deterministic) or all-gathered
-    blk = -(-g.N // P)
     X, Xown = {}, {}
     for K in Ks:
         if args.xmode == "allgather" and P > 1:
-            own = gen.features(configs.FEATURE_SEED[name] * 16, min(blk, max(0, g.N - p * blk)),
-                               K, row0=p * blk)
-            buf = torch.zeros((blk, K), dtype=torch.float32, device=dev)
-            buf[:own.shape[0]] = torch.from_numpy(own).to(dev)
-            Xown[K] = buf
-            X[K] = torch.empty((blk * P, K), dtype=torch.float32, device=dev)
+            own = configs.make_features(name, spec.x1 - spec.x0, K, row0=spec.x0)
+            Xown[K] = torch.zeros((spec.xblk, K), dtype=torch.float32, device=dev)
+            Xown[K][:own.shape[0]] = torch.from_numpy(own).to(dev)
+            X[K] = torch.empty((spec.xblk * P, K), dtype=torch.float32, device=dev)
         else:
             X[K] = torch.from_numpy(configs.make_features(name, g.N, K)).to(dev)
     O = {K: torch.empty((spg.M, K), dtype=torch.float32, device=dev) for K in Ks}
@@ -221,7 +211,7 @@ def run_ours(args):
         n = 0
         for K in Ks:
             if args.xmode == "allgather" and P > 1:
-                dist.all_gather_into_tensor(X[K], Xown[K])
+                gdist.gather_features(Xown[K], spec, g.N, out=X[K])
             if ev is not None:
                 ev[K][0].record(stream)
             pl = gs.plan(spg, K)

@@ -284,7 +284,7 @@ def test_misaligned_subview_falls_back_to_scalar_sparse_loads():
     sh = dg.shard(r0, g.M, e0, g.nnz)
     K = 32
     A = _x(77, g.N, K)
-    p = gs.plan(sh, K)
+    p = gs.plan(sh, K, force_chunk=128)
     assert p.info()["vw_sparse"] == 4
     O = gs.spmm(p, sh, torch.from_numpy(A).to(DEV))
     ref, T = oracle.spmm(g.row_ind, g.col_ind, g.val, A, i0=e0, i1=g.nnz, r0=r0, nrows=g.M - r0)
