@@ -23,7 +23,12 @@ oracle/liboracle.so: oracle/oracle.c oracle/oracle.h
 $(PKG)/libgnnsparse.so: $(CUSRC) $(CUHDR)
 	$(NVCC) $(NVFLAGS) -shared -cudart static -o $@ $(CUSRC) 2> $(PKG)/ptxas.log || (cat $(PKG)/ptxas.log; exit 1)
 
+# tuning variants: make variant TAG=x DEFS="-DGNN_SPMM_MINB=2 ..."  ->  build/libgnnsparse_x.so
+variant: $(CUSRC) $(CUHDR)
+	mkdir -p build
+	$(NVCC) $(NVFLAGS) $(DEFS) -shared -cudart static -o build/libgnnsparse_$(TAG).so $(CUSRC) 2> build/ptxas_$(TAG).log || (cat build/ptxas_$(TAG).log; exit 1)
+
 clean:
 	rm -f gen/libgnngen.so oracle/liboracle.so $(PKG)/libgnnsparse.so
 
-.PHONY: all clean
+.PHONY: all clean variant

@@ -85,7 +85,7 @@ int oracle_plan(int64_t nnz, const int32_t *row_ind, int32_t K, int32_t alpha,
     if (!(force_vw == 1 || force_vw == 2 || force_vw == 4 || force_vw == 8)) return -1;
     if (K % force_vw != 0) return -1;
     vw = force_vw;
-  } else if (K % 8 == 0 && K >= 256) {
+  } else if (K % 8 == 0) {
     vw = 8;
   } else if (K % 4 == 0) {
     vw = 4;

@@ -20,7 +20,8 @@ import numpy as np
 import torch
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libgnnsparse.so")
+# GNN_LIB_PATH selects an alternative in-tree build (tuning sweeps, tools/sweep.py)
+LIB_PATH = os.environ.get("GNN_LIB_PATH", os.path.join(_HERE, "libgnnsparse.so"))
 
 __all__ = ["DeviceGraph", "Plan", "PlanOpts", "plan", "spmm", "sddmm", "shard_rows",
            "shard_edges", "csr_to_coo", "validate", "GnnError", "lib", "LIB_PATH"]

@@ -43,7 +43,7 @@ gnn_status_t make_info(int64_t nnz, int32_t K, const gnn_plan_opts_t *opts,
         K % o.force_vw)
       return fail(GNN_ERR_INVALID_ARG, "plan: force_vw=%d invalid for K=%d", o.force_vw, K);
     vw = o.force_vw;
-  } else if (K % 8 == 0 && K >= 256) {
+  } else if (K % 8 == 0) {
     vw = 8;
   } else if (K % 4 == 0) {
     vw = 4;

@@ -7,27 +7,94 @@
 // Per nonzero i of the chunk: gather the A2T[col_i] slice (U rows in flight per
 // lane), multiply with the register-cached A1[row_i] slice -- reloaded only on a row
 // switch, the reuse Algorithm 4 lines 8-11 describe -- reduce over the L lanes
-// with an xor-shuffle tree (WarpReduce, line 12), scale by val_i after the sum
-// (Algo 2 line 6).  Results are parked in the lane that loaded the nonzero's
-// sparse entry and written back as one coalesced vector store per tile (each output
-// written exactly once: plain stores, deterministic).
+// with a transposed butterfly that reduces U nonzeros at once (WarpReduce, line 12),
+// scale by val_i after the sum (Algo 2 line 6) and store: the U results of a
+// batch land in consecutive lanes, so the store is coalesced; each output is written
+// exactly once (plain stores, deterministic).  Tiles whose nonzeros all share one
+// row (for every group of the warp) take a fast path with no per-nonzero row or
+// bounds logic; the next tile's sparse entries are prefetched into registers.
 #include "device.cuh"
 #include "internal.cuh"
 
 namespace gnn {
 
+#ifndef GNN_SDDMM_DEPTH4
+#define GNN_SDDMM_DEPTH4 8
+#endif
+#ifndef GNN_SDDMM_DEPTH8
+#define GNN_SDDMM_DEPTH8 4
+#endif
+#ifndef GNN_SDDMM_MINB
+#define GNN_SDDMM_MINB 1
+#endif
+
 template <int VW>
 struct SddmmDepth {
-  static constexpr int value = VW == 8 ? 4 : 8;
+  static constexpr int value = VW == 8 ? GNN_SDDMM_DEPTH8 : GNN_SDDMM_DEPTH4;
 };
 
+// WarpReduce (Algo 4 line 12) of U partial dot products at once over the group's L
+// lanes, as a transposed butterfly: each halving step exchanges half of the values
+// (U/2 + U/4 + ... shuffles instead of U * log2 L).  Afterwards value u lives in lane
+// l with u = l * U / L (U <= L; lanes l % (L/U) == 0 are its owners) or, for U > L, in
+// slot i of lane l with u = l * (U/L) + i.  Then S_O = sum * v (Algo 2 line 6) is
+// stored for the first `valid` of the U nonzeros at out[0..U).
+template <int U, int L>
+__device__ __forceinline__ void reduce_scale_store(float (&part)[U], const float (&vj)[U],
+                                                   const int l, float *__restrict__ out,
+                                                   const int valid) {
+  constexpr int P = U > L ? U / L : 1;  // values left per lane after the halving steps
+  int cnt = U;
+#pragma unroll
+  for (int o = L / 2; o >= 1; o >>= 1) {
+    if (cnt > 1) {
+      const int half = cnt / 2;
+      const bool b = (l & o) != 0;
+#pragma unroll
+      for (int i = 0; i < U / 2; ++i) {
+        if (i < half) {
+          const float lo = part[i], hi = part[i + half];
+          const float send = b ? lo : hi;
+          const float keep = b ? hi : lo;
+          part[i] = keep + __shfl_xor_sync(kFull, send, o, L);
+        }
+      }
+      cnt = half;
+    } else {
+      part[0] += __shfl_xor_sync(kFull, part[0], o, L);
+    }
+  }
+  if constexpr (U <= L) {
+    constexpr int R = L / U;
+    const int u = l / R;
+    if (l % R == 0 && u < valid) {
+      float v = vj[0];
+#pragma unroll
+      for (int w = 1; w < U; ++w) v = (w == u) ? vj[w] : v;
+      out[u] = part[0] * v;
+    }
+  } else {
+#pragma unroll
+    for (int i = 0; i < P; ++i) {
+      const int u = l * P + i;
+      if (u < valid) {
+        float v = vj[0];
+#pragma unroll
+        for (int w = 1; w < U; ++w) v = (w == u) ? vj[w] : v;
+        out[u] = part[i] * v;
+      }
+    }
+  }
+}
+
 template <int VW, int L, int VWS, int SMAX>
-__global__ void __launch_bounds__(kMaxThreads)
+__global__ void __launch_bounds__(kMaxThreads, GNN_SDDMM_MINB)
     sddmm_kernel(const SparseArgs a, const float *__restrict__ A1, const int64_t lda1,
                  const float *__restrict__ A2T, const int64_t lda2, float *__restrict__ out) {
   constexpr int G = 32 / L;
   constexpr int T = L * VWS;
-  constexpr int U = SddmmDepth<VW>::value < T ? SddmmDepth<VW>::value : T;
+  constexpr int U0 = SddmmDepth<VW>::value > VWS ? SddmmDepth<VW>::value : VWS;
+  constexpr int U = U0 < T ? U0 : T;
   static_assert(T % U == 0 && U % VWS == 0, "tile / prefetch shape");
   const int lane = threadIdx.x & 31;
   const int g = lane / L;
@@ -36,11 +103,13 @@ __global__ void __launch_bounds__(kMaxThreads)
   const bool item_ok = c < a.num_chunks;
   if (!__any_sync(kFull, item_ok)) return;
   const int64_t cs = c * a.chunk;
-  const int64_t ce = item_ok ? min(cs + (int64_t)a.chunk, a.nnz) : cs;
+  const int n = item_ok ? (int)(min(cs + (int64_t)a.chunk, a.nnz) - cs) : 0;
   const int S = a.slices;  // <= SMAX (host-checked)
+  const uint32_t ld2B = (uint32_t)lda2 * 4u;
+  const char *__restrict__ A2b = reinterpret_cast<const char *>(A2T);
 
   float a1[SMAX][VW];
-  int32_t cur[SMAX];
+  int32_t cur[SMAX];  // row whose A1 slice is cached, per slice
 #pragma unroll
   for (int sl = 0; sl < SMAX; ++sl) {
     cur[sl] = -1;
@@ -48,30 +117,59 @@ __global__ void __launch_bounds__(kMaxThreads)
     for (int v = 0; v < VW; ++v) a1[sl][v] = 0.f;
   }
 
+  const int32_t *__restrict__ ri = a.row_ind + cs;
+  const int32_t *__restrict__ ci = a.col_ind + cs;
+  const float *__restrict__ vi = a.val ? a.val + cs : nullptr;
+  float *__restrict__ oc = out + cs;
+  int32_t rr[VWS], cc[VWS], nr[VWS], nc[VWS];
+  float vv[VWS], nv[VWS];
+  ld_sparse_i32<VWS>(ri, l * VWS, n, 0, nr);
+  ld_sparse_i32<VWS>(ci, l * VWS, n, 0, nc);
+  ld_sparse_f32<VWS>(vi, l * VWS, n, nv);
+
+  auto load_a1 = [&](int32_t row) {
+#pragma unroll
+    for (int sl = 0; sl < SMAX; ++sl) {
+      const int k0 = (sl * L + l) * VW;
+      if (sl < S && k0 < a.K)
+        ld_feat<VW>(A1 + ((int64_t)row - a.row_base) * lda1 + k0, a1[sl]);
+      cur[sl] = row;
+    }
+  };
+
   const int ntiles = (a.chunk + T - 1) / T;
   for (int t = 0; t < ntiles; ++t) {
-    const int64_t tb = cs + (int64_t)t * T;
-    const int64_t li = tb + (int64_t)l * VWS;
-    int32_t rr[VWS], cc[VWS];
-    float vv[VWS];
-    ld_sparse_i32<VWS>(a.row_ind, li, ce, 0, rr);
-    ld_sparse_i32<VWS>(a.col_ind, li, ce, 0, cc);
-    ld_sparse_f32<VWS>(a.val, li, ce, vv);
-    float res[VWS];
+    const int tb = t * T;
 #pragma unroll
-    for (int q = 0; q < VWS; ++q) res[q] = 0.f;
+    for (int q = 0; q < VWS; ++q) {
+      rr[q] = nr[q];
+      cc[q] = nc[q];
+      vv[q] = nv[q];
+    }
+    if (t + 1 < ntiles) {
+      const int li = tb + T + l * VWS;
+      ld_sparse_i32<VWS>(ri, li, n, 0, nr);
+      ld_sparse_i32<VWS>(ci, li, n, 0, nc);
+      ld_sparse_f32<VWS>(vi, li, n, nv);
+    }
+    const int32_t r_first = __shfl_sync(kFull, rr[0], 0, L);
+    const int32_t r_last = __shfl_sync(kFull, rr[VWS - 1], L - 1, L);
+    const bool fast = __all_sync(kFull, ((tb + T <= n) && r_first == r_last) || !item_ok);
+    if (fast && item_ok && r_first != cur[0]) load_a1(r_first);  // row switch at tile start
 #pragma unroll 1
     for (int jj = 0; jj < T; jj += U) {
-      int32_t rj[U], cj[U];
+      int32_t rj[U];
+      uint32_t cj[U];
       float vj[U], part[U];
 #pragma unroll
       for (int u = 0; u < U; ++u) {
         const int src = (jj + u) / VWS;
-        rj[u] = __shfl_sync(kFull, rr[u % VWS], src, L);
-        cj[u] = __shfl_sync(kFull, cc[u % VWS], src, L);
+        cj[u] = (uint32_t)__shfl_sync(kFull, cc[u % VWS], src, L);
         vj[u] = __shfl_sync(kFull, vv[u % VWS], src, L);
+        rj[u] = fast ? r_first : __shfl_sync(kFull, rr[u % VWS], src, L);
         part[u] = 0.f;
       }
+      const int valid = n - (tb + jj);
 #pragma unroll
       for (int sl = 0; sl < SMAX; ++sl) {
         if (sl < S) {
@@ -80,8 +178,9 @@ __global__ void __launch_bounds__(kMaxThreads)
           float x[U][VW];
 #pragma unroll
           for (int u = 0; u < U; ++u) {
-            if (col_ok && tb + jj + u < ce) {
-              ld_feat<VW>(A2T + (int64_t)cj[u] * lda2 + k0, x[u]);
+            if (col_ok && (fast || u < valid)) {
+              ld_feat<VW>(reinterpret_cast<const float *>(A2b + (uint64_t)cj[u] * ld2B) + k0,
+                          x[u]);
             } else {
 #pragma unroll
               for (int v = 0; v < VW; ++v) x[u][v] = 0.f;
@@ -89,43 +188,16 @@ __global__ void __launch_bounds__(kMaxThreads)
           }
 #pragma unroll
           for (int u = 0; u < U; ++u) {
-            if (col_ok && tb + jj + u < ce) {
-              if (rj[u] != cur[sl]) {  // row switch: load the new A1 row (Algo 4 l. 8-11)
-                ld_feat<VW>(A1 + ((int64_t)rj[u] - a.row_base) * lda1 + k0, a1[sl]);
-                cur[sl] = rj[u];
-              }
-              float d = part[u];
-#pragma unroll
-              for (int v = 0; v < VW; ++v) d = fmaf(a1[sl][v], x[u][v], d);
-              part[u] = d;
+            if (!fast && col_ok && u < valid && rj[u] != cur[sl]) {
+              // row-switch procedure: load the new A1 row (Algo 4 lines 8-11)
+              cur[sl] = rj[u];
+              ld_feat<VW>(A1 + ((int64_t)rj[u] - a.row_base) * lda1 + k0, a1[sl]);
             }
+            part[u] = dot_acc<VW>(part[u], a1[sl], x[u]);
           }
         }
       }
-      // WarpReduce over the group's L lanes (Algo 4 line 12), then v scaling.
-#pragma unroll
-      for (int u = 0; u < U; ++u) {
-        float d = part[u];
-#pragma unroll
-        for (int o = L / 2; o > 0; o >>= 1) d += __shfl_xor_sync(kFull, d, o, L);
-        if (l == (jj + u) / VWS) res[u % VWS] = d * vj[u];
-      }
-    }
-    // one coalesced store of the tile's T results
-    if (li < ce) {
-      if (li + VWS <= ce) {
-        if constexpr (VWS == 4) {
-          *reinterpret_cast<float4 *>(out + li) = make_float4(res[0], res[1], res[2], res[3]);
-        } else if constexpr (VWS == 2) {
-          *reinterpret_cast<float2 *>(out + li) = make_float2(res[0], res[1]);
-        } else {
-          out[li] = res[0];
-        }
-      } else {
-#pragma unroll
-        for (int q = 0; q < VWS; ++q)
-          if (li + q < ce) out[li + q] = res[q];
-      }
+      reduce_scale_store<U, L>(part, vj, l, oc + tb + jj, item_ok ? valid : 0);
     }
   }
 }
@@ -178,7 +250,7 @@ extern "C" GNN_API gnn_status_t gnn_sddmm(gnn_plan_t plan, const gnn_graph_t *g,
   const gnn_plan_info_t &in = p->info;
   const int K = in.K, VW = in.vw_feat;
   if (g->nnz == 0) return GNN_OK;
-  if (!A1 || !A2T || !out || lda1 < K || lda2 < K)
+  if (!A1 || !A2T || !out || lda1 < K || lda2 < K || lda2 >= (int64_t(1) << 30))
     return fail(GNN_ERR_INVALID_ARG, "gnn_sddmm: bad dense operand");
   if (!aligned(A1, 4u * VW) || !aligned(A2T, 4u * VW) || lda1 % VW || lda2 % VW)
     return fail(GNN_ERR_UNSUPPORTED,

@@ -9,7 +9,10 @@
 // VW = 8).  G = 32/L groups share a warp.  Per tile of T = L*vw_sparse nonzeros the
 // group loads (row, col, val) coalesced and vectorised, then broadcasts them
 // nonzero by nonzero with width-L shuffles; U feature rows are in flight per lane
-// before the FMAs consume them.  A row switch ("row-switch procedure")
+// before the FMAs consume them, and the next tile's sparse entries are prefetched into
+// registers.  Tiles whose nonzeros all belong to one row (for every group of the warp;
+// the common case at high degree) take a fast path with no per-nonzero row or bounds
+// logic; the others run the general row-switch loop.  A row switch ("row-switch procedure")
 // flushes the accumulator: rows wholly inside the chunk get a plain vector store,
 // rows shared with a neighbouring chunk (plan flags) a vector atomic add into a row
 // zeroed beforehand by spmm_prezero_kernel.  Empty rows are written as zeros by the
@@ -21,21 +24,45 @@
 
 namespace gnn {
 
+#ifndef GNN_SPMM_DEPTH4
+#define GNN_SPMM_DEPTH4 8  // feature rows in flight per lane at VW <= 4
+#endif
+#ifndef GNN_SPMM_DEPTH8
+#define GNN_SPMM_DEPTH8 4  // ... at VW = 8 (256-bit loads)
+#endif
+#ifndef GNN_SPMM_MINB
+#define GNN_SPMM_MINB 1    // min resident 512-thread blocks/SM the register budget must allow
+#endif
+
 template <int VW>
 struct FeatDepth {
-  static constexpr int value = VW == 8 ? 4 : 8;  // feature rows in flight per lane
+  static constexpr int value = VW == 8 ? GNN_SPMM_DEPTH8 : GNN_SPMM_DEPTH4;
 };
 
 template <int VW, int L, int VWS>
 struct TileCfg {
   static constexpr int G = 32 / L;
   static constexpr int T = L * VWS;  // nonzeros per tile per group
-  static constexpr int U = FeatDepth<VW>::value < T ? FeatDepth<VW>::value : T;
+  static constexpr int U0 = FeatDepth<VW>::value > VWS ? FeatDepth<VW>::value : VWS;
+  static constexpr int U = U0 < T ? U0 : T;
   static_assert(T % U == 0 && U % VWS == 0, "tile / prefetch shape");
 };
 
+// Flush the accumulator of row `cur` (Algo 3 line 15, "AtomicStore"): rows shared
+// with a neighbouring chunk are combined with a vector atomic add, rows owned by this
+// chunk get a plain vector store.
+template <int VW>
+__device__ __forceinline__ void flush_row(float *Ok, int64_t ldo, int64_t row_base, int32_t cur,
+                                          int32_t rf, int32_t rl, uint32_t fl,
+                                          const float (&acc)[VW]) {
+  float *o = Ok + ((int64_t)cur - row_base) * ldo;
+  const bool shared = (cur == rf && (fl & 1u)) || (cur == rl && (fl & 2u));
+  if (shared) red_add<VW>(o, acc);
+  else st_vec<VW>(o, acc);
+}
+
 template <int VW, int L, int VWS>
-__global__ void __launch_bounds__(kMaxThreads)
+__global__ void __launch_bounds__(kMaxThreads, GNN_SPMM_MINB)
     spmm_kernel(const SparseArgs a, const float *__restrict__ A, const int64_t lda,
                 float *__restrict__ O, const int64_t ldo) {
   using Cfg = TileCfg<VW, L, VWS>;
@@ -56,7 +83,7 @@ __global__ void __launch_bounds__(kMaxThreads)
   const int k0 = (s * L + l) * VW;
   const bool col_ok = item_ok && k0 < a.K;
   const int64_t cs = c * a.chunk;
-  const int64_t ce = item_ok ? min(cs + (int64_t)a.chunk, a.nnz) : cs;
+  const int n = item_ok ? (int)(min(cs + (int64_t)a.chunk, a.nnz) - cs) : 0;  // nnz here
   int32_t rf = 0, rl = 0;
   uint32_t fl = 0;
   if (item_ok) {
@@ -64,7 +91,9 @@ __global__ void __launch_bounds__(kMaxThreads)
     rl = a.row_last[c];
     fl = a.flags[c];
   }
-  const float *__restrict__ Ak = A + k0;
+  // feature row c of A starts at Ab + c * ldaB (IMAD.WIDE.U32 per gather)
+  const char *__restrict__ Ab = reinterpret_cast<const char *>(A + k0);
+  const uint32_t ldaB = (uint32_t)lda * 4u;
   float *__restrict__ Ok = O + k0;  // row r at Ok + (r - row_base) * ldo
 
   // empty rows between the previous chunk's last row and ours are ours to zero
@@ -78,64 +107,115 @@ __global__ void __launch_bounds__(kMaxThreads)
   for (int v = 0; v < VW; ++v) acc[v] = 0.f;
   int32_t cur = -1;
 
+  const int32_t *__restrict__ ri = a.row_ind + cs;
+  const int32_t *__restrict__ ci = a.col_ind + cs;
+  const float *__restrict__ vi = a.val ? a.val + cs : nullptr;
+  // sparse tile registers: current and next (prefetched one tile ahead)
+  int32_t rr[VWS], cc[VWS], nr[VWS], nc[VWS];
+  float vv[VWS], nv[VWS];
+  ld_sparse_i32<VWS>(ri, l * VWS, n, 0, nr);
+  ld_sparse_i32<VWS>(ci, l * VWS, n, 0, nc);
+  ld_sparse_f32<VWS>(vi, l * VWS, n, nv);
+
   const int ntiles = (a.chunk + T - 1) / T;  // warp-uniform trip count
   for (int t = 0; t < ntiles; ++t) {
-    const int64_t tb = cs + (int64_t)t * T;
-    const int64_t li = tb + (int64_t)l * VWS;
-    int32_t rr[VWS], cc[VWS];
-    float vv[VWS];
-    ld_sparse_i32<VWS>(a.row_ind, li, ce, 0, rr);
-    ld_sparse_i32<VWS>(a.col_ind, li, ce, 0, cc);
-    ld_sparse_f32<VWS>(a.val, li, ce, vv);
-#pragma unroll 1
-    for (int jj = 0; jj < T; jj += U) {
-      int32_t rj[U], cj[U];
-      float vj[U];
+    const int tb = t * T;
 #pragma unroll
-      for (int u = 0; u < U; ++u) {
-        const int src = (jj + u) / VWS;
-        rj[u] = __shfl_sync(kFull, rr[u % VWS], src, L);
-        cj[u] = __shfl_sync(kFull, cc[u % VWS], src, L);
-        vj[u] = __shfl_sync(kFull, vv[u % VWS], src, L);
+    for (int q = 0; q < VWS; ++q) {
+      rr[q] = nr[q];
+      cc[q] = nc[q];
+      vv[q] = nv[q];
+    }
+    if (t + 1 < ntiles) {  // prefetch the next tile's sparse entries
+      const int li = tb + T + l * VWS;
+      ld_sparse_i32<VWS>(ri, li, n, 0, nr);
+      ld_sparse_i32<VWS>(ci, li, n, 0, nc);
+      ld_sparse_f32<VWS>(vi, li, n, nv);
+    }
+    const int32_t r_first = __shfl_sync(kFull, rr[0], 0, L);
+    const int32_t r_last = __shfl_sync(kFull, rr[VWS - 1], L - 1, L);
+    const bool fast_g = (tb + T <= n) && r_first == r_last;
+    if (__all_sync(kFull, fast_g || !item_ok)) {
+      // ---- fast path: the whole tile belongs to one row (all groups of the warp)
+      if (item_ok && r_first != cur) {
+        if (cur >= 0 && col_ok) {
+          flush_row<VW>(Ok, ldo, a.row_base, cur, rf, rl, fl, acc);
+          for (int64_t r = (int64_t)cur + 1; r < r_first; ++r)
+            st_zero<VW>(Ok + (r - a.row_base) * ldo);
+        }
+        cur = r_first;
+#pragma unroll
+        for (int v = 0; v < VW; ++v) acc[v] = 0.f;
       }
-      float x[U][VW];
+#pragma unroll 1
+      for (int jj = 0; jj < T; jj += U) {
+        uint32_t cj[U];
+        float vj[U];
 #pragma unroll
-      for (int u = 0; u < U; ++u) {
-        if (col_ok && tb + jj + u < ce) {
-          ld_feat<VW>(Ak + (int64_t)cj[u] * lda, x[u]);
-        } else {
+        for (int u = 0; u < U; ++u) {
+          const int src = (jj + u) / VWS;
+          cj[u] = (uint32_t)__shfl_sync(kFull, cc[u % VWS], src, L);
+          vj[u] = __shfl_sync(kFull, vv[u % VWS], src, L);
+        }
+        float x[U][VW];
 #pragma unroll
-          for (int v = 0; v < VW; ++v) x[u][v] = 0.f;
+        for (int u = 0; u < U; ++u) {
+          if (col_ok) {
+            ld_feat<VW>(reinterpret_cast<const float *>(Ab + (uint64_t)cj[u] * ldaB), x[u]);
+          } else {
+#pragma unroll
+            for (int v = 0; v < VW; ++v) x[u][v] = 0.f;
+          }
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          axpy<VW>(acc, vj[u], x[u]);
         }
       }
+    } else {
+      // ---- general path: per-nonzero validity and row-switch procedure
+#pragma unroll 1
+      for (int jj = 0; jj < T; jj += U) {
+        int32_t rj[U];
+        uint32_t cj[U];
+        float vj[U];
 #pragma unroll
-      for (int u = 0; u < U; ++u) {
-        if (tb + jj + u < ce) {
-          if (rj[u] != cur) {  // row-switch procedure
-            if (cur >= 0 && col_ok) {
-              float *o = Ok + ((int64_t)cur - a.row_base) * ldo;
-              const bool shared = (cur == rf && (fl & 1u)) || (cur == rl && (fl & 2u));
-              if (shared) red_add<VW>(o, acc);
-              else st_vec<VW>(o, acc);
-              for (int64_t r = (int64_t)cur + 1; r < rj[u]; ++r)
-                st_zero<VW>(Ok + (r - a.row_base) * ldo);
-            }
-            cur = rj[u];
+        for (int u = 0; u < U; ++u) {
+          const int src = (jj + u) / VWS;
+          rj[u] = __shfl_sync(kFull, rr[u % VWS], src, L);
+          cj[u] = (uint32_t)__shfl_sync(kFull, cc[u % VWS], src, L);
+          vj[u] = __shfl_sync(kFull, vv[u % VWS], src, L);
+        }
+        float x[U][VW];
 #pragma unroll
-            for (int v = 0; v < VW; ++v) acc[v] = 0.f;
+        for (int u = 0; u < U; ++u) {
+          if (col_ok && tb + jj + u < n) {
+            ld_feat<VW>(reinterpret_cast<const float *>(Ab + (uint64_t)cj[u] * ldaB), x[u]);
+          } else {
+#pragma unroll
+            for (int v = 0; v < VW; ++v) x[u][v] = 0.f;
           }
+        }
 #pragma unroll
-          for (int v = 0; v < VW; ++v) acc[v] = fmaf(vj[u], x[u][v], acc[v]);
+        for (int u = 0; u < U; ++u) {
+          if (tb + jj + u < n) {
+            if (rj[u] != cur) {  // row-switch procedure
+              if (cur >= 0 && col_ok) {
+                flush_row<VW>(Ok, ldo, a.row_base, cur, rf, rl, fl, acc);
+                for (int64_t r = (int64_t)cur + 1; r < rj[u]; ++r)
+                  st_zero<VW>(Ok + (r - a.row_base) * ldo);
+              }
+              cur = rj[u];
+#pragma unroll
+              for (int v = 0; v < VW; ++v) acc[v] = 0.f;
+            }
+            axpy<VW>(acc, vj[u], x[u]);
+          }
         }
       }
     }
   }
-  if (cur >= 0 && col_ok) {
-    float *o = Ok + ((int64_t)cur - a.row_base) * ldo;
-    const bool shared = (cur == rf && (fl & 1u)) || (cur == rl && (fl & 2u));
-    if (shared) red_add<VW>(o, acc);
-    else st_vec<VW>(o, acc);
-  }
+  if (cur >= 0 && col_ok) flush_row<VW>(Ok, ldo, a.row_base, cur, rf, rl, fl, acc);
   // trailing empty rows after the last chunk
   if (col_ok && c == a.num_chunks - 1) {
     for (int64_t r = (int64_t)rl + 1; r < a.row_base + a.M; ++r)
@@ -261,7 +341,7 @@ extern "C" GNN_API gnn_status_t gnn_spmm(gnn_plan_t plan, const gnn_graph_t *g, 
   const gnn_plan_info_t &in = p->info;
   const int K = in.K, VW = in.vw_feat;
   if (g->M == 0) return GNN_OK;
-  if (!O || ldo < K || (g->nnz > 0 && (!A || lda < K)))
+  if (!O || ldo < K || (g->nnz > 0 && (!A || lda < K || lda >= (int64_t(1) << 30))))
     return fail(GNN_ERR_INVALID_ARG, "gnn_spmm: bad dense operand (lda=%lld ldo=%lld K=%d)",
                 (long long)lda, (long long)ldo, K);
   if (!aligned(O, 4u * VW) || ldo % VW || (g->nnz > 0 && (!aligned(A, 4u * VW) || lda % VW)))

@@ -251,9 +251,9 @@ def _brute_blocks(nnz, C, S, G, WPB):
 
 
 VW_TABLE = {  # K: (vw_feat, lanes, slices, groups) -- DESIGN.md "Plan rule" table
-    32: (4, 8, 1, 4), 64: (4, 16, 1, 2), 128: (4, 32, 1, 1), 256: (8, 32, 1, 1),
+    32: (8, 4, 1, 8), 64: (8, 8, 1, 4), 128: (8, 16, 1, 2), 256: (8, 32, 1, 1),
     100: (4, 32, 1, 1), 33: (1, 32, 2, 1), 1000: (8, 32, 4, 1), 6: (2, 4, 1, 8),
-    1: (1, 1, 1, 32), 512: (8, 32, 2, 1), 24: (4, 8, 1, 4),
+    1: (1, 1, 1, 32), 512: (8, 32, 2, 1), 24: (8, 4, 1, 8), 12: (4, 4, 1, 8),
 }
 
 
