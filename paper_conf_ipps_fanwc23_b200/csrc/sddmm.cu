@@ -18,19 +18,22 @@
 
 namespace gnn {
 
-#ifndef GNN_SDDMM_DEPTH4
-#define GNN_SDDMM_DEPTH4 8
+// Rows in flight per lane (U) and register budget (min blocks of 512 threads per SM)
+// per instantiation, measured on C4 (profiles/r01_sweep4.txt): U = 8 with 256-bit loads,
+// except full-warp groups (L = 32, K >= 256) which prefer more resident warps (2 blocks,
+// U = 2).
+template <int VW, int L>
+struct SddmmShape {
+#if defined(GNN_SDDMM_DEPTH8)
+  static constexpr int depth = VW == 8 ? GNN_SDDMM_DEPTH8 : 8;
+#else
+  static constexpr int depth = (VW == 8 && L == 32) ? 2 : 8;
 #endif
-#ifndef GNN_SDDMM_DEPTH8
-#define GNN_SDDMM_DEPTH8 4
+#if defined(GNN_SDDMM_MINB)
+  static constexpr int minb = GNN_SDDMM_MINB;
+#else
+  static constexpr int minb = (VW == 8 && L == 32) ? 2 : 1;
 #endif
-#ifndef GNN_SDDMM_MINB
-#define GNN_SDDMM_MINB 1
-#endif
-
-template <int VW>
-struct SddmmDepth {
-  static constexpr int value = VW == 8 ? GNN_SDDMM_DEPTH8 : GNN_SDDMM_DEPTH4;
 };
 
 // WarpReduce (Algo 4 line 12) of U partial dot products at once over the group's L
@@ -88,12 +91,12 @@ __device__ __forceinline__ void reduce_scale_store(float (&part)[U], const float
 }
 
 template <int VW, int L, int VWS, int SMAX>
-__global__ void __launch_bounds__(kMaxThreads, GNN_SDDMM_MINB)
+__global__ void __launch_bounds__(kMaxThreads, (SMAX > 1 ? 1 : SddmmShape<VW, L>::minb))
     sddmm_kernel(const SparseArgs a, const float *__restrict__ A1, const int64_t lda1,
                  const float *__restrict__ A2T, const int64_t lda2, float *__restrict__ out) {
   constexpr int G = 32 / L;
   constexpr int T = L * VWS;
-  constexpr int U0 = SddmmDepth<VW>::value > VWS ? SddmmDepth<VW>::value : VWS;
+  constexpr int U0 = SddmmShape<VW, L>::depth > VWS ? SddmmShape<VW, L>::depth : VWS;
   constexpr int U = U0 < T ? U0 : T;
   static_assert(T % U == 0 && U % VWS == 0, "tile / prefetch shape");
   const int lane = threadIdx.x & 31;

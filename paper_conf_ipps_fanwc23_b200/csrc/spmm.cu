@@ -24,26 +24,27 @@
 
 namespace gnn {
 
-#ifndef GNN_SPMM_DEPTH4
-#define GNN_SPMM_DEPTH4 8  // feature rows in flight per lane at VW <= 4
-#endif
-#ifndef GNN_SPMM_DEPTH8
-#define GNN_SPMM_DEPTH8 4  // ... at VW = 8 (256-bit loads)
-#endif
+// Feature rows in flight per lane (U) and the register budget, per instantiation.
+// Measured on C4 (profiles/r01_sweep4.txt): with 256-bit loads U = 4 is best while
+// several chunks share a warp (L <= 8), U = 8 once a group spans >= 16 lanes.
 #ifndef GNN_SPMM_MINB
-#define GNN_SPMM_MINB 1    // min resident 512-thread blocks/SM the register budget must allow
+#define GNN_SPMM_MINB 1  // min resident 512-thread blocks/SM the register budget must allow
 #endif
 
-template <int VW>
+template <int VW, int L>
 struct FeatDepth {
-  static constexpr int value = VW == 8 ? GNN_SPMM_DEPTH8 : GNN_SPMM_DEPTH4;
+#if defined(GNN_SPMM_DEPTH8)
+  static constexpr int value = VW == 8 ? GNN_SPMM_DEPTH8 : 8;
+#else
+  static constexpr int value = VW == 8 ? (L >= 16 ? 8 : 4) : 8;
+#endif
 };
 
 template <int VW, int L, int VWS>
 struct TileCfg {
   static constexpr int G = 32 / L;
   static constexpr int T = L * VWS;  // nonzeros per tile per group
-  static constexpr int U0 = FeatDepth<VW>::value > VWS ? FeatDepth<VW>::value : VWS;
+  static constexpr int U0 = FeatDepth<VW, L>::value > VWS ? FeatDepth<VW, L>::value : VWS;
   static constexpr int U = U0 < T ? U0 : T;
   static_assert(T % U == 0 && U % VWS == 0, "tile / prefetch shape");
 };
