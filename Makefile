@@ -8,7 +8,7 @@ PKG     := paper_conf_ipps_fanwc23_b200
 ARCH    := -gencode arch=compute_100a,code=sm_100a
 NVFLAGS := -ccbin /usr/bin/g++ $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC -Xcompiler -fvisibility=hidden \
            -Iinclude --expt-relaxed-constexpr -Xptxas -v
-CUSRC   := $(wildcard $(PKG)/csrc/*.cu)
+CUSRC   := $(wildcard $(PKG)/csrc/*.cu) $(wildcard $(PKG)/csrc/*.cpp)
 CUHDR   := $(wildcard $(PKG)/csrc/*.cuh) include/gnn_sparse.h
 
 all: gen/libgnngen.so oracle/liboracle.so $(PKG)/libgnnsparse.so

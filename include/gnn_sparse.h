@@ -153,6 +153,40 @@ GNN_API gnn_status_t gnn_shard_rows(const int32_t *row_ptr_host, int64_t M, int3
 /* Equal edge-range shards: bounds[p] = floor(p * nnz / P), [P+1] host array. */
 GNN_API gnn_status_t gnn_shard_edges(int64_t nnz, int32_t P, int64_t *bounds);
 
+/* ------------------------------------------------------------- reorder ---- */
+/* Graph Clustering based Reordering (GCR, Fig. 8) -- optional, HOST side,
+ * offline (it is not part of the timed kernels, P:323 / P:275).  Louvain community
+ * detection (refs [29][30]) on the symmetric square graph given as HOST CSR
+ * (row_ptr[n+1], col_ind[nnz]; self-loops ignored), then a hierarchical node order
+ * (DESIGN.md §2 item 23).  Outputs perm[old] = new (a bijection of [0,n)), optionally
+ * the top-level community of each ORIGINAL node and the modularity of that partition.
+ * Zero-initialised option fields take the defaults (3 levels, 20 passes per level,
+ * min_gain 1e-6, resolution 1.0).  Single-threaded; deterministic. */
+typedef struct {
+  int32_t max_levels;
+  int32_t max_passes;
+  double min_gain;
+  double resolution;
+} gnn_reorder_opts_t;
+GNN_API gnn_status_t gnn_reorder_gcr(const int32_t *row_ptr_host, const int32_t *col_ind_host,
+                                     int64_t n, const gnn_reorder_opts_t *opts,
+                                     int32_t *perm_host, int32_t *comm_host,
+                                     double *modularity);
+/* Apply a node permutation to a square hybrid CSR/COO (HOST arrays): S' = P S P^T with
+ * new row perm[r] holding new columns perm[c] sorted ascending (ties keep the original
+ * order), values carried along; row_ind_out (the decoded RowInd) may be NULL,
+ * val/val_out may be NULL.  Output arrays are caller-allocated (n+1 / nnz entries). */
+GNN_API gnn_status_t gnn_permute_graph(const int32_t *row_ptr_host, const int32_t *col_ind_host,
+                                       const float *val_host, int64_t n, const int32_t *perm_host,
+                                       int32_t *row_ptr_out, int32_t *row_ind_out,
+                                       int32_t *col_ind_out, float *val_out);
+/* Permute dense rows on the device: Y[perm[i]][:K] = X[i][:K] for i in [0, n) (X' = P X,
+ * so SpMM(P S P^T, P X) = P SpMM(S, X)).  perm is a DEVICE array; X and Y must not
+ * overlap. */
+GNN_API gnn_status_t gnn_permute_rows(const float *X, int64_t ldx, int64_t n, int64_t K,
+                                      const int32_t *perm, float *Y, int64_t ldy,
+                                      gnn_stream_t stream);
+
 /* ------------------------------------------------------------- helpers ---- */
 /* Decode CSR offsets into the hybrid format's RowInd (Fig. 2d):
  * row_ind[i - row_ptr[0]] = r + row_base for row_ptr[r] <= i < row_ptr[r+1]. */

@@ -47,6 +47,8 @@ def _load():
     lib.oracle_shard_rows.argtypes = [vp, i64, i32, vp]
     lib.oracle_shard_edges.argtypes = [i64, i32, vp]
     lib.oracle_csr_to_coo.argtypes = [vp, i64, vp]
+    lib.oracle_modularity.argtypes = [vp, vp, i64, vp, i32]
+    lib.oracle_modularity.restype = ctypes.c_double
     for f in ("oracle_spmm", "oracle_sddmm", "oracle_plan", "oracle_shard_rows",
               "oracle_shard_edges", "oracle_csr_to_coo"):
         getattr(lib, f).restype = ctypes.c_int
@@ -178,3 +180,10 @@ def csr_to_coo(row_ptr):
     if lib.oracle_csr_to_coo(_ptr(row_ptr), M, _ptr(out)) != 0:
         raise ValueError("oracle_csr_to_coo: invalid arguments")
     return out
+
+
+def modularity(row_ptr, col_ind, comm, skip_self=True):
+    """Modularity of partition `comm` of the symmetric unit-weight CSR graph."""
+    lib = _load()
+    rp, ci, cm = _i32(row_ptr), _i32(col_ind), _i32(comm)
+    return lib.oracle_modularity(_ptr(rp), _ptr(ci), rp.shape[0] - 1, _ptr(cm), int(skip_self))

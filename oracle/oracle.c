@@ -176,3 +176,28 @@ int oracle_csr_to_coo(const int32_t *row_ptr, int64_t M, int32_t *row_ind) {
     for (int64_t i = row_ptr[r]; i < row_ptr[r + 1]; ++i) row_ind[i - base] = (int32_t)r;
   return 0;
 }
+
+/* ------------------------------------------------------- modularity ------ */
+#include <stdlib.h>
+double oracle_modularity(const int32_t *row_ptr, const int32_t *col_ind, int64_t n,
+                         const int32_t *comm, int32_t skip_self) {
+  double *in = (double *)calloc((size_t)n + 1, sizeof(double));
+  double *tot = (double *)calloc((size_t)n + 1, sizeof(double));
+  double m2 = 0.0;
+  int64_t base = row_ptr[0];
+  for (int64_t i = 0; i < n; ++i) {
+    for (int64_t e = row_ptr[i] - base; e < row_ptr[i + 1] - base; ++e) {
+      int64_t j = col_ind[e];
+      if (skip_self && j == i) continue;
+      m2 += 1.0;                      /* sum_i k_i = 2m */
+      tot[comm[i]] += 1.0;            /* k_i accumulated into tot_{c_i} */
+      if (comm[j] == comm[i]) in[comm[i]] += 1.0;
+    }
+  }
+  double q = 0.0;
+  if (m2 > 0)
+    for (int64_t c = 0; c < n; ++c) q += in[c] / m2 - (tot[c] / m2) * (tot[c] / m2);
+  free(in);
+  free(tot);
+  return q;
+}

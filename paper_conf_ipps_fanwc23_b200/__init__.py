@@ -24,7 +24,8 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("GNN_LIB_PATH", os.path.join(_HERE, "libgnnsparse.so"))
 
 __all__ = ["DeviceGraph", "Plan", "PlanOpts", "plan", "spmm", "sddmm", "shard_rows",
-           "shard_edges", "csr_to_coo", "validate", "GnnError", "lib", "LIB_PATH"]
+           "shard_edges", "reorder_gcr", "permute_graph", "permute_rows", "csr_to_coo",
+           "validate", "GnnError", "lib", "LIB_PATH"]
 
 GNN_OK, GNN_ERR_INVALID_ARG, GNN_ERR_UNSUPPORTED, GNN_ERR_CUDA, GNN_ERR_WORKSPACE, \
     GNN_ERR_INPUT_CHECK = range(6)
@@ -57,8 +58,15 @@ class _PlanInfo(ctypes.Structure):
         ("nnz", ctypes.c_int64), ("num_chunks", ctypes.c_int64), ("num_blocks", ctypes.c_int64)]
 
 
+class ReorderOpts(ctypes.Structure):
+    """gnn_reorder_opts_t; zero fields take defaults (3 levels, 20 passes, 1e-6, 1.0)."""
+    _fields_ = [("max_levels", ctypes.c_int32), ("max_passes", ctypes.c_int32),
+                ("min_gain", ctypes.c_double), ("resolution", ctypes.c_double)]
+
+
 EXPORTS = ["gnn_plan_workspace_bytes", "gnn_plan_create", "gnn_plan_info", "gnn_plan_arrays",
            "gnn_plan_destroy", "gnn_spmm", "gnn_sddmm", "gnn_shard_rows", "gnn_shard_edges",
+           "gnn_reorder_gcr", "gnn_permute_graph", "gnn_permute_rows",
            "gnn_csr_to_coo", "gnn_validate", "gnn_last_error", "gnn_version"]
 
 _lib = None
@@ -86,13 +94,17 @@ def lib():
     L.gnn_shard_rows.argtypes = [vp, i64, i32, vp]
     L.gnn_shard_edges.argtypes = [i64, i32, vp]
     L.gnn_csr_to_coo.argtypes = [vp, i64, i64, vp, vp]
+    L.gnn_reorder_gcr.argtypes = [vp, vp, i64, P(ReorderOpts), vp, vp, P(ctypes.c_double)]
+    L.gnn_permute_graph.argtypes = [vp, vp, vp, i64, vp, vp, vp, vp, vp]
+    L.gnn_permute_rows.argtypes = [vp, i64, i64, i64, vp, vp, i64, vp]
     L.gnn_validate.argtypes = [P(_Graph), vp]
     L.gnn_last_error.argtypes = []
     L.gnn_last_error.restype = ctypes.c_char_p
     L.gnn_version.argtypes = []
     L.gnn_version.restype = ctypes.c_char_p
     for f in ("gnn_plan_create", "gnn_plan_info", "gnn_plan_arrays", "gnn_spmm", "gnn_sddmm",
-              "gnn_shard_rows", "gnn_shard_edges", "gnn_csr_to_coo", "gnn_validate"):
+              "gnn_shard_rows", "gnn_shard_edges", "gnn_csr_to_coo", "gnn_validate",
+              "gnn_reorder_gcr", "gnn_permute_graph", "gnn_permute_rows"):
         getattr(L, f).restype = st
     _lib = L
     return L
@@ -277,3 +289,50 @@ def csr_to_coo(row_ptr: torch.Tensor, row_base: int = 0, stream=None) -> torch.T
 def validate(graph: DeviceGraph, stream=None) -> None:
     g = graph.desc()
     _check(lib().gnn_validate(ctypes.byref(g), _stream(stream)))
+
+
+# ---------------------------------------------------------------- reorder ---
+def reorder_gcr(row_ptr, col_ind, max_levels=0, max_passes=0, min_gain=0.0, resolution=0.0):
+    """gnn_reorder_gcr (host): Louvain-based GCR permutation of a square symmetric graph.
+    Returns (perm, community, modularity) with perm[old] = new."""
+    rp = np.ascontiguousarray(row_ptr, dtype=np.int32)
+    ci = np.ascontiguousarray(col_ind, dtype=np.int32)
+    n = rp.shape[0] - 1
+    perm = np.empty(n, np.int32)
+    comm = np.empty(n, np.int32)
+    q = ctypes.c_double(0.0)
+    o = ReorderOpts(max_levels, max_passes, min_gain, resolution)
+    _check(lib().gnn_reorder_gcr(rp.ctypes.data, ci.ctypes.data, n, ctypes.byref(o),
+                                 perm.ctypes.data, comm.ctypes.data, ctypes.byref(q)))
+    return perm, comm, q.value
+
+
+def permute_graph(row_ptr, col_ind, val, perm):
+    """gnn_permute_graph (host): S' = P S P^T -> (row_ptr, row_ind, col_ind, val)."""
+    rp = np.ascontiguousarray(row_ptr, dtype=np.int32)
+    ci = np.ascontiguousarray(col_ind, dtype=np.int32)
+    v = None if val is None else np.ascontiguousarray(val, dtype=np.float32)
+    pm = np.ascontiguousarray(perm, dtype=np.int32)
+    n = rp.shape[0] - 1
+    nnz = int(rp[-1]) - int(rp[0])
+    orp = np.empty(n + 1, np.int32)
+    ori = np.empty(nnz, np.int32)
+    oci = np.empty(nnz, np.int32)
+    ov = None if v is None else np.empty(nnz, np.float32)
+    _check(lib().gnn_permute_graph(rp.ctypes.data, ci.ctypes.data,
+                                   None if v is None else v.ctypes.data, n, pm.ctypes.data,
+                                   orp.ctypes.data, ori.ctypes.data, oci.ctypes.data,
+                                   None if ov is None else ov.ctypes.data))
+    return orp, ori, oci, ov
+
+
+def permute_rows(X: torch.Tensor, perm: torch.Tensor, out: torch.Tensor | None = None,
+                 stream=None) -> torch.Tensor:
+    """gnn_permute_rows (device): out[perm[i]] = X[i]."""
+    _dense(X, "X")
+    if out is None:
+        out = torch.empty_like(X)
+    perm = perm.to(device=X.device, dtype=torch.int32).contiguous()
+    _check(lib().gnn_permute_rows(_ptr(X), X.stride(0), X.shape[0], X.shape[1], _ptr(perm),
+                                  _ptr(out), out.stride(0), _stream(stream)))
+    return out

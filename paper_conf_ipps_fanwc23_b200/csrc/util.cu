@@ -84,6 +84,20 @@ __global__ void validate_kernel(gnn_graph_t g, unsigned long long *bad) {
   }
 }
 
+// one warp per row: coalesced copy of K floats to the permuted row
+__global__ void permute_rows_kernel(const float *__restrict__ X, int64_t ldx, int64_t n,
+                                    int64_t K, const int32_t *__restrict__ perm,
+                                    float *__restrict__ Y, int64_t ldy) {
+  const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t i = warp; i < n; i += nwarps) {
+    const float *x = X + i * ldx;
+    float *y = Y + (int64_t)perm[i] * ldy;
+    for (int64_t k = lane; k < K; k += 32) y[k] = x[k];
+  }
+}
+
 }  // namespace gnn
 
 using namespace gnn;
@@ -141,6 +155,22 @@ GNN_API gnn_status_t gnn_csr_to_coo(const int32_t *row_ptr, int64_t M, int64_t r
                                                                            row_ind);
   cudaError_t e = cudaGetLastError();
   return e == cudaSuccess ? GNN_OK : cuda_fail(e, "csr_to_coo launch");
+}
+
+GNN_API gnn_status_t gnn_permute_rows(const float *X, int64_t ldx, int64_t n, int64_t K,
+                                      const int32_t *perm, float *Y, int64_t ldy,
+                                      gnn_stream_t stream) {
+  if (n < 0 || K < 1 || (n > 0 && (!X || !Y || !perm || ldx < K || ldy < K)))
+    return fail(GNN_ERR_INVALID_ARG, "gnn_permute_rows: bad arguments");
+  if (n == 0) return GNN_OK;
+  DeviceInfo d;
+  if (gnn_status_t st = device_info(&d)) return st;
+  int64_t blocks = (n * 32 + 255) / 256;
+  if (blocks > (int64_t)d.num_sms * 32) blocks = (int64_t)d.num_sms * 32;
+  permute_rows_kernel<<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>(X, ldx, n, K, perm, Y,
+                                                                         ldy);
+  cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? GNN_OK : cuda_fail(e, "permute_rows launch");
 }
 
 GNN_API gnn_status_t gnn_validate(const gnn_graph_t *g, gnn_stream_t stream) {

@@ -110,7 +110,19 @@ def test_block_shape_and_alpha(wpb, alpha):
 def test_val_none_and_padded_pitch():
     g = gen.powerlaw_graph(3000, 40000, seed=301)
     run_full(g, 64, with_val=False)
-    run_full(g, 64, ld_pad=12)
+    run_full(g, 64, ld_pad=16)            # pitch 80: a multiple of VW = 8
+    run_full(g, 64, ld_pad=12, force_vw=4)  # pitch 76 needs a narrower vector width
+
+
+def test_pitch_incompatible_with_vector_width_is_unsupported():
+    g = gen.powerlaw_graph(500, 5000, seed=302)
+    dg = upload(g)
+    p = gs.plan(dg, 64)
+    assert p.info()["vw_feat"] == 8
+    A = torch.zeros((g.N, 76), device=DEV)[:, :64]
+    with pytest.raises(gs.GnnError) as e:
+        gs.spmm(p, dg, A)
+    assert e.value.status == gs.GNN_ERR_UNSUPPORTED
 
 
 def test_empty_rows_rectangular_duplicates():
@@ -320,3 +332,30 @@ def test_csr_to_coo_matches_oracle():
     rp = torch.from_numpy(g.row_ptr).to(DEV)
     ri = gs.csr_to_coo(rp).cpu().numpy()
     assert np.array_equal(ri, oracle.csr_to_coo(g.row_ptr))
+
+
+def test_gcr_reordered_graph_equivariance():
+    """SpMM(P S P^T, P X) = P SpMM(S, X) and SDDMM outputs move with their edges, on
+    the GCR-reordered graph (gnn_reorder_gcr + gnn_permute_graph + gnn_permute_rows)."""
+    g = gen.powerlaw_graph(20000, 400000, gamma=2.3, n_comm=20, mu=0.3, seed=5)
+    perm, comm, q = gs.reorder_gcr(g.row_ptr, g.col_ind)
+    rp, ri, ci, v = gs.permute_graph(g.row_ptr, g.col_ind, g.val, perm)
+    gp = gen.Graph(g.M, g.N, rp, ri, ci, v)
+    K = 64
+    X = _x(70, g.N, K)
+    Xd = torch.from_numpy(X).to(DEV)
+    Xp = gs.permute_rows(Xd, torch.from_numpy(perm))
+    torch.cuda.synchronize()
+    assert torch.equal(Xp[torch.from_numpy(perm).long().to(DEV)], Xd)
+    dgp = upload(gp)
+    p = gs.plan(dgp, K)
+    check_plan(p, gp, K)
+    Op = gs.spmm(p, dgp, Xp).cpu().numpy()
+    ref, T = oracle.spmm(g.row_ind, g.col_ind, g.val, X, M=g.M)
+    assert_within(Op[perm], ref, T, what="reordered spmm")
+    Ep = gs.sddmm(p, dgp, Xp, Xp).cpu().numpy()
+    r2, T2 = oracle.sddmm(g.row_ind, g.col_ind, g.val, X, X)
+    newkey = gp.row_ind.astype(np.int64) * g.N + gp.col_ind
+    oldkey = perm[g.row_ind].astype(np.int64) * g.N + perm[g.col_ind]
+    pos = np.searchsorted(newkey, oldkey)
+    assert_within(Ep[pos], r2, T2, what="reordered sddmm")

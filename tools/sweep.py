@@ -36,10 +36,18 @@ for K in (32, 64, 128, 256):
                 float((np.abs(E - r2) / np.maximum(T2, 1e-300)).max()))
 res["parity_worst_err_over_T"] = worst
 g = configs.make_graph(WL)
+perm = None
+if REORDER:
+    perm, comm, q = gs.reorder_gcr(g.row_ptr, g.col_ind)
+    rp, ri, ci, v = gs.permute_graph(g.row_ptr, g.col_ind, g.val, perm)
+    g = gen.Graph(g.M, g.N, rp, ri, ci, v)
+    res["modularity"] = q
 dg = gs.DeviceGraph.from_arrays(g.M, g.N, g.row_ind, g.col_ind, g.val, g.row_ptr)
 flush = torch.empty(64 * 1024 * 1024, device="cuda")
 for K, fvw in [(k, 0) for k in KS] + [(k, 8) for k in KS if VW8 and k % 8 == 0 and k < 256]:
     X = torch.from_numpy(configs.make_features(WL, g.N, K)).cuda()
+    if perm is not None:
+        X = gs.permute_rows(X, torch.from_numpy(perm))
     O = torch.empty((g.M, K), device="cuda"); E = torch.empty(g.nnz, device="cuda")
     p = gs.plan(dg, K, force_vw=fvw)
     ts, td = [], []
@@ -62,10 +70,11 @@ def main():
     ap.add_argument("--K", default="32,64,128,256")
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--vw8", action="store_true")
+    ap.add_argument("--reorder", action="store_true")
     ap.add_argument("libs", nargs="+")
     a = ap.parse_args()
     code = CHILD.replace("ROOT", repr(ROOT)).replace("WL", repr(a.workload)).replace(
-        "KS", repr([int(k) for k in a.K.split(",")])).replace("REPS", str(a.reps)).replace("VW8", str(a.vw8))
+        "KS", repr([int(k) for k in a.K.split(",")])).replace("REPS", str(a.reps)).replace("VW8", str(a.vw8)).replace("REORDER", str(a.reorder))
     for lib in a.libs:
         env = dict(os.environ, GNN_LIB_PATH=os.path.abspath(lib))
         r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
