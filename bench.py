@@ -162,6 +162,8 @@ def gcr_reorder(g):
 
 def build_graph(name):
     from gen import configs
+    if name == "C3":
+        return configs.make_c3(0)
     if name in configs.CONFIGS:
         return configs.make_graph(name)
     raise SystemExit(f"unknown workload {name}")
@@ -171,11 +173,16 @@ def parse_ks(s, name):
     from gen import configs
     if s:
         return [int(x) for x in s.split(",")]
+    if name == "C3":
+        return [128]
     return configs.CONFIGS[name]["K"]
 
 
 # ------------------------------------------------------------ our impl ------
-def run_ours(args):
+def time_path(args, g, perm, name, Ks, dev, world, rank):
+    """Resident graph + features for this rank's shard; W warm-up steps, then K timed
+    steps (CUDA events per kernel on the launching stream, L2 flushed between steps
+    outside the events).  Returns per-kernel times, this rank's bytes/flops, launches."""
     import torch
     import torch.distributed as dist
 
@@ -183,31 +190,11 @@ def run_ours(args):
     from gen import configs
     from paper_conf_ipps_fanwc23_b200 import dist as gdist
 
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
-    if world > 1:
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-        ncores = os.cpu_count() or 1
-        os.environ.setdefault("OMP_NUM_THREADS", str(max(1, ncores // world)))
-    dev = torch.device("cuda", local if world > 1 else 0)
-    torch.cuda.set_device(dev)
-    gs.lib()
-
-    name = args.workload
-    Ks = parse_ks(args.K, name)
-    t0 = time.time()
-    g = build_graph(name)
-    gen_s = time.time() - t0
-    perm, reorder_info = None, None
-    if args.reorder:
-        g, perm, reorder_info = gcr_reorder(g)
-    P, p = world, rank
+    P = world
     spec = gdist.shard_spec(g.row_ptr, g.N, rank, world)
     full = gs.DeviceGraph.from_arrays(g.M, g.N, g.row_ind, g.col_ind, g.val, g.row_ptr, device=dev)
     spg, sdg = gdist.local_graphs(full, spec)
-    # X: replicated (generated on every rank: deterministic) or all-gathered
+    perm_d = None if perm is None else torch.from_numpy(perm).to(dev)
     X, Xown = {}, {}
     for K in Ks:
         if args.xmode == "allgather" and P > 1:
@@ -217,18 +204,18 @@ def run_ours(args):
             X[K] = torch.empty((spec.xblk * P, K), dtype=torch.float32, device=dev)
         else:
             X[K] = torch.from_numpy(configs.make_features(name, g.N, K)).to(dev)
-            if perm is not None:  # X' = P X (same features, relabelled nodes)
-                X[K] = gs.permute_rows(X[K], torch.from_numpy(perm))
+        if perm_d is not None:  # X' = P X (same features, relabelled nodes)
+            if K in Xown:
+                raise SystemExit("--reorder with --xmode allgather is not supported")
+            X[K] = gs.permute_rows(X[K], perm_d)
     O = {K: torch.empty((spg.M, K), dtype=torch.float32, device=dev) for K in Ks}
     E = torch.empty(sdg.nnz, dtype=torch.float32, device=dev)
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
     stream = torch.cuda.current_stream()
-    same = (P == 1)
-
-    launches_per_step = 0
+    same = P == 1
+    counts = {"n": 0}
 
     def step(ev=None):
-        nonlocal launches_per_step
         n = 0
         for K in Ks:
             if args.xmode == "allgather" and P > 1:
@@ -249,21 +236,18 @@ def run_ours(args):
             n += 1 if sdg.nnz else 0
             if ev is not None:
                 ev[K][3].record(stream)
-        launches_per_step = n
+        counts["n"] = n
 
-    # warm-up
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
-
     ev = [{K: [torch.cuda.Event(enable_timing=True) for _ in range(4)] for K in Ks}
           for _ in range(args.steps)]
     clk = ClockSampler(dev.index)
     clk.start()
     time.sleep(0.3)
-    step_ms = []
     for s in range(args.steps):
         flush.fill_(float(s))  # L2 flush between timed steps (outside the events)
         torch.cuda.synchronize()
@@ -273,6 +257,7 @@ def run_ours(args):
         torch.cuda.synchronize()
     clocks = clk.stop()
     per = {K: {"plan": [], "spmm": [], "sddmm": []} for K in Ks}
+    step_ms = []
     for s in range(args.steps):
         tot = 0.0
         for K in Ks:
@@ -283,68 +268,128 @@ def run_ours(args):
             per[K]["sddmm"].append(c)
             tot += a + b + c
         step_ms.append(tot)
-    my_ms = float(sum(step_ms))
-
-    # bytes / flops of this rank's kernels
-    my_bytes = 0
-    my_flops = 0
-    detail = {}
+    my_bytes, my_flops, detail = 0, 0, {}
     for K in Ks:
-        b_sp = spmm_bytes(spg.nnz, spg.M, K)
-        b_sd = sddmm_bytes(sdg.nnz, g.M, K) if not same else sddmm_bytes(spg.nnz, spg.M, K)
         info = gs.plan(spg, K).info()
-        b_pl = plan_bytes(info["num_chunks"])
-        my_bytes += b_sp + b_sd + b_pl
+        b_sp = spmm_bytes(spg.nnz, spg.M, K)
+        b_sd = sddmm_bytes(sdg.nnz, g.M if not same else spg.M, K)
+        my_bytes += b_sp + b_sd + plan_bytes(info["num_chunks"])
         my_flops += spmm_flops(spg.nnz, K) + sddmm_flops(sdg.nnz, K)
-        t_sp = statistics.mean(per[K]["spmm"])
-        t_sd = statistics.mean(per[K]["sddmm"])
-        t_pl = statistics.mean(per[K]["plan"])
+        t_sp, t_sd = statistics.mean(per[K]["spmm"]), statistics.mean(per[K]["sddmm"])
         detail[f"K{K}"] = {
             "chunk": info["chunk"], "vw_feat": info["vw_feat"], "lanes": info["lanes"],
             "active_blocks_per_sm": info["active_blocks_per_sm"],
-            "plan_ms": round(t_pl, 4), "spmm_ms": round(t_sp, 4), "sddmm_ms": round(t_sd, 4),
-            "spmm_GBps": round(b_sp / t_sp / 1e6, 1), "sddmm_GBps": round(b_sd / t_sd / 1e6, 1),
+            "plan_ms": round(statistics.mean(per[K]["plan"]), 4), "spmm_ms": round(t_sp, 4),
+            "sddmm_ms": round(t_sd, 4), "spmm_GBps": round(b_sp / t_sp / 1e6, 1),
+            "sddmm_GBps": round(b_sd / t_sd / 1e6, 1),
             "spmm_GFLOPs": round(spmm_flops(spg.nnz, K) / t_sp / 1e6, 1),
             "sddmm_GFLOPs": round(sddmm_flops(sdg.nnz, K) / t_sd / 1e6, 1),
-            "spmm_hbm_compulsory_GBps": round(hbm_compulsory(spg.nnz, spg.M, g.N, K, "spmm")
-                                              / t_sp / 1e6, 1),
+            "spmm_hbm_compulsory_GBps": round(
+                hbm_compulsory(spg.nnz, spg.M, g.N, K, "spmm") / t_sp / 1e6, 1),
         }
+    out = {"per": per, "step_ms": step_ms, "bytes": my_bytes, "flops": my_flops,
+           "detail": detail, "clocks": clocks, "launches": counts["n"], "spg": spg, "sdg": sdg,
+           "full": full}
+    return out
 
-    # aggregate over ranks: sum of work, max of time
+
+def init_dist(world, local):
+    """One process per GPU; NCCL over NVLink for the data path.  GNN_BENCH_BACKEND=gloo
+    runs the multi-rank logic with several ranks sharing one GPU (smoke tests only)."""
+    import torch
+    import torch.distributed as dist
+    dev = torch.device("cuda", local % max(1, torch.cuda.device_count()))
+    torch.cuda.set_device(dev)
     if world > 1:
-        t = torch.tensor([my_ms, float(my_bytes), float(my_flops)], dtype=torch.float64,
-                         device=dev)
-        mx = t.clone()
+        backend = os.environ.get("GNN_BENCH_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
+        ncores = os.cpu_count() or 1
+        os.environ.setdefault("OMP_NUM_THREADS", str(max(1, ncores // world)))
+    return dev
+
+
+def aggregate(r, args, world, dev):
+    import torch
+    import torch.distributed as dist
+    my_ms = float(sum(r["step_ms"]))
+    if world > 1:
+        t = torch.tensor([my_ms, float(r["bytes"]), float(r["flops"])], dtype=torch.float64,
+                         device=dev if dist.get_backend() == "nccl" else "cpu")
+        mx, sm = t.clone(), t.clone()
         dist.all_reduce(mx, op=dist.ReduceOp.MAX)
-        sm = t.clone()
         dist.all_reduce(sm, op=dist.ReduceOp.SUM)
-        tot_ms, tot_bytes, tot_flops = float(mx[0]), float(sm[1]), float(sm[2])
+        return float(mx[0]), float(sm[1]) * args.steps, float(sm[2]) * args.steps
+    return my_ms, float(r["bytes"]) * args.steps, float(r["flops"]) * args.steps
+
+
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ipps_fanwc23_b200 as gs
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    dev = init_dist(world, local)
+    gs.lib()
+    if args.workload == "C3":
+        return run_c3(args, dev, world, rank)
+
+    name = args.workload
+    Ks = parse_ks(args.K, name)
+    t0 = time.time()
+    g0 = build_graph(name)
+    gen_s = time.time() - t0
+    reorder = args.reorder and args.xmode != "allgather"
+    if reorder:
+        g, perm, reorder_info = gcr_reorder(g0)
     else:
-        tot_ms, tot_bytes, tot_flops = my_ms, float(my_bytes), float(my_flops)
-    tot_bytes *= args.steps
-    tot_flops *= args.steps
+        g, perm, reorder_info = g0, None, None
+
+    r = time_path(args, g, perm, name, Ks, dev, world, rank)
+    tot_ms, tot_bytes, tot_flops = aggregate(r, args, world, dev)
     value = tot_bytes / (tot_ms * 1e-3) / 1e9
+    spg, sdg, per = r["spg"], r["sdg"], r["per"]
 
     # dominant kernel (largest share of this rank's step time) -> roofline
     shares = {(K, kind): statistics.mean(per[K][kind]) for K in Ks for kind in ("spmm", "sddmm")}
     (dK, dkind), dms = max(shares.items(), key=lambda kv: kv[1])
-    dbytes = spmm_bytes(spg.nnz, spg.M, dK) if dkind == "spmm" else sddmm_bytes(sdg.nnz, g.M, dK)
+    dbytes = spmm_bytes(spg.nnz, spg.M, dK) if dkind == "spmm" else \
+        sddmm_bytes(sdg.nnz, g.M if world > 1 else spg.M, dK)
     peak, peak_src = load_peaks()
     achieved = dbytes / (dms * 1e-3) / 1e9
-    traffic = load_ncu_traffic().get(f"{name}:{dkind}:K{dK}")
+    tkey = f"{name}{'+gcr' if reorder else ''}:{dkind}:K{dK}"
+    traffic = load_ncu_traffic().get(tkey)
+    my_ms = float(sum(r["step_ms"]))
     roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                 "frac": round(achieved / peak, 4), "traffic": traffic,
-                "kernel": f"{dkind} K={dK} ({name})", "peak_source": peak_src,
-                "algorithmic_bytes_per_launch": int(dbytes),
+                "kernel": f"{dkind} K={dK} ({name}{', GCR-reordered' if reorder else ''})",
+                "peak_source": peak_src, "algorithmic_bytes_per_launch": int(dbytes),
+                "byte_model": "per nnz 12 B sparse (+4 B out for SDDMM) + 4K B gathered "
+                              "feature row; per row 4K B (SURVEY.md §8(d))",
                 "share_of_step": round(dms / (my_ms / args.steps), 4),
                 "hbm_compulsory_frac": round(
                     hbm_compulsory(spg.nnz if dkind == "spmm" else sdg.nnz, spg.M, g.N, dK,
-                                   dkind) / (dms * 1e-3) / 1e9 / peak, 4)}
-
-    # e2e through the public API with host buffers (pinned), rank 0's numbers
-    e2e = run_e2e(args, g, Ks, dev, full if P == 1 else None) if (P == 1 and not args.no_e2e) \
-        else None
-
+                                   dkind) / (dms * 1e-3) / 1e9 / peak, 4),
+                "traffic_key": tkey}
+    launches, clocks, detail = r["launches"], r["clocks"], r["detail"]
+    alt = None
+    if reorder and args.compare:
+        del r
+        torch.cuda.empty_cache()
+        r2 = time_path(args, g0, None, name, Ks, dev, world, rank)
+        ms2, b2, f2 = aggregate(r2, args, world, dev)
+        alt = {"value": round(b2 / (ms2 * 1e-3) / 1e9, 2), "unit": "GB/s",
+               "ms_per_step": round(ms2 / args.steps, 4), "kernels": r2["detail"]}
+        del r2
+        torch.cuda.empty_cache()
+    e2e = None
+    if world == 1 and not args.no_e2e:
+        e2e = run_e2e(args, g, Ks, dev, perm)
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
         cpu = cpu_baseline(g, Ks, args.cpu_seconds, name)
@@ -355,8 +400,9 @@ def run_ours(args):
             "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": round(tot_ms / args.steps, 4), "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": {"workload": f"{name}: {WORKLOAD_DESC.get(name, name)}", "K": Ks,
-                       "nnz": g.nnz, "M": g.M, "N": g.N, "degree": g.degree_stats(),
+            "config": {"workload": f"{name}: {WORKLOAD_DESC.get(name, name)}"
+                                   + (", GCR-reordered offline" if reorder else ""),
+                       "K": Ks, "nnz": g.nnz, "M": g.M, "N": g.N, "degree": g.degree_stats(),
                        "step": "per K: plan (GPU plan kernel) + SpMM + SDDMM",
                        "l2": "flushed between timed steps (256 MiB write, outside events)",
                        "parallelism": f"rowshard-spmm/edgeshard-sddmm x{world}",
@@ -364,8 +410,8 @@ def run_ours(args):
                        "reorder": reorder_info},
             "gflops": round(tot_flops / (tot_ms * 1e-3) / 1e9, 1),
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
-            "gpu_launches": launches_per_step * args.steps, "clocks": clocks,
-            "kernels": detail,
+            "gpu_launches": launches * args.steps, "clocks": clocks, "kernels": detail,
+            "no_reorder": alt,
         }
         print(json.dumps(line), flush=True)
     if world > 1:
@@ -373,7 +419,102 @@ def run_ours(args):
         dist.destroy_process_group()
 
 
-def run_e2e(args, g, Ks, dev, full):
+def run_c3(args, dev, world, rank):
+    """BASELINE.json configs[2]: GraphSAINT-style sampled subgraphs, a new graph every
+    step, K = 128, re-planned every step (plan + SpMM + SDDMM per step).  Subgraphs are
+    pre-generated and resident before timing; rank p takes subgraphs p, p+P, ...
+    (independent problems: weak scaling)."""
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ipps_fanwc23_b200 as gs
+    from gen import configs
+
+    Ks = parse_ks(args.K, "C4") if args.K else [128]
+    K = Ks[0]
+    nsub = max(1, args.c3_graphs)
+    mine = list(range(rank, nsub * world, world))
+    subs = []
+    for t in mine:
+        g = configs.make_c3(t)
+        dg = gs.DeviceGraph.from_arrays(g.M, g.N, g.row_ind, g.col_ind, g.val, g.row_ptr,
+                                        device=dev)
+        X = torch.from_numpy(configs.make_features("C3", g.N, K)).to(dev)
+        subs.append((g, dg, X, torch.empty((g.M, K), device=dev),
+                     torch.empty(g.nnz, device=dev)))
+    stream = torch.cuda.current_stream()
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
+
+    def one(i, ev=None):
+        g, dg, X, O, E = subs[i % len(subs)]
+        if ev:
+            ev[0].record(stream)
+        p = gs.plan(dg, K)
+        if ev:
+            ev[1].record(stream)
+        gs.spmm(p, dg, X, out=O)
+        if ev:
+            ev[2].record(stream)
+        gs.sddmm(p, dg, X, X, out=E)
+        if ev:
+            ev[3].record(stream)
+        return p
+
+    for i in range(args.warmup):
+        one(i)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    nsteps = args.steps
+    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(4)] for _ in range(nsteps)]
+    clk = ClockSampler(dev.index)
+    clk.start()
+    time.sleep(0.3)
+    nbytes, pl, sp, sd, chunks = 0, [], [], [], []
+    for s in range(nsteps):
+        flush.fill_(float(s))
+        torch.cuda.synchronize()
+        p = one(s, evs[s])
+        torch.cuda.synchronize()
+        g = subs[s % len(subs)][0]
+        nbytes += spmm_bytes(g.nnz, g.M, K) + sddmm_bytes(g.nnz, g.M, K)
+        chunks.append(p.info()["chunk"])
+        e = evs[s]
+        pl.append(e[0].elapsed_time(e[1]))
+        sp.append(e[1].elapsed_time(e[2]))
+        sd.append(e[2].elapsed_time(e[3]))
+    clocks = clk.stop()
+    my_ms = sum(pl) + sum(sp) + sum(sd)
+    if world > 1:
+        t = torch.tensor([my_ms, float(nbytes)], dtype=torch.float64)
+        mx, sm = t.clone(), t.clone()
+        dist.all_reduce(mx, op=dist.ReduceOp.MAX)
+        dist.all_reduce(sm, op=dist.ReduceOp.SUM)
+        tot_ms, tot_bytes = float(mx[0]), float(sm[1])
+    else:
+        tot_ms, tot_bytes = my_ms, float(nbytes)
+    if rank == 0:
+        line = {"metric": METRIC, "value": round(tot_bytes / (tot_ms * 1e-3) / 1e9, 2),
+                "unit": "GB/s", "n_gpus": world, "steps": nsteps, "warmup": args.warmup,
+                "ms_per_step": round(tot_ms / nsteps, 4), "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+                "config": {"workload": "C3: GraphSAINT-style sampled subgraphs (N~U[8k,50k], "
+                                       "avg degree U[15,30]), new graph + re-plan every step",
+                           "K": [K], "subgraphs_per_rank": len(subs),
+                           "l2": "flushed between timed steps (256 MiB write, outside events)"},
+                "c3": {"plan_ms_mean": round(statistics.mean(pl), 4),
+                       "spmm_ms_mean": round(statistics.mean(sp), 4),
+                       "sddmm_ms_mean": round(statistics.mean(sd), 4),
+                       "plan_share": round(sum(pl) / my_ms, 4),
+                       "chunks_chosen": sorted(set(chunks))},
+                "gpu_launches": 4 * nsteps, "clocks": clocks}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def run_e2e(args, g, Ks, dev, perm=None):
     """Same metric end to end through the public API: every step copies the graph
     arrays and X from pinned host memory, runs plan + SpMM + SDDMM, and copies O and the
     SDDMM output back to pinned host memory; all inside the CUDA-event timed region."""
@@ -384,7 +525,14 @@ def run_e2e(args, g, Ks, dev, full):
 
     pin = lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory()
     h_ri, h_ci, h_v = pin(g.row_ind), pin(g.col_ind), pin(g.val)
-    h_X = {K: pin(configs.make_features(args.workload, g.N, K)) for K in Ks}
+    def feats(K):
+        X = configs.make_features(args.workload, g.N, K)
+        if perm is not None:  # the reordered graph's features (same values, new row ids)
+            Xp = np.empty_like(X)
+            Xp[perm] = X
+            X = Xp
+        return X
+    h_X = {K: pin(feats(K)) for K in Ks}
     h_O = {K: torch.empty((g.M, K), dtype=torch.float32).pin_memory() for K in Ks}
     h_E = torch.empty(g.nnz, dtype=torch.float32).pin_memory()
     d_ri = torch.empty_like(h_ri, device=dev)
@@ -509,10 +657,14 @@ def main():
     ap.add_argument("--K", default="")
     ap.add_argument("--xmode", default="replicate", choices=["replicate", "allgather"])
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--c3-graphs", type=int, default=20)
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
-    ap.add_argument("--reorder", action="store_true",
-                    help="GCR-reorder the graph offline before timing (paper's full-graph setup)")
+    ap.add_argument("--no-reorder", dest="reorder", action="store_false",
+                    help="time the graph as generated (default: GCR-reordered offline first, "
+                         "the paper's full-graph setup)")
+    ap.add_argument("--no-compare", dest="compare", action="store_false",
+                    help="skip the extra timing of the un-reordered graph")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "ours":
         args.warmup = 3

@@ -359,3 +359,52 @@ def test_gcr_reordered_graph_equivariance():
     oldkey = perm[g.row_ind].astype(np.int64) * g.N + perm[g.col_ind]
     pos = np.searchsorted(newkey, oldkey)
     assert_within(Ep[pos], r2, T2, what="reordered sddmm")
+
+
+# ------------------------------------------------- full BASELINE.json sizes ---
+def _sampled_rows(g, n, seed):
+    """A row sample that always includes the heaviest rows (hubs split across many
+    chunks -> atomics), rows at chunk boundaries and random rows."""
+    rng = np.random.default_rng(seed)
+    deg = np.diff(g.row_ptr)
+    heavy = np.argsort(deg)[-8:]
+    rand = rng.choice(g.M, size=n, replace=False)
+    return np.unique(np.r_[heavy, rand, 0, g.M - 1])
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("name,Ks,reorder", [("C4", (32, 256), False), ("C4", (64, 128), True),
+                                             ("C5", (256,), True)])
+def test_full_size_sampled_parity(name, Ks, reorder):
+    """Full-size Reddit / products-shaped graphs, in bench.py's launch configuration
+    (default plan), checked on sampled output rows (SpMM) and edges (SDDMM) that the
+    oracle computes one by one, plus the global plan arrays bit-exactly."""
+    g = configs.make_graph(name)
+    perm = None
+    if reorder:
+        perm, _, _ = gs.reorder_gcr(g.row_ptr, g.col_ind)
+        rp, ri, ci, v = gs.permute_graph(g.row_ptr, g.col_ind, g.val, perm)
+        g = gen.Graph(g.M, g.N, rp, ri, ci, v)
+    dg = upload(g)
+    rows = _sampled_rows(g, 300, 1)
+    edges = np.unique(np.r_[np.random.default_rng(2).choice(g.nnz, 20000, replace=False),
+                            g.row_ptr[rows[:50]]])
+    for K in Ks:
+        X = configs.make_features(name, g.N, K)
+        Xd = torch.from_numpy(X).to(DEV)
+        p = gs.plan(dg, K)
+        check_plan(p, g, K)
+        O = gs.spmm(p, dg, Xd)
+        E = gs.sddmm(p, dg, Xd, Xd)
+        torch.cuda.synchronize()
+        ref, T = oracle.spmm_rows(g, X, rows)
+        assert_within(O[torch.from_numpy(rows).to(DEV)].cpu().numpy(), ref, T,
+                      what=f"{name} spmm K={K}")
+        r2 = np.empty(edges.size)
+        T2 = np.empty(edges.size)
+        for j, i in enumerate(edges):
+            a, b = oracle.sddmm(g.row_ind, g.col_ind, g.val, X, X, i0=int(i), i1=int(i) + 1)
+            r2[j], T2[j] = a[0], b[0]
+        assert_within(E[torch.from_numpy(edges).to(DEV)].cpu().numpy(), r2, T2,
+                      what=f"{name} sddmm K={K}")
+        del O, E, Xd

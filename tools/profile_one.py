@@ -21,11 +21,20 @@ def main():
     ap.add_argument("--K", default="32,256")
     ap.add_argument("--reps", type=int, default=1)
     ap.add_argument("--scale", type=float, default=1.0)
+    ap.add_argument("--reorder", action="store_true")
     a = ap.parse_args()
     g = configs.make_graph(a.workload, a.scale)
+    perm = None
+    if a.reorder:
+        import gen
+        perm, _, _ = gs.reorder_gcr(g.row_ptr, g.col_ind)
+        rp, ri, ci, v = gs.permute_graph(g.row_ptr, g.col_ind, g.val, perm)
+        g = gen.Graph(g.M, g.N, rp, ri, ci, v)
     dg = gs.DeviceGraph.from_arrays(g.M, g.N, g.row_ind, g.col_ind, g.val, g.row_ptr)
     for K in [int(k) for k in a.K.split(",")]:
         X = torch.from_numpy(configs.make_features(a.workload, g.N, K)).cuda()
+        if perm is not None:
+            X = gs.permute_rows(X, torch.from_numpy(perm))
         O = torch.empty((g.M, K), device="cuda")
         E = torch.empty(g.nnz, device="cuda")
         for _ in range(a.reps):
