@@ -18,21 +18,28 @@
 
 namespace gnn {
 
-// Rows in flight per lane (U) and register budget (min blocks of 512 threads per SM)
-// per instantiation, measured on C4 (profiles/r01_sweep4.txt): U = 8 with 256-bit loads,
-// except full-warp groups (L = 32, K >= 256) which prefer more resident warps (2 blocks,
-// U = 2).
-template <int VW, int L>
-struct SddmmShape {
-#if defined(GNN_SDDMM_DEPTH8)
-  static constexpr int depth = VW == 8 ? GNN_SDDMM_DEPTH8 : 8;
-#else
-  static constexpr int depth = (VW == 8 && L == 32) ? 2 : 8;
+// Lane mapping of SDDMM.  The plan's L lanes x VW columns cover a K-slice; SDDMM
+// splits them into R vectors per lane over a group of Lg = L / R lanes, so each dot
+// product is reduced over fewer lanes (fewer shuffles per nonzero) and 32/Lg nonzeros
+// are in flight per warp step; U = nonzeros per batch per group, U * R = 8 feature
+// vectors in flight per lane.  Measured on the GCR-reordered C4 (profiles/
+// r01_sweep8.txt): R = 2 from L = 8 on (K=64: 2.07 -> 1.94 ms, K=128: 4.82 -> 3.61 ms,
+// K=256: 8.85 -> 7.05 ms), R = 1 below.  GNN_SDDMM_R2_FROM / GNN_SDDMM_UR override.
+#ifndef GNN_SDDMM_R2_FROM
+#define GNN_SDDMM_R2_FROM 8  // smallest L that uses R = 2
 #endif
+#ifndef GNN_SDDMM_UR
+#define GNN_SDDMM_UR 8       // U * R: feature vectors in flight per lane
+#endif
+template <int VW, int L, int SMAX>
+struct SddmmShape {
+  static constexpr int R = (SMAX == 1 && L >= GNN_SDDMM_R2_FROM && L >= 2) ? 2 : 1;
+  static constexpr int Lg = L / R;
+  static constexpr int depth = GNN_SDDMM_UR / R > 1 ? GNN_SDDMM_UR / R : 1;
 #if defined(GNN_SDDMM_MINB)
   static constexpr int minb = GNN_SDDMM_MINB;
 #else
-  static constexpr int minb = (VW == 8 && L == 32) ? 2 : 1;
+  static constexpr int minb = 1;
 #endif
 };
 
@@ -91,17 +98,19 @@ __device__ __forceinline__ void reduce_scale_store(float (&part)[U], const float
 }
 
 template <int VW, int L, int VWS, int SMAX>
-__global__ void __launch_bounds__(kMaxThreads, (SMAX > 1 ? 1 : SddmmShape<VW, L>::minb))
+__global__ void __launch_bounds__(kMaxThreads, (SddmmShape<VW, L, SMAX>::minb))
     sddmm_kernel(const SparseArgs a, const float *__restrict__ A1, const int64_t lda1,
                  const float *__restrict__ A2T, const int64_t lda2, float *__restrict__ out) {
-  constexpr int G = 32 / L;
-  constexpr int T = L * VWS;
-  constexpr int U0 = SddmmShape<VW, L>::depth > VWS ? SddmmShape<VW, L>::depth : VWS;
+  using Sh = SddmmShape<VW, L, SMAX>;
+  constexpr int R = Sh::R, Lg = Sh::Lg;
+  constexpr int G = 32 / Lg;
+  constexpr int T = Lg * VWS;
+  constexpr int U0 = Sh::depth > VWS ? Sh::depth : VWS;
   constexpr int U = U0 < T ? U0 : T;
   static_assert(T % U == 0 && U % VWS == 0, "tile / prefetch shape");
   const int lane = threadIdx.x & 31;
-  const int g = lane / L;
-  const int l = lane & (L - 1);
+  const int g = lane / Lg;
+  const int l = lane & (Lg - 1);
   const int64_t c = ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * G + g;
   const bool item_ok = c < a.num_chunks;
   if (!__any_sync(kFull, item_ok)) return;
@@ -111,13 +120,16 @@ __global__ void __launch_bounds__(kMaxThreads, (SMAX > 1 ? 1 : SddmmShape<VW, L>
   const uint32_t ld2B = (uint32_t)lda2 * 4u;
   const char *__restrict__ A2b = reinterpret_cast<const char *>(A2T);
 
-  float a1[SMAX][VW];
+  // column of vector r of slice sl owned by lane l: (sl*L + r*Lg + l) * VW
+  float a1[SMAX][R][VW];
   int32_t cur[SMAX];  // row whose A1 slice is cached, per slice
 #pragma unroll
   for (int sl = 0; sl < SMAX; ++sl) {
     cur[sl] = -1;
 #pragma unroll
-    for (int v = 0; v < VW; ++v) a1[sl][v] = 0.f;
+    for (int r = 0; r < R; ++r)
+#pragma unroll
+      for (int v = 0; v < VW; ++v) a1[sl][r][v] = 0.f;
   }
 
   const int32_t *__restrict__ ri = a.row_ind + cs;
@@ -130,14 +142,14 @@ __global__ void __launch_bounds__(kMaxThreads, (SMAX > 1 ? 1 : SddmmShape<VW, L>
   ld_sparse_i32<VWS>(ci, l * VWS, n, 0, nc);
   ld_sparse_f32<VWS>(vi, l * VWS, n, nv);
 
-  auto load_a1 = [&](int32_t row) {
+  auto load_a1_slice = [&](int sl, int32_t row) {
+    const float *base = A1 + ((int64_t)row - a.row_base) * lda1;
 #pragma unroll
-    for (int sl = 0; sl < SMAX; ++sl) {
-      const int k0 = (sl * L + l) * VW;
-      if (sl < S && k0 < a.K)
-        ld_feat<VW>(A1 + ((int64_t)row - a.row_base) * lda1 + k0, a1[sl]);
-      cur[sl] = row;
+    for (int r = 0; r < R; ++r) {
+      const int k0 = (sl * L + r * Lg + l) * VW;
+      if (k0 < a.K) ld_feat<VW>(base + k0, a1[sl][r]);
     }
+    cur[sl] = row;
   };
 
   const int ntiles = (a.chunk + T - 1) / T;
@@ -155,10 +167,14 @@ __global__ void __launch_bounds__(kMaxThreads, (SMAX > 1 ? 1 : SddmmShape<VW, L>
       ld_sparse_i32<VWS>(ci, li, n, 0, nc);
       ld_sparse_f32<VWS>(vi, li, n, nv);
     }
-    const int32_t r_first = __shfl_sync(kFull, rr[0], 0, L);
-    const int32_t r_last = __shfl_sync(kFull, rr[VWS - 1], L - 1, L);
+    const int32_t r_first = __shfl_sync(kFull, rr[0], 0, Lg);
+    const int32_t r_last = __shfl_sync(kFull, rr[VWS - 1], Lg - 1, Lg);
     const bool fast = __all_sync(kFull, ((tb + T <= n) && r_first == r_last) || !item_ok);
-    if (fast && item_ok && r_first != cur[0]) load_a1(r_first);  // row switch at tile start
+    if (fast && item_ok && r_first != cur[0]) {  // row switch at the tile start
+#pragma unroll
+      for (int sl = 0; sl < SMAX; ++sl)
+        if (sl < S) load_a1_slice(sl, r_first);
+    }
 #pragma unroll 1
     for (int jj = 0; jj < T; jj += U) {
       int32_t rj[U];
@@ -167,40 +183,43 @@ __global__ void __launch_bounds__(kMaxThreads, (SMAX > 1 ? 1 : SddmmShape<VW, L>
 #pragma unroll
       for (int u = 0; u < U; ++u) {
         const int src = (jj + u) / VWS;
-        cj[u] = (uint32_t)__shfl_sync(kFull, cc[u % VWS], src, L);
-        vj[u] = __shfl_sync(kFull, vv[u % VWS], src, L);
-        rj[u] = fast ? r_first : __shfl_sync(kFull, rr[u % VWS], src, L);
+        cj[u] = (uint32_t)__shfl_sync(kFull, cc[u % VWS], src, Lg);
+        vj[u] = __shfl_sync(kFull, vv[u % VWS], src, Lg);
+        rj[u] = fast ? r_first : __shfl_sync(kFull, rr[u % VWS], src, Lg);
         part[u] = 0.f;
       }
       const int valid = n - (tb + jj);
 #pragma unroll
       for (int sl = 0; sl < SMAX; ++sl) {
         if (sl < S) {
-          const int k0 = (sl * L + l) * VW;
-          const bool col_ok = item_ok && k0 < a.K;
-          float x[U][VW];
+          float x[U][R][VW];
 #pragma unroll
           for (int u = 0; u < U; ++u) {
-            if (col_ok && (fast || u < valid)) {
-              ld_feat<VW>(reinterpret_cast<const float *>(A2b + (uint64_t)cj[u] * ld2B) + k0,
-                          x[u]);
-            } else {
+            const float *rowp =
+                reinterpret_cast<const float *>(A2b + (uint64_t)cj[u] * ld2B);
 #pragma unroll
-              for (int v = 0; v < VW; ++v) x[u][v] = 0.f;
+            for (int r = 0; r < R; ++r) {
+              const int k0 = (sl * L + r * Lg + l) * VW;
+              if (item_ok && k0 < a.K && (fast || u < valid)) {
+                ld_feat<VW>(rowp + k0, x[u][r]);
+              } else {
+#pragma unroll
+                for (int v = 0; v < VW; ++v) x[u][r][v] = 0.f;
+              }
             }
           }
 #pragma unroll
           for (int u = 0; u < U; ++u) {
-            if (!fast && col_ok && u < valid && rj[u] != cur[sl]) {
+            if (!fast && item_ok && u < valid && rj[u] != cur[sl]) {
               // row-switch procedure: load the new A1 row (Algo 4 lines 8-11)
-              cur[sl] = rj[u];
-              ld_feat<VW>(A1 + ((int64_t)rj[u] - a.row_base) * lda1 + k0, a1[sl]);
+              load_a1_slice(sl, rj[u]);
             }
-            part[u] = dot_acc<VW>(part[u], a1[sl], x[u]);
+#pragma unroll
+            for (int r = 0; r < R; ++r) part[u] = dot_acc<VW>(part[u], a1[sl][r], x[u][r]);
           }
         }
       }
-      reduce_scale_store<U, L>(part, vj, l, oc + tb + jj, item_ok ? valid : 0);
+      reduce_scale_store<U, Lg>(part, vj, l, oc + tb + jj, item_ok ? valid : 0);
     }
   }
 }
@@ -210,6 +229,9 @@ using SddmmFn = void (*)(const SparseArgs, const float *__restrict__, const int6
 
 template <int VW, int L, int SMAX>
 SddmmFn pick_sddmm_vws(int vws) {
+  // a batch must cover whole sparse vectors: narrow the sparse loads when U < vw_sparse
+  constexpr int D = SddmmShape<VW, L, SMAX>::depth;
+  while (vws > D) vws >>= 1;
   switch (vws) {
     case 1: return sddmm_kernel<VW, L, 1, SMAX>;
     case 2: return sddmm_kernel<VW, L, 2, SMAX>;
@@ -230,6 +252,28 @@ SddmmFn pick_sddmm_l(int L, int vws, int S) {
   }
   return nullptr;
 }
+// lanes per dot product of the instantiation pick_sddmm returns
+template <int VW>
+int group_lanes_vw(int L, int S) {
+  if (S > 1) return SddmmShape<VW, 32, 4>::Lg;
+  switch (L) {
+    case 1: return SddmmShape<VW, 1, 1>::Lg;
+    case 2: return SddmmShape<VW, 2, 1>::Lg;
+    case 4: return SddmmShape<VW, 4, 1>::Lg;
+    case 8: return SddmmShape<VW, 8, 1>::Lg;
+    case 16: return SddmmShape<VW, 16, 1>::Lg;
+    default: return SddmmShape<VW, 32, 1>::Lg;
+  }
+}
+int sddmm_group_lanes(int vw, int L, int S) {
+  switch (vw) {
+    case 1: return group_lanes_vw<1>(L, S);
+    case 2: return group_lanes_vw<2>(L, S);
+    case 4: return group_lanes_vw<4>(L, S);
+    default: return group_lanes_vw<8>(L, S);
+  }
+}
+
 SddmmFn pick_sddmm(int vw, int L, int vws, int S) {
   if (S > 4) return nullptr;
   switch (vw) {
@@ -266,7 +310,8 @@ extern "C" GNN_API gnn_status_t gnn_sddmm(gnn_plan_t plan, const gnn_graph_t *g,
                 in.slices, VW);
   const SparseArgs a = make_args(p, g);
   const int threads = in.warps_per_block * 32;
-  const int64_t per_block = (int64_t)in.groups * in.warps_per_block;
+  const int lg = sddmm_group_lanes(VW, in.lanes, in.slices);
+  const int64_t per_block = (int64_t)(32 / lg) * in.warps_per_block;
   const int64_t blocks = (a.num_chunks + per_block - 1) / per_block;
   f<<<(unsigned)blocks, threads, 0, (cudaStream_t)stream>>>(a, A1, lda1, A2T, lda2, out);
   cudaError_t e = cudaGetLastError();

@@ -17,6 +17,7 @@
 // rows shared with a neighbouring chunk (plan flags) a vector atomic add into a row
 // zeroed beforehand by spmm_prezero_kernel.  Empty rows are written as zeros by the
 // chunk that precedes them, so O is fully overwritten without a memset.
+#include <atomic>
 #include <climits>
 
 #include "device.cuh"
@@ -276,11 +277,22 @@ SpmmFn pick_spmm(int vw, int L, int vws) {
   return nullptr;
 }
 
+// Cached per (device, vw, lanes, wpb): the occupancy API is a host-side query but not
+// free, and plans are rebuilt every step in graph-sampling training (C3).
 int spmm_active_blocks_per_sm(int vw, int lanes, int wpb) {
+  static std::atomic<int> cache[64][4][6][17];
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64 || wpb < 1 || wpb > 16) return 0;
+  const int iv = vw == 1 ? 0 : vw == 2 ? 1 : vw == 4 ? 2 : 3;
+  int il = 0;
+  while ((1 << il) < lanes && il < 5) ++il;
+  std::atomic<int> &slot = cache[dev][iv][il][wpb];
+  int n = slot.load(std::memory_order_relaxed);
+  if (n > 0) return n;
   SpmmFn f = pick_spmm(vw, lanes, 1);
   if (!f) return 0;
-  int n = 0;
   if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, f, wpb * 32, 0) != cudaSuccess) return 0;
+  slot.store(n, std::memory_order_relaxed);
   return n;
 }
 
