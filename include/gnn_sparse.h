@@ -81,6 +81,7 @@ typedef struct {
   int32_t vw_feat;         /* feature-row vector width VW (floats per lane)         */
   int32_t vw_sparse;       /* sparse-array vector width (HVMA): 1, 2 or 4     */
   int32_t lanes;           /* L: lanes per chunk-slice                              */
+  int32_t vecs;            /* R: VW-wide vectors per lane per slice (1 or 2)         */
   int32_t slices;          /* S: K-slices per chunk                                 */
   int32_t groups;          /* G = 32 / L chunk-slices per warp                      */
   int32_t warps_per_block;

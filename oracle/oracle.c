@@ -94,11 +94,12 @@ int oracle_plan(int64_t nnz, const int32_t *row_ind, int32_t K, int32_t alpha,
   } else {
     vw = 1;
   }
-  /* step 2: lanes per chunk-slice, slices, groups per warp */
-  int64_t need = cdiv(K, vw);
+  /* step 2: vectors per lane, lanes per chunk-slice, slices, groups per warp */
+  int64_t need = cdiv(K, vw);          /* VW-wide vectors in a feature row */
+  int32_t R = need >= 16 ? 2 : 1;
   int32_t L = 1;
-  while (L < need && L < 32) L *= 2;
-  int32_t S = (int32_t)cdiv(K, (int64_t)L * vw);
+  while (L < cdiv(need, R) && L < 32) L *= 2;
+  int32_t S = (int32_t)cdiv(K, (int64_t)L * R * vw);
   int32_t G = 32 / L;
   /* step 3: FullWaveSize = NumSM x ActiveblocksPerSM (Eqs. 3-4) */
   int64_t FW = (int64_t)num_sms * active_blocks_per_sm;
@@ -119,6 +120,7 @@ int oracle_plan(int64_t nnz, const int32_t *row_ind, int32_t K, int32_t alpha,
   info->vw_feat = vw;
   info->vw_sparse = vws;
   info->lanes = L;
+  info->vecs = R;
   info->slices = S;
   info->groups = G;
   info->warps_per_block = warps_per_block;

@@ -53,7 +53,7 @@ class PlanOpts(ctypes.Structure):
 
 class _PlanInfo(ctypes.Structure):
     _fields_ = [(n, ctypes.c_int32) for n in (
-        "chunk", "vw_feat", "vw_sparse", "lanes", "slices", "groups", "warps_per_block",
+        "chunk", "vw_feat", "vw_sparse", "lanes", "vecs", "slices", "groups", "warps_per_block",
         "active_blocks_per_sm", "num_sms", "alpha", "K")] + [
         ("nnz", ctypes.c_int64), ("num_chunks", ctypes.c_int64), ("num_blocks", ctypes.c_int64)]
 

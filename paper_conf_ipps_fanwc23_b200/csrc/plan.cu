@@ -52,16 +52,17 @@ gnn_status_t make_info(int64_t nnz, int32_t K, const gnn_plan_opts_t *opts,
   } else {
     vw = 1;
   }
-  // step 2: lanes per chunk-slice, slices, chunk-slices per warp
-  const int64_t need = cdiv(K, vw);
+  // step 2: vectors per lane, lanes per chunk-slice, slices, chunk-slices per warp
+  const int64_t need = cdiv(K, vw);  // VW-wide vectors in a feature row
+  const int32_t R = need >= 16 ? 2 : 1;
   int32_t L = 1;
-  while (L < need && L < 32) L *= 2;
-  const int32_t S = (int32_t)cdiv(K, (int64_t)L * vw);
+  while (L < cdiv(need, R) && L < 32) L *= 2;
+  const int32_t S = (int32_t)cdiv(K, (int64_t)L * R * vw);
   const int32_t G = 32 / L;
   // step 3: FullWaveSize (Eqs. 3-4) from the occupancy of the SpMM kernel
   DeviceInfo d;
   if (gnn_status_t st = device_info(&d)) return st;
-  const int32_t abs = spmm_active_blocks_per_sm(vw, L, wpb);
+  const int32_t abs = spmm_active_blocks_per_sm(vw, L, R, wpb);
   if (abs < 1) return fail(GNN_ERR_CUDA, "plan: occupancy query failed (vw=%d L=%d)", vw, L);
   const int64_t FW = (int64_t)d.num_sms * abs;
   // steps 4-5: the largest candidate satisfying InEq. (5); none -> 8
@@ -78,6 +79,7 @@ gnn_status_t make_info(int64_t nnz, int32_t K, const gnn_plan_opts_t *opts,
   info->vw_feat = vw;
   info->vw_sparse = vws;
   info->lanes = L;
+  info->vecs = R;
   info->slices = S;
   info->groups = G;
   info->warps_per_block = wpb;

@@ -18,23 +18,22 @@
 
 namespace gnn {
 
-// Lane mapping of SDDMM.  The plan's L lanes x VW columns cover a K-slice; SDDMM
-// splits them into R vectors per lane over a group of Lg = L / R lanes, so each dot
-// product is reduced over fewer lanes (fewer shuffles per nonzero) and 32/Lg nonzeros
-// are in flight per warp step; U = nonzeros per batch per group, U * R = 8 feature
-// vectors in flight per lane.  Measured on the GCR-reordered C4 (profiles/
-// r01_sweep8.txt): R = 2 from L = 8 on (K=64: 2.07 -> 1.94 ms, K=128: 4.82 -> 3.61 ms,
-// K=256: 8.85 -> 7.05 ms), R = 1 below.  GNN_SDDMM_R2_FROM / GNN_SDDMM_UR override.
+// Lane mapping of SDDMM.  A K-slice holds V = L * R VW-wide vectors (plan rule step 2);
+// SDDMM spreads them over Lg = V / Rsd lanes with Rsd vectors per lane, so each dot
+// product is reduced over Lg lanes and 32 / Lg nonzeros are in flight per warp step;
+// U = nonzeros per batch per group, U * Rsd = 8 feature vectors in flight per lane.
+// Measured on the GCR-reordered C4 (profiles/r01_sweep8.txt): Rsd = 2 from V = 8 on
+// (K=64: 2.07 -> 1.94 ms, K=128: 4.82 -> 3.61 ms, K=256: 8.85 -> 7.05 ms), 1 below.
 #ifndef GNN_SDDMM_R2_FROM
-#define GNN_SDDMM_R2_FROM 8  // smallest L that uses R = 2
+#define GNN_SDDMM_R2_FROM 8  // smallest V that uses Rsd = 2
 #endif
 #ifndef GNN_SDDMM_UR
-#define GNN_SDDMM_UR 8       // U * R: feature vectors in flight per lane
+#define GNN_SDDMM_UR 8       // U * Rsd: feature vectors in flight per lane
 #endif
-template <int VW, int L, int SMAX>
+template <int VW, int V, int SMAX>
 struct SddmmShape {
-  static constexpr int R = (SMAX == 1 && L >= GNN_SDDMM_R2_FROM && L >= 2) ? 2 : 1;
-  static constexpr int Lg = L / R;
+  static constexpr int R = (V >= GNN_SDDMM_R2_FROM && V >= 2) ? 2 : 1;
+  static constexpr int Lg = V / R;
   static constexpr int depth = GNN_SDDMM_UR / R > 1 ? GNN_SDDMM_UR / R : 1;
 #if defined(GNN_SDDMM_MINB)
   static constexpr int minb = GNN_SDDMM_MINB;
@@ -97,6 +96,7 @@ __device__ __forceinline__ void reduce_scale_store(float (&part)[U], const float
   }
 }
 
+// L here is V, the number of VW-wide vectors in one K-slice (plan lanes x vecs).
 template <int VW, int L, int VWS, int SMAX>
 __global__ void __launch_bounds__(kMaxThreads, (SddmmShape<VW, L, SMAX>::minb))
     sddmm_kernel(const SparseArgs a, const float *__restrict__ A1, const int64_t lda1,
@@ -227,62 +227,64 @@ __global__ void __launch_bounds__(kMaxThreads, (SddmmShape<VW, L, SMAX>::minb))
 using SddmmFn = void (*)(const SparseArgs, const float *__restrict__, const int64_t,
                          const float *__restrict__, const int64_t, float *__restrict__);
 
-template <int VW, int L, int SMAX>
+template <int VW, int V, int SMAX>
 SddmmFn pick_sddmm_vws(int vws) {
   // a batch must cover whole sparse vectors: narrow the sparse loads when U < vw_sparse
-  constexpr int D = SddmmShape<VW, L, SMAX>::depth;
+  constexpr int D = SddmmShape<VW, V, SMAX>::depth;
   while (vws > D) vws >>= 1;
   switch (vws) {
-    case 1: return sddmm_kernel<VW, L, 1, SMAX>;
-    case 2: return sddmm_kernel<VW, L, 2, SMAX>;
-    case 4: return sddmm_kernel<VW, L, 4, SMAX>;
+    case 1: return sddmm_kernel<VW, V, 1, SMAX>;
+    case 2: return sddmm_kernel<VW, V, 2, SMAX>;
+    case 4: return sddmm_kernel<VW, V, 4, SMAX>;
   }
   return nullptr;
 }
 template <int VW>
-SddmmFn pick_sddmm_l(int L, int vws, int S) {
-  if (S > 1) return L == 32 ? pick_sddmm_vws<VW, 32, 4>(vws) : nullptr;
-  switch (L) {
+SddmmFn pick_sddmm_v(int V, int vws, int S) {
+  if (S > 1) return V == 64 ? pick_sddmm_vws<VW, 64, 4>(vws) : nullptr;
+  switch (V) {
     case 1: return pick_sddmm_vws<VW, 1, 1>(vws);
     case 2: return pick_sddmm_vws<VW, 2, 1>(vws);
     case 4: return pick_sddmm_vws<VW, 4, 1>(vws);
     case 8: return pick_sddmm_vws<VW, 8, 1>(vws);
     case 16: return pick_sddmm_vws<VW, 16, 1>(vws);
     case 32: return pick_sddmm_vws<VW, 32, 1>(vws);
+    case 64: return pick_sddmm_vws<VW, 64, 1>(vws);
+  }
+  return nullptr;
+}
+// V = L * R vectors per slice; S slices (<= 4)
+SddmmFn pick_sddmm(int vw, int V, int vws, int S) {
+  if (S > 4) return nullptr;
+  switch (vw) {
+    case 1: return pick_sddmm_v<1>(V, vws, S);
+    case 2: return pick_sddmm_v<2>(V, vws, S);
+    case 4: return pick_sddmm_v<4>(V, vws, S);
+    case 8: return pick_sddmm_v<8>(V, vws, S);
   }
   return nullptr;
 }
 // lanes per dot product of the instantiation pick_sddmm returns
 template <int VW>
-int group_lanes_vw(int L, int S) {
-  if (S > 1) return SddmmShape<VW, 32, 4>::Lg;
-  switch (L) {
+int group_lanes_vw(int V, int S) {
+  if (S > 1) return SddmmShape<VW, 64, 4>::Lg;
+  switch (V) {
     case 1: return SddmmShape<VW, 1, 1>::Lg;
     case 2: return SddmmShape<VW, 2, 1>::Lg;
     case 4: return SddmmShape<VW, 4, 1>::Lg;
     case 8: return SddmmShape<VW, 8, 1>::Lg;
     case 16: return SddmmShape<VW, 16, 1>::Lg;
-    default: return SddmmShape<VW, 32, 1>::Lg;
+    case 32: return SddmmShape<VW, 32, 1>::Lg;
+    default: return SddmmShape<VW, 64, 1>::Lg;
   }
 }
-int sddmm_group_lanes(int vw, int L, int S) {
+int sddmm_group_lanes(int vw, int V, int S) {
   switch (vw) {
-    case 1: return group_lanes_vw<1>(L, S);
-    case 2: return group_lanes_vw<2>(L, S);
-    case 4: return group_lanes_vw<4>(L, S);
-    default: return group_lanes_vw<8>(L, S);
+    case 1: return group_lanes_vw<1>(V, S);
+    case 2: return group_lanes_vw<2>(V, S);
+    case 4: return group_lanes_vw<4>(V, S);
+    default: return group_lanes_vw<8>(V, S);
   }
-}
-
-SddmmFn pick_sddmm(int vw, int L, int vws, int S) {
-  if (S > 4) return nullptr;
-  switch (vw) {
-    case 1: return pick_sddmm_l<1>(L, vws, S);
-    case 2: return pick_sddmm_l<2>(L, vws, S);
-    case 4: return pick_sddmm_l<4>(L, vws, S);
-    case 8: return pick_sddmm_l<8>(L, vws, S);
-  }
-  return nullptr;
 }
 
 }  // namespace gnn
@@ -304,13 +306,14 @@ extern "C" GNN_API gnn_status_t gnn_sddmm(gnn_plan_t plan, const gnn_graph_t *g,
                 "gnn_sddmm: A1/A2T must be %d-byte aligned with pitches multiple of %d", 4 * VW,
                 VW);
   const int vws = effective_vws(in.vw_sparse, g, out);
-  SddmmFn f = pick_sddmm(VW, in.lanes, vws, in.slices);
+  const int V = in.lanes * in.vecs;  // vectors per K-slice
+  SddmmFn f = pick_sddmm(VW, V, vws, in.slices);
   if (!f)
     return fail(GNN_ERR_UNSUPPORTED, "gnn_sddmm: K=%d needs %d slices (max 4 at vw=%d)", K,
                 in.slices, VW);
   const SparseArgs a = make_args(p, g);
   const int threads = in.warps_per_block * 32;
-  const int lg = sddmm_group_lanes(VW, in.lanes, in.slices);
+  const int lg = sddmm_group_lanes(VW, V, in.slices);
   const int64_t per_block = (int64_t)(32 / lg) * in.warps_per_block;
   const int64_t blocks = (a.num_chunks + per_block - 1) / per_block;
   f<<<(unsigned)blocks, threads, 0, (cudaStream_t)stream>>>(a, A1, lda1, A2T, lda2, out);

@@ -32,22 +32,19 @@ namespace gnn {
 #define GNN_SPMM_MINB 1  // min resident 512-thread blocks/SM the register budget must allow
 #endif
 
-template <int VW, int L>
+// Feature vectors in flight per lane.  Measured on C4 (profiles/r01_sweep4.txt,
+// r01_sweep11.txt): 4 while several chunks share a warp (L <= 8, R = 1), 8 for wider
+// groups and whenever a lane holds R = 2 vectors per row.
+#ifndef GNN_SPMM_DEPTH_R2
+#define GNN_SPMM_DEPTH_R2 4
+#endif
+template <int VW, int L, int R>
 struct FeatDepth {
 #if defined(GNN_SPMM_DEPTH8)
   static constexpr int value = VW == 8 ? GNN_SPMM_DEPTH8 : 8;
 #else
-  static constexpr int value = VW == 8 ? (L >= 16 ? 8 : 4) : 8;
+  static constexpr int value = R == 2 ? GNN_SPMM_DEPTH_R2 : (VW == 8 ? (L >= 16 ? 8 : 4) : 8);
 #endif
-};
-
-template <int VW, int L, int VWS>
-struct TileCfg {
-  static constexpr int G = 32 / L;
-  static constexpr int T = L * VWS;  // nonzeros per tile per group
-  static constexpr int U0 = FeatDepth<VW, L>::value > VWS ? FeatDepth<VW, L>::value : VWS;
-  static constexpr int U = U0 < T ? U0 : T;
-  static_assert(T % U == 0 && U % VWS == 0, "tile / prefetch shape");
 };
 
 // Flush the accumulator of row `cur` (Algo 3 line 15, "AtomicStore"): rows shared
@@ -63,15 +60,21 @@ __device__ __forceinline__ void flush_row(float *Ok, int64_t ldo, int64_t row_ba
   else st_vec<VW>(o, acc);
 }
 
-template <int VW, int L, int VWS>
+// L lanes per (chunk, K-slice) work item, R VW-wide vectors per lane (plan rule step 2).
+template <int VW, int L, int R, int VWS>
 __global__ void __launch_bounds__(kMaxThreads, GNN_SPMM_MINB)
     spmm_kernel(const SparseArgs a, const float *__restrict__ A, const int64_t lda,
                 float *__restrict__ O, const int64_t ldo) {
-  using Cfg = TileCfg<VW, L, VWS>;
-  constexpr int G = Cfg::G, T = Cfg::T, U = Cfg::U;
+  constexpr int Lg = L;
+  constexpr int G = 32 / Lg;
+  constexpr int T = Lg * VWS;  // nonzeros per tile per group
+  // U nonzeros per batch: FeatDepth vectors in flight per lane, whole sparse vectors
+  constexpr int D = FeatDepth<VW, L, R>::value / R;
+  constexpr int U = D > T ? T : (D < VWS ? VWS : D);
+  static_assert(T % U == 0 && U % VWS == 0, "tile / prefetch shape");
   const int lane = threadIdx.x & 31;
-  const int g = lane / L;
-  const int l = lane & (L - 1);
+  const int g = lane / Lg;
+  const int l = lane & (Lg - 1);
   const int64_t item = ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * G + g;
   const bool item_ok = item < a.num_chunks * a.slices;
   if (!__any_sync(kFull, item_ok)) return;  // warp-uniform exit
@@ -82,8 +85,11 @@ __global__ void __launch_bounds__(kMaxThreads, GNN_SPMM_MINB)
     c = item / a.slices;
     s = (int)(item - c * a.slices);
   }
-  const int k0 = (s * L + l) * VW;
-  const bool col_ok = item_ok && k0 < a.K;
+  // vector r of this lane covers columns k0 + r * L * VW .. + VW of slice s
+  const int k0 = (s * L * R + l) * VW;
+  bool col_ok[R];
+#pragma unroll
+  for (int r = 0; r < R; ++r) col_ok[r] = item_ok && k0 + r * Lg * VW < a.K;
   const int64_t cs = c * a.chunk;
   const int n = item_ok ? (int)(min(cs + (int64_t)a.chunk, a.nnz) - cs) : 0;  // nnz here
   int32_t rf = 0, rl = 0;
@@ -98,15 +104,29 @@ __global__ void __launch_bounds__(kMaxThreads, GNN_SPMM_MINB)
   const uint32_t ldaB = (uint32_t)lda * 4u;
   float *__restrict__ Ok = O + k0;  // row r at Ok + (r - row_base) * ldo
 
+  auto zero_row = [&](int64_t row) {
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+      if (col_ok[r]) st_zero<VW>(Ok + (row - a.row_base) * ldo + r * Lg * VW);
+  };
+  float acc[R][VW];
+  auto flush = [&](int32_t row) {
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+      if (col_ok[r])
+        flush_row<VW>(Ok + r * Lg * VW, ldo, a.row_base, row, rf, rl, fl, acc[r]);
+  };
+
   // empty rows between the previous chunk's last row and ours are ours to zero
-  if (col_ok) {
+  if (item_ok) {
     const int64_t prev = (c == 0) ? a.row_base - 1 : (int64_t)a.row_last[c - 1];
-    for (int64_t r = prev + 1; r < rf; ++r) st_zero<VW>(Ok + (r - a.row_base) * ldo);
+    for (int64_t r = prev + 1; r < rf; ++r) zero_row(r);
   }
 
-  float acc[VW];
 #pragma unroll
-  for (int v = 0; v < VW; ++v) acc[v] = 0.f;
+  for (int r = 0; r < R; ++r)
+#pragma unroll
+    for (int v = 0; v < VW; ++v) acc[r][v] = 0.f;
   int32_t cur = -1;
 
   const int32_t *__restrict__ ri = a.row_ind + cs;
@@ -134,20 +154,21 @@ __global__ void __launch_bounds__(kMaxThreads, GNN_SPMM_MINB)
       ld_sparse_i32<VWS>(ci, li, n, 0, nc);
       ld_sparse_f32<VWS>(vi, li, n, nv);
     }
-    const int32_t r_first = __shfl_sync(kFull, rr[0], 0, L);
-    const int32_t r_last = __shfl_sync(kFull, rr[VWS - 1], L - 1, L);
+    const int32_t r_first = __shfl_sync(kFull, rr[0], 0, Lg);
+    const int32_t r_last = __shfl_sync(kFull, rr[VWS - 1], Lg - 1, Lg);
     const bool fast_g = (tb + T <= n) && r_first == r_last;
     if (__all_sync(kFull, fast_g || !item_ok)) {
       // ---- fast path: the whole tile belongs to one row (all groups of the warp)
       if (item_ok && r_first != cur) {
-        if (cur >= 0 && col_ok) {
-          flush_row<VW>(Ok, ldo, a.row_base, cur, rf, rl, fl, acc);
-          for (int64_t r = (int64_t)cur + 1; r < r_first; ++r)
-            st_zero<VW>(Ok + (r - a.row_base) * ldo);
+        if (cur >= 0) {
+          flush(cur);
+          for (int64_t r = (int64_t)cur + 1; r < r_first; ++r) zero_row(r);
         }
         cur = r_first;
 #pragma unroll
-        for (int v = 0; v < VW; ++v) acc[v] = 0.f;
+        for (int r = 0; r < R; ++r)
+#pragma unroll
+          for (int v = 0; v < VW; ++v) acc[r][v] = 0.f;
       }
 #pragma unroll 1
       for (int jj = 0; jj < T; jj += U) {
@@ -156,23 +177,27 @@ __global__ void __launch_bounds__(kMaxThreads, GNN_SPMM_MINB)
 #pragma unroll
         for (int u = 0; u < U; ++u) {
           const int src = (jj + u) / VWS;
-          cj[u] = (uint32_t)__shfl_sync(kFull, cc[u % VWS], src, L);
-          vj[u] = __shfl_sync(kFull, vv[u % VWS], src, L);
+          cj[u] = (uint32_t)__shfl_sync(kFull, cc[u % VWS], src, Lg);
+          vj[u] = __shfl_sync(kFull, vv[u % VWS], src, Lg);
         }
-        float x[U][VW];
+        float x[U][R][VW];
 #pragma unroll
         for (int u = 0; u < U; ++u) {
-          if (col_ok) {
-            ld_feat<VW>(reinterpret_cast<const float *>(Ab + (uint64_t)cj[u] * ldaB), x[u]);
-          } else {
+          const float *rowp = reinterpret_cast<const float *>(Ab + (uint64_t)cj[u] * ldaB);
 #pragma unroll
-            for (int v = 0; v < VW; ++v) x[u][v] = 0.f;
+          for (int r = 0; r < R; ++r) {
+            if (col_ok[r]) {
+              ld_feat<VW>(rowp + r * Lg * VW, x[u][r]);
+            } else {
+#pragma unroll
+              for (int v = 0; v < VW; ++v) x[u][r][v] = 0.f;
+            }
           }
         }
 #pragma unroll
-        for (int u = 0; u < U; ++u) {
-          axpy<VW>(acc, vj[u], x[u]);
-        }
+        for (int u = 0; u < U; ++u)
+#pragma unroll
+          for (int r = 0; r < R; ++r) axpy<VW>(acc[r], vj[u], x[u][r]);
       }
     } else {
       // ---- general path: per-nonzero validity and row-switch procedure
@@ -184,44 +209,49 @@ __global__ void __launch_bounds__(kMaxThreads, GNN_SPMM_MINB)
 #pragma unroll
         for (int u = 0; u < U; ++u) {
           const int src = (jj + u) / VWS;
-          rj[u] = __shfl_sync(kFull, rr[u % VWS], src, L);
-          cj[u] = (uint32_t)__shfl_sync(kFull, cc[u % VWS], src, L);
-          vj[u] = __shfl_sync(kFull, vv[u % VWS], src, L);
+          rj[u] = __shfl_sync(kFull, rr[u % VWS], src, Lg);
+          cj[u] = (uint32_t)__shfl_sync(kFull, cc[u % VWS], src, Lg);
+          vj[u] = __shfl_sync(kFull, vv[u % VWS], src, Lg);
         }
-        float x[U][VW];
+        float x[U][R][VW];
 #pragma unroll
         for (int u = 0; u < U; ++u) {
-          if (col_ok && tb + jj + u < n) {
-            ld_feat<VW>(reinterpret_cast<const float *>(Ab + (uint64_t)cj[u] * ldaB), x[u]);
-          } else {
+          const float *rowp = reinterpret_cast<const float *>(Ab + (uint64_t)cj[u] * ldaB);
 #pragma unroll
-            for (int v = 0; v < VW; ++v) x[u][v] = 0.f;
+          for (int r = 0; r < R; ++r) {
+            if (col_ok[r] && tb + jj + u < n) {
+              ld_feat<VW>(rowp + r * Lg * VW, x[u][r]);
+            } else {
+#pragma unroll
+              for (int v = 0; v < VW; ++v) x[u][r][v] = 0.f;
+            }
           }
         }
 #pragma unroll
         for (int u = 0; u < U; ++u) {
           if (tb + jj + u < n) {
             if (rj[u] != cur) {  // row-switch procedure
-              if (cur >= 0 && col_ok) {
-                flush_row<VW>(Ok, ldo, a.row_base, cur, rf, rl, fl, acc);
-                for (int64_t r = (int64_t)cur + 1; r < rj[u]; ++r)
-                  st_zero<VW>(Ok + (r - a.row_base) * ldo);
+              if (cur >= 0) {
+                flush(cur);
+                for (int64_t r = (int64_t)cur + 1; r < rj[u]; ++r) zero_row(r);
               }
               cur = rj[u];
 #pragma unroll
-              for (int v = 0; v < VW; ++v) acc[v] = 0.f;
+              for (int r = 0; r < R; ++r)
+#pragma unroll
+                for (int v = 0; v < VW; ++v) acc[r][v] = 0.f;
             }
-            axpy<VW>(acc, vj[u], x[u]);
+#pragma unroll
+            for (int r = 0; r < R; ++r) axpy<VW>(acc[r], vj[u], x[u][r]);
           }
         }
       }
     }
   }
-  if (cur >= 0 && col_ok) flush_row<VW>(Ok, ldo, a.row_base, cur, rf, rl, fl, acc);
+  if (cur >= 0) flush(cur);
   // trailing empty rows after the last chunk
-  if (col_ok && c == a.num_chunks - 1) {
-    for (int64_t r = (int64_t)rl + 1; r < a.row_base + a.M; ++r)
-      st_zero<VW>(Ok + (r - a.row_base) * ldo);
+  if (item_ok && c == a.num_chunks - 1) {
+    for (int64_t r = (int64_t)rl + 1; r < a.row_base + a.M; ++r) zero_row(r);
   }
 }
 
@@ -246,50 +276,60 @@ __global__ void spmm_prezero_kernel(const SparseArgs a, float *__restrict__ O,
 using SpmmFn = void (*)(const SparseArgs, const float *__restrict__, const int64_t,
                         float *__restrict__, const int64_t);
 
-template <int VW, int L>
+template <int VW, int L, int R>
 SpmmFn pick_vws(int vws) {
   switch (vws) {
-    case 1: return spmm_kernel<VW, L, 1>;
-    case 2: return spmm_kernel<VW, L, 2>;
-    case 4: return spmm_kernel<VW, L, 4>;
+    case 1: return spmm_kernel<VW, L, R, 1>;
+    case 2: return spmm_kernel<VW, L, R, 2>;
+    case 4: return spmm_kernel<VW, L, R, 4>;
   }
   return nullptr;
 }
 template <int VW>
-SpmmFn pick_l(int L, int vws) {
+SpmmFn pick_l(int L, int R, int vws) {
+  if (R == 2) {  // the plan uses R = 2 only for rows of >= 16 vectors, i.e. L >= 8
+    switch (L) {
+      case 8: return pick_vws<VW, 8, 2>(vws);
+      case 16: return pick_vws<VW, 16, 2>(vws);
+      case 32: return pick_vws<VW, 32, 2>(vws);
+    }
+    return nullptr;
+  }
   switch (L) {
-    case 1: return pick_vws<VW, 1>(vws);
-    case 2: return pick_vws<VW, 2>(vws);
-    case 4: return pick_vws<VW, 4>(vws);
-    case 8: return pick_vws<VW, 8>(vws);
-    case 16: return pick_vws<VW, 16>(vws);
-    case 32: return pick_vws<VW, 32>(vws);
+    case 1: return pick_vws<VW, 1, 1>(vws);
+    case 2: return pick_vws<VW, 2, 1>(vws);
+    case 4: return pick_vws<VW, 4, 1>(vws);
+    case 8: return pick_vws<VW, 8, 1>(vws);
+    case 16: return pick_vws<VW, 16, 1>(vws);
+    case 32: return pick_vws<VW, 32, 1>(vws);
   }
   return nullptr;
 }
-SpmmFn pick_spmm(int vw, int L, int vws) {
+SpmmFn pick_spmm(int vw, int L, int R, int vws) {
   switch (vw) {
-    case 1: return pick_l<1>(L, vws);
-    case 2: return pick_l<2>(L, vws);
-    case 4: return pick_l<4>(L, vws);
-    case 8: return pick_l<8>(L, vws);
+    case 1: return pick_l<1>(L, R, vws);
+    case 2: return pick_l<2>(L, R, vws);
+    case 4: return pick_l<4>(L, R, vws);
+    case 8: return pick_l<8>(L, R, vws);
   }
   return nullptr;
 }
 
-// Cached per (device, vw, lanes, wpb): the occupancy API is a host-side query but not
-// free, and plans are rebuilt every step in graph-sampling training (C3).
-int spmm_active_blocks_per_sm(int vw, int lanes, int wpb) {
-  static std::atomic<int> cache[64][4][6][17];
+// Cached per (device, vw, lanes, vecs, wpb): the occupancy API is a host-side query but
+// not free, and plans are rebuilt every step in graph-sampling training (C3).
+int spmm_active_blocks_per_sm(int vw, int lanes, int vecs, int wpb) {
+  static std::atomic<int> cache[64][4][6][2][17];
   int dev = 0;
-  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64 || wpb < 1 || wpb > 16) return 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64 || wpb < 1 || wpb > 16 ||
+      vecs < 1 || vecs > 2)
+    return 0;
   const int iv = vw == 1 ? 0 : vw == 2 ? 1 : vw == 4 ? 2 : 3;
   int il = 0;
   while ((1 << il) < lanes && il < 5) ++il;
-  std::atomic<int> &slot = cache[dev][iv][il][wpb];
+  std::atomic<int> &slot = cache[dev][iv][il][vecs - 1][wpb];
   int n = slot.load(std::memory_order_relaxed);
   if (n > 0) return n;
-  SpmmFn f = pick_spmm(vw, lanes, 1);
+  SpmmFn f = pick_spmm(vw, lanes, vecs, 1);
   if (!f) return 0;
   if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, f, wpb * 32, 0) != cudaSuccess) return 0;
   slot.store(n, std::memory_order_relaxed);
@@ -339,6 +379,7 @@ SparseArgs make_args(const Plan *p, const gnn_graph_t *g) {
   a.chunk = p->info.chunk;
   a.K = p->info.K;
   a.slices = p->info.slices;
+  a.vecs = p->info.vecs;
   return a;
 }
 
@@ -367,7 +408,7 @@ extern "C" GNN_API gnn_status_t gnn_spmm(gnn_plan_t plan, const gnn_graph_t *g, 
     return e == cudaSuccess ? GNN_OK : cuda_fail(e, "gnn_spmm memset");
   }
   const int vws = effective_vws(in.vw_sparse, g, nullptr);
-  SpmmFn f = pick_spmm(VW, in.lanes, vws);
+  SpmmFn f = pick_spmm(VW, in.lanes, in.vecs, vws);
   if (!f) return fail(GNN_ERR_UNSUPPORTED, "gnn_spmm: no kernel for vw=%d L=%d", VW, in.lanes);
   const SparseArgs a = make_args(p, g);
   const int threads = in.warps_per_block * 32;

@@ -250,17 +250,19 @@ def _brute_blocks(nnz, C, S, G, WPB):
     return int(np.unique(blocks).size)
 
 
-VW_TABLE = {  # K: (vw_feat, lanes, slices, groups) -- DESIGN.md "Plan rule" table
-    32: (8, 4, 1, 8), 64: (8, 8, 1, 4), 128: (8, 16, 1, 2), 256: (8, 32, 1, 1),
-    100: (4, 32, 1, 1), 33: (1, 32, 2, 1), 1000: (8, 32, 4, 1), 6: (2, 4, 1, 8),
-    1: (1, 1, 1, 32), 512: (8, 32, 2, 1), 24: (8, 4, 1, 8), 12: (4, 4, 1, 8),
+VW_TABLE = {  # K: (vw_feat, lanes, vecs, slices, groups) -- DESIGN.md "Plan rule" table
+    32: (8, 4, 1, 1, 8), 64: (8, 8, 1, 1, 4), 128: (8, 8, 2, 1, 4), 256: (8, 16, 2, 1, 2),
+    100: (4, 16, 2, 1, 2), 33: (1, 32, 2, 1, 1), 1000: (8, 32, 2, 2, 1), 6: (2, 4, 1, 1, 8),
+    1: (1, 1, 1, 1, 32), 512: (8, 32, 2, 1, 1), 24: (8, 4, 1, 1, 8), 12: (4, 4, 1, 1, 8),
+    2048: (8, 32, 2, 4, 1), 120: (8, 16, 1, 1, 2),
 }
 
 
 @pytest.mark.parametrize("K", sorted(VW_TABLE))
 def test_plan_vector_width_table(K):
     p = oracle.plan(np.zeros(100, np.int32), K, num_sms=148, active_blocks_per_sm=8)
-    assert (p.info["vw_feat"], p.info["lanes"], p.info["slices"], p.info["groups"]) == VW_TABLE[K]
+    assert (p.info["vw_feat"], p.info["lanes"], p.info["vecs"], p.info["slices"],
+            p.info["groups"]) == VW_TABLE[K]
 
 
 @pytest.mark.parametrize("nnz,K,alpha,abs_", [
