@@ -85,6 +85,35 @@ def load_peaks():
     return 6650.0, "fallback (B200_PROFILING.md)"
 
 
+def measure_gather_ceiling(K, dev):
+    """Live roofline probe (gnn_probe_gather): random-row gather rate of K fp32 columns
+    from an L2-resident (32 MiB) and an HBM-resident (4 GiB) matrix, GB/s."""
+    import torch
+    import paper_conf_ipps_fanwc23_b200 as gs
+    if K not in (32, 64, 128, 256):
+        return None
+    out = {}
+    n = 32 * 1024 * 1024
+    sink = torch.zeros(1, device=dev)
+    for tier, nbytes in (("l2", 32 << 20), ("hbm", 4 << 30)):
+        rows = nbytes // (4 * K)
+        X = torch.empty((rows, K), device=dev).uniform_(-1, 1)
+        idx = torch.randint(0, rows, (n,), device=dev, dtype=torch.int32)
+        best = 1e9
+        for it in range(5):
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record()
+            gs.probe_gather(X, idx, sink)
+            b.record()
+            torch.cuda.synchronize()
+            if it:
+                best = min(best, a.elapsed_time(b))
+        out[f"{tier}_GBps"] = round(n * 4 * K / best / 1e6, 1)
+        del X, idx
+    torch.cuda.empty_cache()
+    return out
+
+
 def load_ncu_traffic():
     """DRAM bytes per launch from the committed `ncu --set full` summary, if any."""
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -376,6 +405,10 @@ def run_ours(args):
                     hbm_compulsory(spg.nnz if dkind == "spmm" else sdg.nnz, spg.M, g.N, dK,
                                    dkind) / (dms * 1e-3) / 1e9 / peak, 4),
                 "traffic_key": tkey}
+    ceil = measure_gather_ceiling(dK, dev)
+    if ceil:
+        roofline["gather_ceiling_measured"] = ceil
+        roofline["frac_of_l2_gather"] = round(achieved / ceil["l2_GBps"], 4)
     launches, clocks, detail = r["launches"], r["clocks"], r["detail"]
     alt = None
     if reorder and args.compare:

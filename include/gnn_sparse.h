@@ -188,6 +188,15 @@ GNN_API gnn_status_t gnn_permute_rows(const float *X, int64_t ldx, int64_t n, in
                                       const int32_t *perm, float *Y, int64_t ldy,
                                       gnn_stream_t stream);
 
+/* ----------------------------------------------------------- measurement --- */
+/* Roofline probe (not part of the method): gathers rows X[idx[i]][0:K] for i in [0, n)
+ * with the same 256-bit row loads the kernels use and no other work (sums are folded
+ * into *sink so the loads are live).  Timing it on an L1-, L2- or HBM-resident X gives
+ * the on-chip / off-chip gather ceilings bench.py reports beside the HBM roofline.
+ * K in {32, 64, 128, 256}; X 32-byte aligned with ld % 8 == 0; idx in [0, rows). */
+GNN_API gnn_status_t gnn_probe_gather(const float *X, int64_t ld, const int32_t *idx, int64_t n,
+                                      int32_t K, float *sink, gnn_stream_t stream);
+
 /* ------------------------------------------------------------- helpers ---- */
 /* Decode CSR offsets into the hybrid format's RowInd (Fig. 2d):
  * row_ind[i - row_ptr[0]] = r + row_base for row_ptr[r] <= i < row_ptr[r+1]. */

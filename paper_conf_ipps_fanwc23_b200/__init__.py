@@ -67,7 +67,8 @@ class ReorderOpts(ctypes.Structure):
 EXPORTS = ["gnn_plan_workspace_bytes", "gnn_plan_create", "gnn_plan_info", "gnn_plan_arrays",
            "gnn_plan_destroy", "gnn_spmm", "gnn_sddmm", "gnn_shard_rows", "gnn_shard_edges",
            "gnn_reorder_gcr", "gnn_permute_graph", "gnn_permute_rows",
-           "gnn_csr_to_coo", "gnn_validate", "gnn_last_error", "gnn_version"]
+           "gnn_probe_gather", "gnn_csr_to_coo", "gnn_validate", "gnn_last_error",
+           "gnn_version"]
 
 _lib = None
 
@@ -97,6 +98,7 @@ def lib():
     L.gnn_reorder_gcr.argtypes = [vp, vp, i64, P(ReorderOpts), vp, vp, P(ctypes.c_double)]
     L.gnn_permute_graph.argtypes = [vp, vp, vp, i64, vp, vp, vp, vp, vp]
     L.gnn_permute_rows.argtypes = [vp, i64, i64, i64, vp, vp, i64, vp]
+    L.gnn_probe_gather.argtypes = [vp, i64, vp, i64, i32, vp, vp]
     L.gnn_validate.argtypes = [P(_Graph), vp]
     L.gnn_last_error.argtypes = []
     L.gnn_last_error.restype = ctypes.c_char_p
@@ -104,7 +106,7 @@ def lib():
     L.gnn_version.restype = ctypes.c_char_p
     for f in ("gnn_plan_create", "gnn_plan_info", "gnn_plan_arrays", "gnn_spmm", "gnn_sddmm",
               "gnn_shard_rows", "gnn_shard_edges", "gnn_csr_to_coo", "gnn_validate",
-              "gnn_reorder_gcr", "gnn_permute_graph", "gnn_permute_rows"):
+              "gnn_reorder_gcr", "gnn_permute_graph", "gnn_permute_rows", "gnn_probe_gather"):
         getattr(L, f).restype = st
     _lib = L
     return L
@@ -336,3 +338,12 @@ def permute_rows(X: torch.Tensor, perm: torch.Tensor, out: torch.Tensor | None =
     _check(lib().gnn_permute_rows(_ptr(X), X.stride(0), X.shape[0], X.shape[1], _ptr(perm),
                                   _ptr(out), out.stride(0), _stream(stream)))
     return out
+
+
+def probe_gather(X: torch.Tensor, idx: torch.Tensor, sink: torch.Tensor | None = None,
+                 stream=None) -> None:
+    """gnn_probe_gather: pure row gather X[idx] (measurement utility)."""
+    if sink is None:
+        sink = torch.zeros(1, device=X.device)
+    _check(lib().gnn_probe_gather(_ptr(X), X.stride(0), _ptr(idx), idx.numel(), X.shape[1],
+                                  _ptr(sink), _stream(stream)))
