@@ -2,14 +2,17 @@
 #   gen/libgnngen.so                       seeded input generators (shared by both sides)
 #   oracle/liboracle.so                    fp64 CPU oracle (test infrastructure only)
 #   paper_conf_ipps_fanwc23_b200/libgnnsparse.so   the product: C-ABI + sm_100a kernels
+# Translation units compile to objects in parallel (make -j), then link once.
 NVCC    ?= /usr/local/cuda/bin/nvcc
 HOSTCC  ?= /usr/bin/gcc
 PKG     := paper_conf_ipps_fanwc23_b200
 ARCH    := -gencode arch=compute_100a,code=sm_100a
-NVFLAGS := -ccbin /usr/bin/g++ $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC -Xcompiler -fvisibility=hidden \
-           -Iinclude --expt-relaxed-constexpr -Xptxas -v
+NVFLAGS := -ccbin /usr/bin/g++ $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC \
+           -Xcompiler -fvisibility=hidden -Iinclude --expt-relaxed-constexpr -Xptxas -v
 CUSRC   := $(wildcard $(PKG)/csrc/*.cu) $(wildcard $(PKG)/csrc/*.cpp)
 CUHDR   := $(wildcard $(PKG)/csrc/*.cuh) include/gnn_sparse.h
+OBJDIR  := build/obj$(if $(TAG),_$(TAG),)
+OBJS    := $(patsubst $(PKG)/csrc/%,$(OBJDIR)/%.o,$(CUSRC))
 
 all: gen/libgnngen.so oracle/liboracle.so $(PKG)/libgnnsparse.so
 
@@ -20,15 +23,21 @@ gen/libgnngen.so: gen/gen.c gen/gen.h
 oracle/liboracle.so: oracle/oracle.c oracle/oracle.h
 	$(HOSTCC) -O2 -ffp-contract=off -fno-fast-math -fPIC -shared -o $@ oracle/oracle.c -lm
 
-$(PKG)/libgnnsparse.so: $(CUSRC) $(CUHDR)
-	$(NVCC) $(NVFLAGS) -shared -cudart static -o $@ $(CUSRC) 2> $(PKG)/ptxas.log || (cat $(PKG)/ptxas.log; exit 1)
+$(OBJDIR)/%.o: $(PKG)/csrc/% $(CUHDR)
+	@mkdir -p $(OBJDIR)
+	$(NVCC) $(NVFLAGS) $(DEFS) -c -o $@ $< 2> $@.ptxas.log || (cat $@.ptxas.log; exit 1)
 
-# tuning variants: make variant TAG=x DEFS="-DGNN_SPMM_MINB=2 ..."  ->  build/libgnnsparse_x.so
-variant: $(CUSRC) $(CUHDR)
-	mkdir -p build
-	$(NVCC) $(NVFLAGS) $(DEFS) -shared -cudart static -o build/libgnnsparse_$(TAG).so $(CUSRC) 2> build/ptxas_$(TAG).log || (cat build/ptxas_$(TAG).log; exit 1)
+$(PKG)/libgnnsparse.so: $(OBJS)
+	$(NVCC) $(ARCH) -shared -cudart static -o $@ $(OBJS)
+	cat $(OBJDIR)/*.ptxas.log > $(PKG)/ptxas.log
+
+# tuning variants: make -j variant TAG=x DEFS="-DGNN_SPMM_MINB=2 ..." -> build/libgnnsparse_x.so
+variant: $(OBJS)
+	@mkdir -p build
+	$(NVCC) $(ARCH) -shared -cudart static -o build/libgnnsparse_$(TAG).so $(OBJS)
+	cat $(OBJDIR)/*.ptxas.log > build/ptxas_$(TAG).log
 
 clean:
-	rm -f gen/libgnngen.so oracle/liboracle.so $(PKG)/libgnnsparse.so
+	rm -rf gen/libgnngen.so oracle/liboracle.so $(PKG)/libgnnsparse.so build/obj*
 
 .PHONY: all clean variant

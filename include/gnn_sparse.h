@@ -52,6 +52,10 @@ typedef enum {
 
 typedef void *gnn_stream_t; /* a cudaStream_t */
 
+/* Element type of the gathered feature matrices (A, A1, A2T).  Accumulation and the
+ * outputs (O, S_O) are fp32 for both (bf16 halves the gathered bytes). */
+typedef enum { GNN_F32 = 0, GNN_BF16 = 1 } gnn_dtype_t;
+
 /* A hybrid CSR/COO adjacency S (M x N) or a row/edge shard of one.
  * A shard's row_ind holds GLOBAL row ids in [row_base, row_base + M); its
  * row_ind/col_ind/val pointers are sub-views starting at the shard's first nnz.
@@ -73,12 +77,13 @@ typedef struct {
   int32_t force_chunk;     /* 0 = DTP choice; >0 forces NnzPerWarp (ablation/tests) */
   int32_t force_vw;        /* 0 = from K; 1/2/4/8 forces the feature vector width   */
   int32_t deterministic;   /* reserved (must be 0 in this version)                  */
+  int32_t feature_dtype;   /* gnn_dtype_t of the feature matrices; default GNN_F32   */
 } gnn_plan_opts_t;
 
 /* What the plan decided (all integers; bit-exact with the oracle's plan). */
 typedef struct {
   int32_t chunk;           /* C*: nnz per work chunk ("NnzPerWarp")    */
-  int32_t vw_feat;         /* feature-row vector width VW (floats per lane)         */
+  int32_t vw_feat;         /* feature-row vector width VW (elements per lane-vector) */
   int32_t vw_sparse;       /* sparse-array vector width (HVMA): 1, 2 or 4     */
   int32_t lanes;           /* L: lanes per chunk-slice                              */
   int32_t vecs;            /* R: VW-wide vectors per lane per slice (1 or 2)         */
@@ -89,6 +94,7 @@ typedef struct {
   int32_t num_sms;         /* NumSM (Eq. 4)                                         */
   int32_t alpha;
   int32_t K;
+  int32_t feature_dtype;   /* gnn_dtype_t the plan was built for                    */
   int64_t nnz;
   int64_t num_chunks;      /* ceil(nnz / chunk)                                     */
   int64_t num_blocks;      /* SpMM grid size (integer form of InEq. (5) RHS)         */
@@ -134,6 +140,13 @@ GNN_API void gnn_plan_destroy(gnn_plan_t plan);
 GNN_API gnn_status_t gnn_spmm(gnn_plan_t plan, const gnn_graph_t *graph, const float *A,
                               int64_t lda, float *O, int64_t ldo, gnn_stream_t stream);
 
+/* gnn_spmm with bf16 features A (raw bf16 bit patterns, N x K, lda >= K elements;
+ * A 2*vw_feat-byte aligned, lda a multiple of vw_feat), fp32 accumulation, fp32 O.
+ * The plan must have been built with feature_dtype = GNN_BF16. */
+GNN_API gnn_status_t gnn_spmm_bf16(gnn_plan_t plan, const gnn_graph_t *graph,
+                                   const uint16_t *A, int64_t lda, float *O, int64_t ldo,
+                                   gnn_stream_t stream);
+
 /* SDDMM, S_O = (A1 A2) (.) S (Algorithm 2), hybrid-parallel
  * (Algorithm 4): out[i] = val[i] * sum_k A1[row_ind[i] - row_base][k] *
  * A2T[col_ind[i]][k] for i in [0, nnz).  A1: M x K (destination rows, lda1 >= K);
@@ -143,6 +156,12 @@ GNN_API gnn_status_t gnn_spmm(gnn_plan_t plan, const gnn_graph_t *graph, const f
 GNN_API gnn_status_t gnn_sddmm(gnn_plan_t plan, const gnn_graph_t *graph, const float *A1,
                                int64_t lda1, const float *A2T, int64_t lda2, float *out,
                                gnn_stream_t stream);
+
+/* gnn_sddmm with bf16 A1 / A2T (raw bf16 bit patterns), fp32 products and sums, fp32
+ * out.  Plan built with feature_dtype = GNN_BF16. */
+GNN_API gnn_status_t gnn_sddmm_bf16(gnn_plan_t plan, const gnn_graph_t *graph,
+                                    const uint16_t *A1, int64_t lda1, const uint16_t *A2T,
+                                    int64_t lda2, float *out, gnn_stream_t stream);
 
 /* -------------------------------------------------------------- shards ---- */
 /* nnz-balanced contiguous row shards for P GPUs (HOST arrays; DESIGN.md

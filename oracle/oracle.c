@@ -74,25 +74,26 @@ static int64_t blocks_for(int64_t nnz, int64_t C, int64_t S, int64_t G, int64_t 
 
 int oracle_plan(int64_t nnz, const int32_t *row_ind, int32_t K, int32_t alpha,
                 int32_t warps_per_block, int32_t force_chunk, int32_t force_vw,
-                int32_t num_sms, int32_t active_blocks_per_sm, oracle_plan_info_t *info,
+                int32_t feature_dtype, int32_t num_sms, int32_t active_blocks_per_sm, oracle_plan_info_t *info,
                 int32_t *row_first, int32_t *row_last, uint8_t *flags) {
   if (nnz < 0 || K < 1 || alpha < 1 || warps_per_block < 1 || num_sms < 1 ||
       active_blocks_per_sm < 1 || force_chunk < 0 || !info)
     return -1;
-  /* step 1: feature vector width from K alone (or forced) */
-  int32_t vw;
+  /* step 1: feature vector width in elements of the feature dtype (0 fp32: 8,4,2,1;
+   * 1 bf16: 16,8,4,2): the widest that divides K, or forced */
+  int32_t vmax, vmin, vw = 0;
+  if (feature_dtype == 0) { vmax = 8; vmin = 1; }
+  else if (feature_dtype == 1) { vmax = 16; vmin = 2; }
+  else return -1;
   if (force_vw > 0) {
-    if (!(force_vw == 1 || force_vw == 2 || force_vw == 4 || force_vw == 8)) return -1;
-    if (K % force_vw != 0) return -1;
+    int ok = 0;
+    for (int32_t v = vmin; v <= vmax; v *= 2) ok |= (force_vw == v);
+    if (!ok || K % force_vw != 0) return -1;
     vw = force_vw;
-  } else if (K % 8 == 0) {
-    vw = 8;
-  } else if (K % 4 == 0) {
-    vw = 4;
-  } else if (K % 2 == 0) {
-    vw = 2;
   } else {
-    vw = 1;
+    for (int32_t v = vmax; v >= vmin; v /= 2)
+      if (vw == 0 && K % v == 0) vw = v;
+    if (vw == 0) return -1;
   }
   /* step 2: vectors per lane, lanes per chunk-slice, slices, groups per warp */
   int64_t need = cdiv(K, vw);          /* VW-wide vectors in a feature row */
@@ -128,6 +129,7 @@ int oracle_plan(int64_t nnz, const int32_t *row_ind, int32_t K, int32_t alpha,
   info->num_sms = num_sms;
   info->alpha = alpha;
   info->K = K;
+  info->feature_dtype = feature_dtype;
   info->nnz = nnz;
   info->num_chunks = nch;
   info->num_blocks = nnz > 0 ? blocks_for(nnz, C, S, G, warps_per_block) : 0;

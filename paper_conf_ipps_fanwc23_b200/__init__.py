@@ -48,13 +48,13 @@ class PlanOpts(ctypes.Structure):
     """gnn_plan_opts_t; zero fields take the library defaults (alpha 2, 8 warps/block)."""
     _fields_ = [("alpha", ctypes.c_int32), ("warps_per_block", ctypes.c_int32),
                 ("force_chunk", ctypes.c_int32), ("force_vw", ctypes.c_int32),
-                ("deterministic", ctypes.c_int32)]
+                ("deterministic", ctypes.c_int32), ("feature_dtype", ctypes.c_int32)]
 
 
 class _PlanInfo(ctypes.Structure):
     _fields_ = [(n, ctypes.c_int32) for n in (
         "chunk", "vw_feat", "vw_sparse", "lanes", "vecs", "slices", "groups", "warps_per_block",
-        "active_blocks_per_sm", "num_sms", "alpha", "K")] + [
+        "active_blocks_per_sm", "num_sms", "alpha", "K", "feature_dtype")] + [
         ("nnz", ctypes.c_int64), ("num_chunks", ctypes.c_int64), ("num_blocks", ctypes.c_int64)]
 
 
@@ -65,7 +65,8 @@ class ReorderOpts(ctypes.Structure):
 
 
 EXPORTS = ["gnn_plan_workspace_bytes", "gnn_plan_create", "gnn_plan_info", "gnn_plan_arrays",
-           "gnn_plan_destroy", "gnn_spmm", "gnn_sddmm", "gnn_shard_rows", "gnn_shard_edges",
+           "gnn_plan_destroy", "gnn_spmm", "gnn_sddmm", "gnn_spmm_bf16", "gnn_sddmm_bf16",
+           "gnn_shard_rows", "gnn_shard_edges",
            "gnn_reorder_gcr", "gnn_permute_graph", "gnn_permute_rows",
            "gnn_probe_gather", "gnn_csr_to_coo", "gnn_validate", "gnn_last_error",
            "gnn_version"]
@@ -92,6 +93,9 @@ def lib():
     L.gnn_plan_destroy.restype = None
     L.gnn_spmm.argtypes = [vp, P(_Graph), vp, i64, vp, i64, vp]
     L.gnn_sddmm.argtypes = [vp, P(_Graph), vp, i64, vp, i64, vp, vp]
+    if hasattr(L, "gnn_spmm_bf16"):  # (GNN_LIB_PATH may point at an older tuning build)
+        L.gnn_spmm_bf16.argtypes = [vp, P(_Graph), vp, i64, vp, i64, vp]
+        L.gnn_sddmm_bf16.argtypes = [vp, P(_Graph), vp, i64, vp, i64, vp, vp]
     L.gnn_shard_rows.argtypes = [vp, i64, i32, vp]
     L.gnn_shard_edges.argtypes = [i64, i32, vp]
     L.gnn_csr_to_coo.argtypes = [vp, i64, i64, vp, vp]
@@ -106,8 +110,10 @@ def lib():
     L.gnn_version.restype = ctypes.c_char_p
     for f in ("gnn_plan_create", "gnn_plan_info", "gnn_plan_arrays", "gnn_spmm", "gnn_sddmm",
               "gnn_shard_rows", "gnn_shard_edges", "gnn_csr_to_coo", "gnn_validate",
-              "gnn_reorder_gcr", "gnn_permute_graph", "gnn_permute_rows", "gnn_probe_gather"):
-        getattr(L, f).restype = st
+              "gnn_reorder_gcr", "gnn_permute_graph", "gnn_permute_rows", "gnn_probe_gather",
+              "gnn_spmm_bf16", "gnn_sddmm_bf16"):
+        if hasattr(L, f):
+            getattr(L, f).restype = st
     _lib = L
     return L
 
@@ -211,15 +217,27 @@ class Plan:
             _lib.gnn_plan_destroy(h)
 
 
-def _opts(alpha=0, warps_per_block=0, force_chunk=0, force_vw=0):
-    return PlanOpts(alpha, warps_per_block, force_chunk, force_vw, 0)
+GNN_F32, GNN_BF16 = 0, 1
+
+
+def _dtype_code(d):
+    if d in (None, 0, "f32", "fp32", "float32", torch.float32):
+        return GNN_F32
+    if d in (1, "bf16", "bfloat16", torch.bfloat16):
+        return GNN_BF16
+    raise ValueError(f"unsupported feature dtype {d!r}")
+
+
+def _opts(alpha=0, warps_per_block=0, force_chunk=0, force_vw=0, feature_dtype=0):
+    return PlanOpts(alpha, warps_per_block, force_chunk, force_vw, 0, _dtype_code(feature_dtype))
 
 
 def plan(graph: DeviceGraph, K: int, alpha: int = 0, warps_per_block: int = 0,
-         force_chunk: int = 0, force_vw: int = 0, stream=None) -> Plan:
-    """gnn_plan_create: DTP/HVMA chunking + the GPU plan kernel (no host sync)."""
+         force_chunk: int = 0, force_vw: int = 0, feature_dtype=GNN_F32, stream=None) -> Plan:
+    """gnn_plan_create: DTP/HVMA chunking + the GPU plan kernel (no host sync).
+    feature_dtype: fp32 (default) or bf16 feature matrices."""
     L = lib()
-    o = _opts(alpha, warps_per_block, force_chunk, force_vw)
+    o = _opts(alpha, warps_per_block, force_chunk, force_vw, feature_dtype)
     nbytes = L.gnn_plan_workspace_bytes(graph.nnz, K, ctypes.byref(o))
     if nbytes == ctypes.c_size_t(-1).value:
         _check(GNN_ERR_INVALID_ARG)
@@ -232,36 +250,41 @@ def plan(graph: DeviceGraph, K: int, alpha: int = 0, warps_per_block: int = 0,
     return Plan(h, ws, graph, K)
 
 
-def _dense(t, name):
-    if t.dtype != torch.float32 or t.dim() != 2 or t.stride(1) != 1 or not t.is_cuda:
-        raise ValueError(f"{name} must be a CUDA fp32 row-major 2-D tensor")
+def _dense(t, name, dtypes=(torch.float32,)):
+    if t.dtype not in dtypes or t.dim() != 2 or t.stride(1) != 1 or not t.is_cuda:
+        raise ValueError(f"{name} must be a CUDA row-major 2-D tensor of {dtypes}")
     return t
+
+
+_FEAT = (torch.float32, torch.bfloat16)
 
 
 def spmm(p: Plan, graph: DeviceGraph, A: torch.Tensor, out: torch.Tensor | None = None,
          stream=None) -> torch.Tensor:
     """gnn_spmm: O = S A (overwrites out; returns it)."""
     K = p.K
-    _dense(A, "A")
+    _dense(A, "A", _FEAT)
     if out is None:
         out = torch.empty((graph.M, K), dtype=torch.float32, device=A.device)
     _dense(out, "out")
     g = graph.desc()
-    _check(lib().gnn_spmm(p.handle, ctypes.byref(g), _ptr(A), A.stride(0), _ptr(out),
-                          out.stride(0), _stream(stream)))
+    fn = lib().gnn_spmm_bf16 if A.dtype == torch.bfloat16 else lib().gnn_spmm
+    _check(fn(p.handle, ctypes.byref(g), _ptr(A), A.stride(0), _ptr(out), out.stride(0),
+              _stream(stream)))
     return out
 
 
 def sddmm(p: Plan, graph: DeviceGraph, A1: torch.Tensor, A2T: torch.Tensor,
           out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
     """gnn_sddmm: out[i] = val[i] * <A1[row_i], A2T[col_i]> (returns out)."""
-    _dense(A1, "A1")
-    _dense(A2T, "A2T")
+    _dense(A1, "A1", _FEAT)
+    _dense(A2T, "A2T", (A1.dtype,))
     if out is None:
         out = torch.empty(graph.nnz, dtype=torch.float32, device=A1.device)
     g = graph.desc()
-    _check(lib().gnn_sddmm(p.handle, ctypes.byref(g), _ptr(A1), A1.stride(0), _ptr(A2T),
-                           A2T.stride(0), _ptr(out), _stream(stream)))
+    fn = lib().gnn_sddmm_bf16 if A1.dtype == torch.bfloat16 else lib().gnn_sddmm
+    _check(fn(p.handle, ctypes.byref(g), _ptr(A1), A1.stride(0), _ptr(A2T), A2T.stride(0),
+              _ptr(out), _stream(stream)))
     return out
 
 

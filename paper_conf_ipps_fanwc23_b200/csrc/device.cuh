@@ -86,9 +86,12 @@ __device__ __forceinline__ void st_vec(float *p, const float (&x)[VW]) {
   } else if constexpr (VW == 4) {
     *reinterpret_cast<float4 *>(p) = make_float4(x[0], x[1], x[2], x[3]);
   } else {
-    asm volatile("st.global.v8.f32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "f"(x[0]),
-                 "f"(x[1]), "f"(x[2]), "f"(x[3]), "f"(x[4]), "f"(x[5]), "f"(x[6]), "f"(x[7])
-                 : "memory");
+#pragma unroll
+    for (int h = 0; h < VW; h += 8)
+      asm volatile("st.global.v8.f32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p + h),
+                   "f"(x[h]), "f"(x[h + 1]), "f"(x[h + 2]), "f"(x[h + 3]), "f"(x[h + 4]),
+                   "f"(x[h + 5]), "f"(x[h + 6]), "f"(x[h + 7])
+                   : "memory");
   }
 }
 
@@ -168,6 +171,94 @@ __device__ __forceinline__ float dot_acc(float d, const float (&a)[VW], const fl
   return d;
 }
 
+// ---------------------------------------------------------- feature types ----
+// Gathered feature rows are fp32 or bf16; arithmetic and outputs are
+// fp32 either way.  FeatVec<TF, VW> holds one VW-element vector as loaded (bf16 stays
+// packed two per register, widened exactly to fp32 when consumed: bf16 -> fp32 is a
+// 16-bit shift).
+struct F32 {
+  static constexpr int bytes = 4;
+};
+struct BF16 {
+  static constexpr int bytes = 2;
+};
+
+template <typename TF, int VW>
+struct FeatVec;
+
+template <int VW>
+struct FeatVec<F32, VW> {
+  float r[VW];
+  __device__ __forceinline__ void load(const char *p) {
+    ld_feat<VW>(reinterpret_cast<const float *>(p), r);
+  }
+  __device__ __forceinline__ void zero() {
+#pragma unroll
+    for (int v = 0; v < VW; ++v) r[v] = 0.f;
+  }
+  __device__ __forceinline__ float get(int v) const { return r[v]; }
+};
+
+template <int VW>
+struct FeatVec<BF16, VW> {
+  static_assert(VW % 2 == 0 && VW <= 16, "bf16 vectors hold 2..16 elements");
+  uint32_t r[VW / 2];
+  __device__ __forceinline__ void load(const char *p) {
+    if constexpr (VW == 16) {
+      asm("ld.global.nc.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+          : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+            "=r"(r[7])
+          : "l"(p));
+    } else if constexpr (VW == 8) {
+      asm("ld.global.nc.v4.b32 {%0,%1,%2,%3}, [%4];"
+          : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3])
+          : "l"(p));
+    } else if constexpr (VW == 4) {
+      asm("ld.global.nc.v2.b32 {%0,%1}, [%2];" : "=r"(r[0]), "=r"(r[1]) : "l"(p));
+    } else {
+      asm("ld.global.nc.b32 %0, [%1];" : "=r"(r[0]) : "l"(p));
+    }
+  }
+  __device__ __forceinline__ void zero() {
+#pragma unroll
+    for (int v = 0; v < VW / 2; ++v) r[v] = 0u;
+  }
+  __device__ __forceinline__ float get(int v) const {
+    return (v & 1) ? __uint_as_float(r[v >> 1] & 0xffff0000u) : __uint_as_float(r[v >> 1] << 16);
+  }
+};
+
+// acc[v] += s * x[v] (FFMA2 pairs)
+template <typename TF, int VW>
+__device__ __forceinline__ void axpy_f(float (&acc)[VW], float s, const FeatVec<TF, VW> &x) {
+#if GNN_USE_FFMA2
+  if constexpr (VW >= 2) {
+#pragma unroll
+    for (int v = 0; v < VW; v += 2) fma2_bcast(acc[v], acc[v + 1], s, x.get(v), x.get(v + 1));
+    return;
+  }
+#endif
+#pragma unroll
+  for (int v = 0; v < VW; ++v) acc[v] = fmaf(s, x.get(v), acc[v]);
+}
+
+// d + sum_v a[v] * x[v] (two interleaved FFMA2 chains for VW >= 4)
+template <typename TF, int VW>
+__device__ __forceinline__ float dot_f(float d, const FeatVec<TF, VW> &a,
+                                       const FeatVec<TF, VW> &x) {
+#if GNN_USE_FFMA2
+  if constexpr (VW >= 4) {
+    float e0 = 0.f, e1 = 0.f;
+#pragma unroll
+    for (int v = 0; v < VW; v += 2) fma2_pair(e0, e1, a.get(v), a.get(v + 1), x.get(v), x.get(v + 1));
+    return d + (e0 + e1);
+  }
+#endif
+#pragma unroll
+  for (int v = 0; v < VW; ++v) d = fmaf(a.get(v), x.get(v), d);
+  return d;
+}
+
 // -------------------------------------------------------------- sparse ----
 // Load VWS consecutive entries starting at index i (vector when the whole vector is
 // in range; element-wise with a default otherwise).  The base pointer + i is
@@ -227,5 +318,61 @@ __device__ __forceinline__ void ld_sparse_f32(const float *p, int64_t i, int64_t
     for (int q = 0; q < VWS; ++q) x[q] = (i + q < end) ? __ldg(p + i + q) : 0.f;
   }
 }
+
+// ------------------------------------------------------- sparse tiles ----
+// The streamed sparse arrays are staged through a per-warp, double-buffered shared
+// memory ring with cp.async (LDGSTS, L1-bypassing for 16-byte copies): the next tile
+// is in flight while the current one is consumed, and no registers hold tiles.  Each
+// lane group's tile of T = L * VWS nonzeros sits at a padded stride of T + 4 words so
+// that the groups of a warp hit different banks when they read "their" nonzero.
+template <int BYTES>
+__device__ __forceinline__ void cp_async(void *smem_dst, const void *gsrc, int src_bytes) {
+  const uint32_t d = (uint32_t)__cvta_generic_to_shared(smem_dst);
+  if constexpr (BYTES == 16) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(d), "l"(gsrc),
+                 "r"(src_bytes)
+                 : "memory");
+  } else {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], %2, %3;" ::"r"(d), "l"(gsrc),
+                 "n"(BYTES), "r"(src_bytes)
+                 : "memory");
+  }
+}
+__device__ __forceinline__ void cp_async_commit() {
+  asm volatile("cp.async.commit_group;" ::: "memory");
+}
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+
+template <int L, int VWS>
+struct SparseTiles {
+  static constexpr int G = 32 / L;
+  static constexpr int T = L * VWS;        // nonzeros per tile per lane group
+  static constexpr int STRIDE = T + 4;     // words per group (bank padding, 16-B aligned)
+  static constexpr int WORDS = G * STRIDE;  // words per array per stage
+  static constexpr int WARP_WORDS = 2 * 3 * WORDS;
+  static constexpr int BYTES_PER_WARP = WARP_WORDS * 4;
+  int32_t *w;  // this warp's region: [stage][row|col|val][G * STRIDE]
+  __device__ __forceinline__ int32_t *rows(int st, int g) const { return w + (st * 3 + 0) * WORDS + g * STRIDE; }
+  __device__ __forceinline__ int32_t *cols(int st, int g) const { return w + (st * 3 + 1) * WORDS + g * STRIDE; }
+  __device__ __forceinline__ float *vals(int st, int g) const {
+    return reinterpret_cast<float *>(w + (st * 3 + 2) * WORDS + g * STRIDE);
+  }
+  // Lane l of group g copies entries [tb + l*VWS, +VWS) of its chunk (n valid entries;
+  // the rest zero-filled) into stage st.
+  __device__ __forceinline__ void load(int st, int g, int l, const int32_t *ri, const int32_t *ci,
+                                       const float *vi, int tb, int n) const {
+    const int i = tb + l * VWS;
+    int cnt = n - i;
+    cnt = cnt < 0 ? 0 : (cnt > VWS ? VWS : cnt);
+    const int bytes = cnt * 4;
+    const int off = cnt > 0 ? i : 0;  // no bytes are read when cnt == 0
+    cp_async<4 * VWS>(rows(st, g) + l * VWS, ri + off, bytes);
+    cp_async<4 * VWS>(cols(st, g) + l * VWS, ci + off, bytes);
+    if (vi) cp_async<4 * VWS>(vals(st, g) + l * VWS, vi + off, bytes);
+  }
+};
 
 }  // namespace gnn

@@ -52,7 +52,7 @@ struct SparseArgs {
 
 // Occupancy (active blocks / SM) of the SpMM kernel for a feature width/lane count;
 // DTP's ActiveblocksPerSM (Eq. 3) -- defined in spmm.cu.
-int spmm_active_blocks_per_sm(int vw, int lanes, int vecs, int warps_per_block);
+int spmm_active_blocks_per_sm(int dtype, int vw, int lanes, int vecs, int warps_per_block);
 
 // Shared launcher helpers (spmm.cu).
 gnn_status_t check_common(const Plan *p, const gnn_graph_t *g, const char *who);

@@ -36,21 +36,25 @@ gnn_status_t make_info(int64_t nnz, int32_t K, const gnn_plan_opts_t *opts,
     return fail(GNN_ERR_INVALID_ARG,
                 "plan: bad arguments (nnz=%lld K=%d alpha=%d wpb=%d force_chunk=%d det=%d)",
                 (long long)nnz, K, alpha, wpb, o.force_chunk, o.deterministic);
-  // step 1: feature vector width from K alone (or forced)
+  // step 1: feature vector width (elements of the feature dtype) from K alone, or forced;
+  // the widest of 256/128/64/32-bit that divides the row
+  const int32_t dt = o.feature_dtype;
+  if (dt != GNN_F32 && dt != GNN_BF16)
+    return fail(GNN_ERR_INVALID_ARG, "plan: feature_dtype %d unknown", dt);
+  const int32_t vmax = dt == GNN_BF16 ? 16 : 8, vmin = dt == GNN_BF16 ? 2 : 1;
   int32_t vw;
   if (o.force_vw) {
-    if (!(o.force_vw == 1 || o.force_vw == 2 || o.force_vw == 4 || o.force_vw == 8) ||
-        K % o.force_vw)
-      return fail(GNN_ERR_INVALID_ARG, "plan: force_vw=%d invalid for K=%d", o.force_vw, K);
+    bool ok = false;
+    for (int32_t v = vmin; v <= vmax; v *= 2) ok |= (o.force_vw == v);
+    if (!ok || K % o.force_vw)
+      return fail(GNN_ERR_INVALID_ARG, "plan: force_vw=%d invalid for K=%d (dtype %d)",
+                  o.force_vw, K, dt);
     vw = o.force_vw;
-  } else if (K % 8 == 0) {
-    vw = 8;
-  } else if (K % 4 == 0) {
-    vw = 4;
-  } else if (K % 2 == 0) {
-    vw = 2;
   } else {
-    vw = 1;
+    vw = 0;
+    for (int32_t v = vmax; v >= vmin && !vw; v /= 2)
+      if (K % v == 0) vw = v;
+    if (!vw) return fail(GNN_ERR_INVALID_ARG, "plan: bf16 features need an even K (K=%d)", K);
   }
   // step 2: vectors per lane, lanes per chunk-slice, slices, chunk-slices per warp
   const int64_t need = cdiv(K, vw);  // VW-wide vectors in a feature row
@@ -62,7 +66,7 @@ gnn_status_t make_info(int64_t nnz, int32_t K, const gnn_plan_opts_t *opts,
   // step 3: FullWaveSize (Eqs. 3-4) from the occupancy of the SpMM kernel
   DeviceInfo d;
   if (gnn_status_t st = device_info(&d)) return st;
-  const int32_t abs = spmm_active_blocks_per_sm(vw, L, R, wpb);
+  const int32_t abs = spmm_active_blocks_per_sm(dt, vw, L, R, wpb);
   if (abs < 1) return fail(GNN_ERR_CUDA, "plan: occupancy query failed (vw=%d L=%d)", vw, L);
   const int64_t FW = (int64_t)d.num_sms * abs;
   // steps 4-5: the largest candidate satisfying InEq. (5); none -> 8
@@ -87,6 +91,7 @@ gnn_status_t make_info(int64_t nnz, int32_t K, const gnn_plan_opts_t *opts,
   info->num_sms = d.num_sms;
   info->alpha = alpha;
   info->K = K;
+  info->feature_dtype = dt;
   info->nnz = nnz;
   info->num_chunks = nnz > 0 ? cdiv(nnz, C) : 0;
   info->num_blocks = nnz > 0 ? blocks_for(nnz, C, S, G, wpb) : 0;

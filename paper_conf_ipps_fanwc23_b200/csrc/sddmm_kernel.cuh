@@ -1,0 +1,275 @@
+// sddmm_kernel.cuh -- the hybrid-parallel SDDMM kernel template (design notes in
+// sddmm.cu) and its dispatch table; instantiated per feature type in sddmm_f32.cu /
+// sddmm_bf16.cu.
+#pragma once
+#include <type_traits>
+
+#include "device.cuh"
+#include "internal.cuh"
+
+namespace gnn {
+
+// Lane mapping of SDDMM.  A K-slice holds V = L * R VW-wide vectors (plan rule step 2);
+// SDDMM spreads them over Lg = V / Rsd lanes with Rsd vectors per lane, so each dot
+// product is reduced over Lg lanes and 32 / Lg nonzeros are in flight per warp step;
+// U = nonzeros per batch per group, U * Rsd = 8 feature vectors in flight per lane.
+// Measured on the GCR-reordered C4 (profiles/r01_sweep8.txt): Rsd = 2 from V = 8 on
+// (K=64: 2.07 -> 1.94 ms, K=128: 4.82 -> 3.61 ms, K=256: 8.85 -> 7.05 ms), 1 below.
+#ifndef GNN_SDDMM_R2_FROM
+#define GNN_SDDMM_R2_FROM 8  // smallest V that uses Rsd = 2
+#endif
+#ifndef GNN_SDDMM_UR
+#define GNN_SDDMM_UR 8       // U * Rsd: feature vectors in flight per lane
+#endif
+template <int VW, int V, int SMAX>
+struct SddmmShape {
+  static constexpr int R = (V >= GNN_SDDMM_R2_FROM && V >= 2) ? 2 : 1;
+  static constexpr int Lg = V / R;
+  static constexpr int depth = GNN_SDDMM_UR / R > 1 ? GNN_SDDMM_UR / R : 1;
+#if defined(GNN_SDDMM_MINB)
+  static constexpr int minb = GNN_SDDMM_MINB;
+#else
+  static constexpr int minb = 1;
+#endif
+};
+
+// WarpReduce (Algo 4 line 12) of U partial dot products at once over the group's L
+// lanes, as a transposed butterfly: each halving step exchanges half of the values
+// (U/2 + U/4 + ... shuffles instead of U * log2 L).  Afterwards value u lives in lane
+// l with u = l * U / L (U <= L; lanes l % (L/U) == 0 are its owners) or, for U > L, in
+// slot i of lane l with u = l * (U/L) + i.  Then S_O = sum * v (Algo 2 line 6) is
+// stored for the first `valid` of the U nonzeros at out[0..U).
+template <int U, int L>
+__device__ __forceinline__ void reduce_scale_store(float (&part)[U], const float (&vj)[U],
+                                                   const int l, float *__restrict__ out,
+                                                   const int valid) {
+  constexpr int P = U > L ? U / L : 1;  // values left per lane after the halving steps
+  int cnt = U;
+#pragma unroll
+  for (int o = L / 2; o >= 1; o >>= 1) {
+    if (cnt > 1) {
+      const int half = cnt / 2;
+      const bool b = (l & o) != 0;
+#pragma unroll
+      for (int i = 0; i < U / 2; ++i) {
+        if (i < half) {
+          const float lo = part[i], hi = part[i + half];
+          const float send = b ? lo : hi;
+          const float keep = b ? hi : lo;
+          part[i] = keep + __shfl_xor_sync(kFull, send, o, L);
+        }
+      }
+      cnt = half;
+    } else {
+      part[0] += __shfl_xor_sync(kFull, part[0], o, L);
+    }
+  }
+  if constexpr (U <= L) {
+    constexpr int R = L / U;
+    const int u = l / R;
+    if (l % R == 0 && u < valid) {
+      float v = vj[0];
+#pragma unroll
+      for (int w = 1; w < U; ++w) v = (w == u) ? vj[w] : v;
+      out[u] = part[0] * v;
+    }
+  } else {
+#pragma unroll
+    for (int i = 0; i < P; ++i) {
+      const int u = l * P + i;
+      if (u < valid) {
+        float v = vj[0];
+#pragma unroll
+        for (int w = 1; w < U; ++w) v = (w == u) ? vj[w] : v;
+        out[u] = part[i] * v;
+      }
+    }
+  }
+}
+
+// L here is V, the number of VW-wide vectors in one K-slice (plan lanes x vecs).
+template <typename TF, int VW, int L, int VWS, int SMAX>
+__global__ void __launch_bounds__(kMaxThreads, (SddmmShape<VW, L, SMAX>::minb))
+    sddmm_kernel(const SparseArgs a, const void *__restrict__ A1, const int64_t lda1,
+                 const void *__restrict__ A2T, const int64_t lda2, float *__restrict__ out) {
+  constexpr int ES = TF::bytes;
+  using Sh = SddmmShape<VW, L, SMAX>;
+  constexpr int R = Sh::R, Lg = Sh::Lg;
+  constexpr int G = 32 / Lg;
+  constexpr int T = Lg * VWS;
+  constexpr int U0 = Sh::depth > VWS ? Sh::depth : VWS;
+  constexpr int U = U0 < T ? U0 : T;
+  static_assert(T % U == 0 && U % VWS == 0, "tile / prefetch shape");
+  const int lane = threadIdx.x & 31;
+  const int g = lane / Lg;
+  const int l = lane & (Lg - 1);
+  const int64_t c = ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * G + g;
+  const bool item_ok = c < a.num_chunks;
+  if (!__any_sync(kFull, item_ok)) return;
+  const int64_t cs = c * a.chunk;
+  const int n = item_ok ? (int)(min(cs + (int64_t)a.chunk, a.nnz) - cs) : 0;
+  const int S = a.slices;  // <= SMAX (host-checked)
+  const uint32_t ld2B = (uint32_t)lda2 * (uint32_t)ES;
+  const char *__restrict__ A2b = reinterpret_cast<const char *>(A2T);
+
+  // column of vector r of slice sl owned by lane l: (sl*L + r*Lg + l) * VW
+  FeatVec<TF, VW> a1[SMAX][R];
+  int32_t cur[SMAX];  // row whose A1 slice is cached, per slice
+#pragma unroll
+  for (int sl = 0; sl < SMAX; ++sl) {
+    cur[sl] = -1;
+#pragma unroll
+    for (int r = 0; r < R; ++r) a1[sl][r].zero();
+  }
+
+  const int32_t *__restrict__ ri = a.row_ind + cs;
+  const int32_t *__restrict__ ci = a.col_ind + cs;
+  const float *__restrict__ vi = a.val ? a.val + cs : nullptr;
+  float *__restrict__ oc = out + cs;
+  // sparse tiles: per-warp double-buffered shared-memory ring filled with cp.async
+  extern __shared__ int32_t gnn_smem[];
+  using Tiles = SparseTiles<Lg, VWS>;
+  const Tiles tiles{gnn_smem + (threadIdx.x >> 5) * Tiles::WARP_WORDS};
+  tiles.load(0, g, l, ri, ci, vi, 0, n);
+  cp_async_commit();
+
+  auto load_a1_slice = [&](int sl, int32_t row) {
+    const char *base = reinterpret_cast<const char *>(A1) +
+                       (((int64_t)row - a.row_base) * lda1 + (sl * L + l) * VW) * ES;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      const int k0 = (sl * L + r * Lg + l) * VW;
+      if (k0 < a.K) a1[sl][r].load(base + r * Lg * VW * ES);
+    }
+    cur[sl] = row;
+  };
+
+  const int ntiles = (a.chunk + T - 1) / T;
+  for (int t = 0; t < ntiles; ++t) {
+    const int tb = t * T;
+    const int st = t & 1;
+    __syncwarp();  // every lane is done with the stage the next copy overwrites
+    if (t + 1 < ntiles) tiles.load(st ^ 1, g, l, ri, ci, vi, tb + T, n);
+    cp_async_commit();
+    cp_async_wait<1>();
+    __syncwarp();
+    const int32_t *s_row = tiles.rows(st, g);
+    const int32_t *s_col = tiles.cols(st, g);
+    const float *s_val = tiles.vals(st, g);
+    const int32_t r_first = s_row[0];
+    const bool fast =
+        __all_sync(kFull, ((tb + T <= n) && r_first == s_row[T - 1]) || !item_ok);
+    if (fast && item_ok && r_first != cur[0]) {  // row switch at the tile start
+#pragma unroll
+      for (int sl = 0; sl < SMAX; ++sl)
+        if (sl < S) load_a1_slice(sl, r_first);
+    }
+    // The batch loop is instantiated twice: FAST (whole tile in one row, every nonzero
+    // valid: no per-nonzero row or bounds logic) and general.
+    auto run_tile = [&](auto fast_tag) {
+      constexpr bool FAST = decltype(fast_tag)::value;
+#pragma unroll 1
+      for (int jj = 0; jj < T; jj += U) {
+        int32_t rj[U];
+        uint32_t cj[U];
+        float vj[U], part[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          cj[u] = (uint32_t)s_col[jj + u];
+          vj[u] = vi ? s_val[jj + u] : 1.f;
+          if constexpr (!FAST) rj[u] = s_row[jj + u];
+          part[u] = 0.f;
+        }
+        const int valid = n - (tb + jj);
+#pragma unroll
+        for (int sl = 0; sl < SMAX; ++sl) {
+          if (sl < S) {
+            // this lane's first element of slice sl; vector r sits r*Lg*VW elements on
+            const char *A2l = A2b + (int64_t)((sl * L + l) * VW) * ES;
+            bool lane_ok[R];
+#pragma unroll
+            for (int r = 0; r < R; ++r) lane_ok[r] = item_ok && (sl * L + r * Lg + l) * VW < a.K;
+            FeatVec<TF, VW> x[U][R];
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+              const char *rowp = A2l + (uint64_t)cj[u] * ld2B;
+#pragma unroll
+              for (int r = 0; r < R; ++r) {
+                if (lane_ok[r] && (FAST || u < valid)) x[u][r].load(rowp + r * Lg * VW * ES);
+                else x[u][r].zero();
+              }
+            }
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+              if constexpr (!FAST) {
+                if (item_ok && u < valid && rj[u] != cur[sl]) {
+                  // row-switch procedure: load the new A1 row (Algo 4 lines 8-11)
+                  load_a1_slice(sl, rj[u]);
+                }
+              }
+#pragma unroll
+              for (int r = 0; r < R; ++r) part[u] = dot_f<TF, VW>(part[u], a1[sl][r], x[u][r]);
+            }
+          }
+        }
+        reduce_scale_store<U, Lg>(part, vj, l, oc + tb + jj, item_ok ? (FAST ? U : valid) : 0);
+      }
+    };
+    if (fast) run_tile(std::true_type{});
+    else run_tile(std::false_type{});
+  }
+}
+
+using SddmmFn = void (*)(const SparseArgs, const void *__restrict__, const int64_t,
+                         const void *__restrict__, const int64_t, float *__restrict__);
+
+template <typename TF, int VW, int V, int SMAX>
+SddmmFn pick_sddmm_vws(int vws) {
+  // a batch must cover whole sparse vectors: narrow the sparse loads when U < vw_sparse
+  constexpr int D = SddmmShape<VW, V, SMAX>::depth;
+  while (vws > D) vws >>= 1;
+  switch (vws) {
+    case 1: return sddmm_kernel<TF, VW, V, 1, SMAX>;
+    case 2: return sddmm_kernel<TF, VW, V, 2, SMAX>;
+    case 4: return sddmm_kernel<TF, VW, V, 4, SMAX>;
+  }
+  return nullptr;
+}
+template <typename TF, int VW>
+SddmmFn pick_sddmm_v(int V, int vws, int S) {
+  if (S > 1) return V == 64 ? pick_sddmm_vws<TF, VW, 64, 4>(vws) : nullptr;
+  switch (V) {
+    case 1: return pick_sddmm_vws<TF, VW, 1, 1>(vws);
+    case 2: return pick_sddmm_vws<TF, VW, 2, 1>(vws);
+    case 4: return pick_sddmm_vws<TF, VW, 4, 1>(vws);
+    case 8: return pick_sddmm_vws<TF, VW, 8, 1>(vws);
+    case 16: return pick_sddmm_vws<TF, VW, 16, 1>(vws);
+    case 32: return pick_sddmm_vws<TF, VW, 32, 1>(vws);
+    case 64: return pick_sddmm_vws<TF, VW, 64, 1>(vws);
+  }
+  return nullptr;
+}
+// defined in sddmm_f32.cu / sddmm_bf16.cu (V = L * R vectors per slice, S <= 4 slices)
+SddmmFn pick_sddmm_f32(int vw, int V, int vws, int S);
+SddmmFn pick_sddmm_bf16(int vw, int V, int vws, int S);
+
+// dynamic shared memory per warp of the instantiation with Lg lanes per dot product
+inline int sddmm_tile_bytes_per_warp(int lg, int vws) {
+  return 2 * 3 * (32 / lg) * (lg * vws + 4) * 4;
+}
+// the vw_sparse the dispatcher actually instantiates (a batch must cover whole vectors)
+inline int sddmm_effective_vws(int V, int S, int vws) {
+  const int r = S > 1 ? 2 : ((V >= GNN_SDDMM_R2_FROM && V >= 2) ? 2 : 1);
+  int depth = GNN_SDDMM_UR / r;
+  if (depth < 1) depth = 1;
+  while (vws > depth) vws >>= 1;
+  return vws;
+}
+
+// lanes per dot product of the instantiation pick_sddmm_* returns
+inline int sddmm_group_lanes(int V, int S) {
+  if (S > 1) return SddmmShape<8, 64, 4>::Lg;
+  const int r = (V >= GNN_SDDMM_R2_FROM && V >= 2) ? 2 : 1;
+  return V / r;
+}
+}  // namespace gnn

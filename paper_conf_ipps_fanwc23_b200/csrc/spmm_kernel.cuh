@@ -1,0 +1,272 @@
+// spmm_kernel.cuh -- the hybrid-parallel SpMM kernel template (see spmm.cu for the
+// design notes) and its dispatch table; instantiated per feature type in
+// spmm_f32.cu / spmm_bf16.cu so the two halves compile in parallel.
+#pragma once
+#include "device.cuh"
+#include "internal.cuh"
+
+namespace gnn {
+
+// Feature rows in flight per lane (U) and the register budget, per instantiation.
+// Measured on C4 (profiles/r01_sweep4.txt): with 256-bit loads U = 4 is best while
+// several chunks share a warp (L <= 8), U = 8 once a group spans >= 16 lanes.
+#ifndef GNN_SPMM_MINB
+#define GNN_SPMM_MINB 1  // min resident 512-thread blocks/SM the register budget must allow
+#endif
+
+// Feature vectors in flight per lane.  Measured on C4 (profiles/r01_sweep4.txt,
+// r01_sweep11.txt): 4 while several chunks share a warp (L <= 8, R = 1), 8 for wider
+// groups and whenever a lane holds R = 2 vectors per row.
+#ifndef GNN_SPMM_DEPTH_R2
+#define GNN_SPMM_DEPTH_R2 4
+#endif
+template <typename TF, int VW, int L, int R>
+struct FeatDepth {
+  static constexpr bool wide = VW * TF::bytes == 32;  // 256-bit vectors
+#if defined(GNN_SPMM_DEPTH8)
+  static constexpr int value = wide ? GNN_SPMM_DEPTH8 : 8;
+#else
+  static constexpr int value = R == 2 ? GNN_SPMM_DEPTH_R2 : (wide ? (L >= 16 ? 8 : 4) : 8);
+#endif
+};
+
+// Flush the accumulator of row `cur` (Algo 3 line 15, "AtomicStore"): rows shared
+// with a neighbouring chunk are combined with a vector atomic add, rows owned by this
+// chunk get a plain vector store.
+template <int VW>
+__device__ __forceinline__ void flush_row(float *Ok, int64_t ldo, int64_t row_base, int32_t cur,
+                                          int32_t rf, int32_t rl, uint32_t fl,
+                                          const float (&acc)[VW]) {
+  float *o = Ok + ((int64_t)cur - row_base) * ldo;
+  const bool shared = (cur == rf && (fl & 1u)) || (cur == rl && (fl & 2u));
+  if (shared) red_add<VW>(o, acc);
+  else st_vec<VW>(o, acc);
+}
+
+// L lanes per (chunk, K-slice) work item, R VW-wide vectors per lane (plan rule step 2).
+// TF: feature element type (F32 or BF16); accumulation and O are fp32.
+template <typename TF, int VW, int L, int R, int VWS>
+__global__ void __launch_bounds__(kMaxThreads, GNN_SPMM_MINB)
+    spmm_kernel(const SparseArgs a, const void *__restrict__ A, const int64_t lda,
+                float *__restrict__ O, const int64_t ldo) {
+  constexpr int ES = TF::bytes;
+  constexpr int Lg = L;
+  constexpr int G = 32 / Lg;
+  constexpr int T = Lg * VWS;  // nonzeros per tile per group
+  // U nonzeros per batch: FeatDepth vectors in flight per lane, whole sparse vectors
+  constexpr int D = FeatDepth<TF, VW, L, R>::value / R;
+  constexpr int U = D > T ? T : (D < VWS ? VWS : D);
+  static_assert(T % U == 0 && U % VWS == 0, "tile / prefetch shape");
+  const int lane = threadIdx.x & 31;
+  const int g = lane / Lg;
+  const int l = lane & (Lg - 1);
+  const int64_t item = ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * G + g;
+  const bool item_ok = item < a.num_chunks * a.slices;
+  if (!__any_sync(kFull, item_ok)) return;  // warp-uniform exit
+
+  int64_t c = 0;
+  int s = 0;
+  if (item_ok) {
+    c = item / a.slices;
+    s = (int)(item - c * a.slices);
+  }
+  // vector r of this lane covers columns k0 + r * L * VW .. + VW of slice s
+  const int k0 = (s * L * R + l) * VW;
+  bool col_ok[R];
+#pragma unroll
+  for (int r = 0; r < R; ++r) col_ok[r] = item_ok && k0 + r * Lg * VW < a.K;
+  const int64_t cs = c * a.chunk;
+  const int n = item_ok ? (int)(min(cs + (int64_t)a.chunk, a.nnz) - cs) : 0;  // nnz here
+  int32_t rf = 0, rl = 0;
+  uint32_t fl = 0;
+  if (item_ok) {
+    rf = a.row_first[c];
+    rl = a.row_last[c];
+    fl = a.flags[c];
+  }
+  // feature row c of A starts at Ab + c * ldaB (IMAD.WIDE.U32 per gather)
+  const char *__restrict__ Ab = reinterpret_cast<const char *>(A) + (int64_t)k0 * ES;
+  const uint32_t ldaB = (uint32_t)lda * (uint32_t)ES;
+  float *__restrict__ Ok = O + k0;  // row r at Ok + (r - row_base) * ldo
+
+  auto zero_row = [&](int64_t row) {
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+      if (col_ok[r]) st_zero<VW>(Ok + (row - a.row_base) * ldo + r * Lg * VW);
+  };
+  float acc[R][VW];
+  auto flush = [&](int32_t row) {
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+      if (col_ok[r])
+        flush_row<VW>(Ok + r * Lg * VW, ldo, a.row_base, row, rf, rl, fl, acc[r]);
+  };
+
+  // empty rows between the previous chunk's last row and ours are ours to zero
+  if (item_ok) {
+    const int64_t prev = (c == 0) ? a.row_base - 1 : (int64_t)a.row_last[c - 1];
+    for (int64_t r = prev + 1; r < rf; ++r) zero_row(r);
+  }
+
+#pragma unroll
+  for (int r = 0; r < R; ++r)
+#pragma unroll
+    for (int v = 0; v < VW; ++v) acc[r][v] = 0.f;
+  int32_t cur = -1;
+
+  const int32_t *__restrict__ ri = a.row_ind + cs;
+  const int32_t *__restrict__ ci = a.col_ind + cs;
+  const float *__restrict__ vi = a.val ? a.val + cs : nullptr;
+  // sparse tiles: per-warp double-buffered shared-memory ring filled with cp.async
+  extern __shared__ int32_t gnn_smem[];
+  using Tiles = SparseTiles<L, VWS>;
+  const Tiles tiles{gnn_smem + (threadIdx.x >> 5) * Tiles::WARP_WORDS};
+  tiles.load(0, g, l, ri, ci, vi, 0, n);
+  cp_async_commit();
+
+  const int ntiles = (a.chunk + T - 1) / T;  // warp-uniform trip count
+  for (int t = 0; t < ntiles; ++t) {
+    const int tb = t * T;
+    const int st = t & 1;
+    __syncwarp();  // every lane is done with the stage the next copy overwrites
+    if (t + 1 < ntiles) tiles.load(st ^ 1, g, l, ri, ci, vi, tb + T, n);
+    cp_async_commit();
+    cp_async_wait<1>();  // this lane's copies of tile t have landed
+    __syncwarp();        // ... and every other lane's
+    const int32_t *s_row = tiles.rows(st, g);
+    const int32_t *s_col = tiles.cols(st, g);
+    const float *s_val = tiles.vals(st, g);
+    const int32_t r_first = s_row[0];
+    const bool fast_g = (tb + T <= n) && r_first == s_row[T - 1];
+    if (__all_sync(kFull, fast_g || !item_ok)) {
+      // ---- fast path: the whole tile belongs to one row (all groups of the warp)
+      if (item_ok && r_first != cur) {
+        if (cur >= 0) {
+          flush(cur);
+          for (int64_t r = (int64_t)cur + 1; r < r_first; ++r) zero_row(r);
+        }
+        cur = r_first;
+#pragma unroll
+        for (int r = 0; r < R; ++r)
+#pragma unroll
+          for (int v = 0; v < VW; ++v) acc[r][v] = 0.f;
+      }
+#pragma unroll 1
+      for (int jj = 0; jj < T; jj += U) {
+        uint32_t cj[U];
+        float vj[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          cj[u] = (uint32_t)s_col[jj + u];
+          vj[u] = vi ? s_val[jj + u] : 1.f;
+        }
+        FeatVec<TF, VW> x[U][R];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          const char *rowp = Ab + (uint64_t)cj[u] * ldaB;
+#pragma unroll
+          for (int r = 0; r < R; ++r) {
+            if (col_ok[r]) x[u][r].load(rowp + r * Lg * VW * ES);
+            else x[u][r].zero();
+          }
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+#pragma unroll
+          for (int r = 0; r < R; ++r) axpy_f<TF, VW>(acc[r], vj[u], x[u][r]);
+      }
+    } else {
+      // ---- general path: per-nonzero validity and row-switch procedure
+#pragma unroll 1
+      for (int jj = 0; jj < T; jj += U) {
+        int32_t rj[U];
+        uint32_t cj[U];
+        float vj[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          rj[u] = s_row[jj + u];
+          cj[u] = (uint32_t)s_col[jj + u];
+          vj[u] = vi ? s_val[jj + u] : 1.f;
+        }
+        FeatVec<TF, VW> x[U][R];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          const char *rowp = Ab + (uint64_t)cj[u] * ldaB;
+#pragma unroll
+          for (int r = 0; r < R; ++r) {
+            if (col_ok[r] && tb + jj + u < n) x[u][r].load(rowp + r * Lg * VW * ES);
+            else x[u][r].zero();
+          }
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          if (tb + jj + u < n) {
+            if (rj[u] != cur) {  // row-switch procedure
+              if (cur >= 0) {
+                flush(cur);
+                for (int64_t r = (int64_t)cur + 1; r < rj[u]; ++r) zero_row(r);
+              }
+              cur = rj[u];
+#pragma unroll
+              for (int r = 0; r < R; ++r)
+#pragma unroll
+                for (int v = 0; v < VW; ++v) acc[r][v] = 0.f;
+            }
+#pragma unroll
+            for (int r = 0; r < R; ++r) axpy_f<TF, VW>(acc[r], vj[u], x[u][r]);
+          }
+        }
+      }
+    }
+  }
+  if (cur >= 0) flush(cur);
+  // trailing empty rows after the last chunk
+  if (item_ok && c == a.num_chunks - 1) {
+    for (int64_t r = (int64_t)rl + 1; r < a.row_base + a.M; ++r) zero_row(r);
+  }
+}
+
+using SpmmFn = void (*)(const SparseArgs, const void *__restrict__, const int64_t,
+                        float *__restrict__, const int64_t);
+
+template <typename TF, int VW, int L, int R>
+SpmmFn spmm_pick_vws(int vws) {
+  switch (vws) {
+    case 1: return spmm_kernel<TF, VW, L, R, 1>;
+    case 2: return spmm_kernel<TF, VW, L, R, 2>;
+    case 4: return spmm_kernel<TF, VW, L, R, 4>;
+  }
+  return nullptr;
+}
+template <typename TF, int VW>
+SpmmFn spmm_pick_l(int L, int R, int vws) {
+  if (R == 2) {  // the plan uses R = 2 only for rows of >= 16 vectors, i.e. L >= 8
+    switch (L) {
+      case 8: return spmm_pick_vws<TF, VW, 8, 2>(vws);
+      case 16: return spmm_pick_vws<TF, VW, 16, 2>(vws);
+      case 32: return spmm_pick_vws<TF, VW, 32, 2>(vws);
+    }
+    return nullptr;
+  }
+  switch (L) {
+    case 1: return spmm_pick_vws<TF, VW, 1, 1>(vws);
+    case 2: return spmm_pick_vws<TF, VW, 2, 1>(vws);
+    case 4: return spmm_pick_vws<TF, VW, 4, 1>(vws);
+    case 8: return spmm_pick_vws<TF, VW, 8, 1>(vws);
+    case 16: return spmm_pick_vws<TF, VW, 16, 1>(vws);
+    case 32: return spmm_pick_vws<TF, VW, 32, 1>(vws);
+  }
+  return nullptr;
+}
+
+// dynamic shared memory of spmm_kernel<.., L, .., VWS> per warp
+inline int spmm_tile_bytes_per_warp(int L, int vws) {
+  const int T = L * vws;
+  return 2 * 3 * (32 / L) * (T + 4) * 4;
+}
+
+// defined in spmm_f32.cu / spmm_bf16.cu
+SpmmFn pick_spmm_f32(int vw, int L, int R, int vws);
+SpmmFn pick_spmm_bf16(int vw, int L, int R, int vws);
+
+}  // namespace gnn

@@ -408,3 +408,46 @@ def test_full_size_sampled_parity(name, Ks, reorder):
         assert_within(E[torch.from_numpy(edges).to(DEV)].cpu().numpy(), r2, T2,
                       what=f"{name} sddmm K={K}")
         del O, E, Xd
+
+
+# ------------------------------------------------------------ bf16 (f2) ----
+def _bf16_pair(seed, rows, K):
+    """bf16 features (round-to-nearest-even of the fp32 generator) and their exact fp32
+    values (bf16 -> fp32 widening is exact)."""
+    X = torch.from_numpy(_x(seed, rows, K))
+    Xb = X.to(torch.bfloat16)
+    return Xb.to(DEV), Xb.float().numpy(), X.numpy()
+
+
+@pytest.mark.parametrize("K", [2, 6, 24, 32, 64, 128, 256, 512])
+def test_bf16_features_parity(K):
+    """bf16 gathered features, fp32 accumulation: exact-input parity within 1e-5 * T
+    (the oracle is fed the bf16 values), and within 1e-2 * T of the fp32-feature result
+    (BASELINE.json bf16 bar)."""
+    g = gen.powerlaw_graph(4000, 120000, gamma=2.2, n_comm=6, seed=500 + K)
+    dg = upload(g)
+    p = gs.plan(dg, K, feature_dtype="bf16")
+    info = p.info()
+    ref = oracle.plan(g.row_ind, K, info["num_sms"], info["active_blocks_per_sm"],
+                      feature_dtype=1)
+    assert info == ref.info
+    Xb, Xexact, X32 = _bf16_pair(600 + K, g.N, K)
+    A1b, A1exact, A132 = _bf16_pair(700 + K, g.M, K)
+    O = gs.spmm(p, dg, Xb).cpu().numpy()
+    E = gs.sddmm(p, dg, A1b, Xb).cpu().numpy()
+    r, T = oracle.spmm(g.row_ind, g.col_ind, g.val, Xexact, M=g.M)
+    assert_within(O, r, T, what=f"bf16 spmm K={K} (exact inputs)")
+    r32, T32 = oracle.spmm(g.row_ind, g.col_ind, g.val, X32, M=g.M)
+    assert_within(O, r32, T32, tol=1e-2, what=f"bf16 spmm K={K} vs fp32")
+    r2, T2 = oracle.sddmm(g.row_ind, g.col_ind, g.val, A1exact, Xexact)
+    assert_within(E, r2, T2, what=f"bf16 sddmm K={K} (exact inputs)")
+    r232, T232 = oracle.sddmm(g.row_ind, g.col_ind, g.val, A132, X32)
+    assert_within(E, r232, T232, tol=1e-2, what=f"bf16 sddmm K={K} vs fp32")
+
+
+def test_bf16_plan_dtype_mismatch_rejected():
+    g = gen.powerlaw_graph(500, 5000, seed=510)
+    dg = upload(g)
+    p = gs.plan(dg, 32)  # fp32 plan
+    with pytest.raises(gs.GnnError):
+        gs.spmm(p, dg, torch.zeros((g.N, 32), dtype=torch.bfloat16, device=DEV))

@@ -363,3 +363,26 @@ def test_csr_to_coo_matches_repeat():
     g = gen.powerlaw_graph(300, 3000, seed=41)
     assert np.array_equal(oracle.csr_to_coo(g.row_ptr), g.row_ind)
     assert np.array_equal(np.repeat(np.arange(g.M), np.diff(g.row_ptr)), g.row_ind)
+
+
+BF16_TABLE = {  # K: (vw_feat, lanes, vecs, slices, groups) with bf16 features
+    32: (16, 2, 1, 1, 16), 64: (16, 4, 1, 1, 8), 128: (16, 8, 1, 1, 4), 256: (16, 8, 2, 1, 4),
+    24: (8, 4, 1, 1, 8), 6: (2, 4, 1, 1, 8), 512: (16, 16, 2, 1, 2), 1000: (8, 32, 2, 2, 1),
+}
+
+
+@pytest.mark.parametrize("K", sorted(BF16_TABLE))
+def test_plan_bf16_vector_width_table(K):
+    p = oracle.plan(np.zeros(100, np.int32), K, 148, 8, feature_dtype=1)
+    assert (p.info["vw_feat"], p.info["lanes"], p.info["vecs"], p.info["slices"],
+            p.info["groups"]) == BF16_TABLE[K]
+    assert p.info["feature_dtype"] == 1
+
+
+def test_plan_bf16_rejects_odd_K_and_bad_force_vw():
+    with pytest.raises(ValueError):
+        oracle.plan(np.zeros(10, np.int32), 33, 148, 8, feature_dtype=1)
+    with pytest.raises(ValueError):
+        oracle.plan(np.zeros(10, np.int32), 32, 148, 8, feature_dtype=1, force_vw=1)
+    with pytest.raises(ValueError):
+        oracle.plan(np.zeros(10, np.int32), 32, 148, 8, feature_dtype=0, force_vw=16)

@@ -20,7 +20,7 @@ import numpy as np, torch
 import gen, oracle
 import paper_conf_ipps_fanwc23_b200 as gs
 from gen import configs
-res = {"lib": os.environ["GNN_LIB_PATH"]}
+res = {"lib": os.environ["GNN_LIB_PATH"], "dtype": DTYPE}
 # parity on a small graph
 g = gen.powerlaw_graph(4000, 200000, gamma=2.2, n_comm=5, seed=3)
 dg = gs.DeviceGraph.from_arrays(g.M, g.N, g.row_ind, g.col_ind, g.val, g.row_ptr)
@@ -48,8 +48,10 @@ for K, fvw in [(k, 0) for k in KS] + [(k, 8) for k in KS if VW8 and k % 8 == 0 a
     X = torch.from_numpy(configs.make_features(WL, g.N, K)).cuda()
     if perm is not None:
         X = gs.permute_rows(X, torch.from_numpy(perm))
+    if DTYPE == "bf16":
+        X = X.to(torch.bfloat16)
     O = torch.empty((g.M, K), device="cuda"); E = torch.empty(g.nnz, device="cuda")
-    p = gs.plan(dg, K, force_vw=fvw)
+    p = gs.plan(dg, K, force_vw=fvw, feature_dtype=DTYPE)
     ts, td = [], []
     for it in range(REPS + 2):
         flush.fill_(it)
@@ -71,10 +73,11 @@ def main():
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--vw8", action="store_true")
     ap.add_argument("--reorder", action="store_true")
+    ap.add_argument("--dtype", default="f32", choices=["f32", "bf16"])
     ap.add_argument("libs", nargs="+")
     a = ap.parse_args()
     code = CHILD.replace("ROOT", repr(ROOT)).replace("WL", repr(a.workload)).replace(
-        "KS", repr([int(k) for k in a.K.split(",")])).replace("REPS", str(a.reps)).replace("VW8", str(a.vw8)).replace("REORDER", str(a.reorder))
+        "KS", repr([int(k) for k in a.K.split(",")])).replace("REPS", str(a.reps)).replace("VW8", str(a.vw8)).replace("REORDER", str(a.reorder)).replace("DTYPE", repr(a.dtype))
     for lib in a.libs:
         env = dict(os.environ, GNN_LIB_PATH=os.path.abspath(lib))
         r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
