@@ -14,9 +14,9 @@ namespace gnn {
 #define GNN_SPMM_MINB 1  // min resident 512-thread blocks/SM the register budget must allow
 #endif
 
-// Feature vectors in flight per lane.  Measured on C4 (profiles/r01_sweep4.txt,
-// r01_sweep11.txt): 4 while several chunks share a warp (L <= 8, R = 1), 8 for wider
-// groups and whenever a lane holds R = 2 vectors per row.
+// Feature vectors in flight per lane (U * R).  Measured on the GCR-reordered C4
+// (profiles/r01_sweep12.txt, r01_sweep19.txt): 8, except 4 when a lane holds two
+// vectors per row (R = 2) or a row is only 2 lanes wide.
 #ifndef GNN_SPMM_DEPTH_R2
 #define GNN_SPMM_DEPTH_R2 4
 #endif
@@ -26,7 +26,7 @@ struct FeatDepth {
 #if defined(GNN_SPMM_DEPTH8)
   static constexpr int value = wide ? GNN_SPMM_DEPTH8 : 8;
 #else
-  static constexpr int value = R == 2 ? GNN_SPMM_DEPTH_R2 : (wide ? (L >= 16 ? 8 : 4) : 8);
+  static constexpr int value = R == 2 ? GNN_SPMM_DEPTH_R2 : ((wide && L <= 2) ? 4 : 8);
 #endif
 };
 
