@@ -48,15 +48,15 @@ WORKLOAD_DESC = {
 
 
 # ------------------------------------------------------------- byte model ---
-def spmm_bytes(nnz, M, K):
-    """Per nnz: 12 B sparse (row, col, val) + 4K B gathered feature row; per output
-    row 4K B written."""
-    return nnz * (12 + 4 * K) + 4 * K * M
+def spmm_bytes(nnz, M, K, eb=4):
+    """Per nnz: 12 B sparse (row, col, val) + eb*K B gathered feature row; per output
+    row 4K B written (eb = 4 fp32, 2 bf16 features)."""
+    return nnz * (12 + eb * K) + 4 * K * M
 
 
-def sddmm_bytes(nnz, M, K):
-    """Per nnz: 12 B sparse + 4 B out + 4K B gathered A2T row; per row 4K B of A1."""
-    return nnz * (16 + 4 * K) + 4 * K * M
+def sddmm_bytes(nnz, M, K, eb=4):
+    """Per nnz: 12 B sparse + 4 B out + eb*K B gathered A2T row; per row eb*K B of A1."""
+    return nnz * (16 + eb * K) + eb * K * M
 
 
 def plan_bytes(nch):
@@ -208,7 +208,7 @@ def parse_ks(s, name):
 
 
 # ------------------------------------------------------------ our impl ------
-def time_path(args, g, perm, name, Ks, dev, world, rank):
+def time_path(args, g, perm, name, Ks, dev, world, rank, dtype="f32"):
     """Resident graph + features for this rank's shard; W warm-up steps, then K timed
     steps (CUDA events per kernel on the launching stream, L2 flushed between steps
     outside the events).  Returns per-kernel times, this rank's bytes/flops, launches."""
@@ -237,6 +237,10 @@ def time_path(args, g, perm, name, Ks, dev, world, rank):
             if K in Xown:
                 raise SystemExit("--reorder with --xmode allgather is not supported")
             X[K] = gs.permute_rows(X[K], perm_d)
+        if dtype == "bf16":  # bf16 feature storage, fp32 accumulate
+            X[K] = X[K].to(torch.bfloat16)
+            if K in Xown:
+                Xown[K] = Xown[K].to(torch.bfloat16)
     O = {K: torch.empty((spg.M, K), dtype=torch.float32, device=dev) for K in Ks}
     E = torch.empty(sdg.nnz, dtype=torch.float32, device=dev)
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
@@ -251,7 +255,7 @@ def time_path(args, g, perm, name, Ks, dev, world, rank):
                 gdist.gather_features(Xown[K], spec, g.N, out=X[K])
             if ev is not None:
                 ev[K][0].record(stream)
-            pl = gs.plan(spg, K)
+            pl = gs.plan(spg, K, feature_dtype=dtype)
             n += 1
             if ev is not None:
                 ev[K][1].record(stream)
@@ -259,7 +263,7 @@ def time_path(args, g, perm, name, Ks, dev, world, rank):
             n += 2 if spg.nnz else 0
             if ev is not None:
                 ev[K][2].record(stream)
-            pl2 = pl if same else gs.plan(sdg, K)
+            pl2 = pl if same else gs.plan(sdg, K, feature_dtype=dtype)
             n += 0 if same else 1
             gs.sddmm(pl2, sdg, X[K], X[K], out=E)
             n += 1 if sdg.nnz else 0
@@ -298,10 +302,11 @@ def time_path(args, g, perm, name, Ks, dev, world, rank):
             tot += a + b + c
         step_ms.append(tot)
     my_bytes, my_flops, detail = 0, 0, {}
+    eb = 2 if dtype == "bf16" else 4
     for K in Ks:
-        info = gs.plan(spg, K).info()
-        b_sp = spmm_bytes(spg.nnz, spg.M, K)
-        b_sd = sddmm_bytes(sdg.nnz, g.M if not same else spg.M, K)
+        info = gs.plan(spg, K, feature_dtype=dtype).info()
+        b_sp = spmm_bytes(spg.nnz, spg.M, K, eb)
+        b_sd = sddmm_bytes(sdg.nnz, g.M if not same else spg.M, K, eb)
         my_bytes += b_sp + b_sd + plan_bytes(info["num_chunks"])
         my_flops += spmm_flops(spg.nnz, K) + sddmm_flops(sdg.nnz, K)
         t_sp, t_sd = statistics.mean(per[K]["spmm"]), statistics.mean(per[K]["sddmm"])
@@ -410,6 +415,19 @@ def run_ours(args):
         roofline["gather_ceiling_measured"] = ceil
         roofline["frac_of_l2_gather"] = round(achieved / ceil["l2_GBps"], 4)
     launches, clocks, detail = r["launches"], r["clocks"], r["detail"]
+    bf16 = None
+    if args.bf16 and world == 1:
+        del r
+        torch.cuda.empty_cache()
+        rb = time_path(args, g, perm, name, Ks, dev, world, rank, dtype="bf16")
+        msb, bb, fb = aggregate(rb, args, world, dev)
+        bf16 = {"value": round(bb / (msb * 1e-3) / 1e9, 2), "unit": "GB/s",
+                "ms_per_step": round(msb / args.steps, 4),
+                "note": "bf16 feature storage, fp32 accumulation/outputs (SURVEY §8(f) f2); "
+                        "bytes counted at 2 B per gathered element",
+                "kernels": rb["detail"]}
+        del rb
+        r = None
     alt = None
     if reorder and args.compare:
         del r
@@ -444,7 +462,7 @@ def run_ours(args):
             "gflops": round(tot_flops / (tot_ms * 1e-3) / 1e9, 1),
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": launches * args.steps, "clocks": clocks, "kernels": detail,
-            "no_reorder": alt,
+            "no_reorder": alt, "bf16": bf16,
         }
         print(json.dumps(line), flush=True)
     if world > 1:
@@ -696,6 +714,8 @@ def main():
     ap.add_argument("--no-reorder", dest="reorder", action="store_false",
                     help="time the graph as generated (default: GCR-reordered offline first, "
                          "the paper's full-graph setup)")
+    ap.add_argument("--no-bf16", dest="bf16", action="store_false",
+                    help="skip the extra timing with bf16 feature storage")
     ap.add_argument("--no-compare", dest="compare", action="store_false",
                     help="skip the extra timing of the un-reordered graph")
     args = ap.parse_args()

@@ -50,7 +50,7 @@ def main():
     for rep in reps:
         for d in rows_of(rep):
             name = d['Kernel Name'][0]
-            m = re.search(r'(spmm|sddmm)_kernel<(\d+), (\d+), (\d+)', name)
+            m = re.search(r'(spmm|sddmm)_kernel<', name)
             rec = {k: f"{v} {un}".strip() for k, (v, un) in d.items()}
             if m:
                 kind = m.group(1)
