@@ -147,6 +147,19 @@ GNN_API gnn_status_t gnn_spmm_bf16(gnn_plan_t plan, const gnn_graph_t *graph,
                                    const uint16_t *A, int64_t lda, float *O, int64_t ldo,
                                    gnn_stream_t stream);
 
+/* Aggregators of the MPP node-wise op (Eq. 1: "max, min, sum"), f_n = v * X_u. */
+typedef enum { GNN_AGG_SUM = 0, GNN_AGG_MEAN = 1, GNN_AGG_MAX = 2, GNN_AGG_MIN = 3 } gnn_agg_t;
+
+/* Generalised SpMM: O[r] = (+)_{i : row_ind[i] = r} val[i] * A[col_ind[i]]
+ * with (+) = sum, mean (sum / number of nonzeros of the row; needs graph->row_ptr), max or
+ * min (elementwise over the row's terms); rows without nonzeros give 0.  A's element type
+ * is the plan's feature_dtype (max / min: fp32 only).  accumulate = 1 (sum only) computes
+ * O += S A and leaves rows without nonzeros untouched (beta = 1, used to sum partial
+ * products, e.g. per column block).  Other rules as gnn_spmm. */
+GNN_API gnn_status_t gnn_spmm_ex(gnn_plan_t plan, const gnn_graph_t *graph, const void *A,
+                                 int64_t lda, float *O, int64_t ldo, int32_t agg,
+                                 int32_t accumulate, gnn_stream_t stream);
+
 /* SDDMM, S_O = (A1 A2) (.) S (Algorithm 2), hybrid-parallel
  * (Algorithm 4): out[i] = val[i] * sum_k A1[row_ind[i] - row_base][k] *
  * A2T[col_ind[i]][k] for i in [0, nnz).  A1: M x K (destination rows, lda1 >= K);
@@ -172,6 +185,18 @@ GNN_API gnn_status_t gnn_shard_rows(const int32_t *row_ptr_host, int64_t M, int3
                                     int64_t *bounds);
 /* Equal edge-range shards: bounds[p] = floor(p * nnz / P), [P+1] host array. */
 GNN_API gnn_status_t gnn_shard_edges(int64_t nnz, int32_t P, int64_t *bounds);
+
+/* ----------------------------------------------------------- transpose ---- */
+/* S^T (N x M) in hybrid CSR/COO on the device, for the backward pass dX = S^T dO
+ * (SURVEY §8(f) f3).  Outputs (caller-allocated, device): row_ptr_t[N+1], row_ind_t[nnz]
+ * (= columns of S), col_ind_t[nnz] (= rows of S minus row_base), val_t[nnz] (may be NULL;
+ * ones when graph->val is NULL), edge_perm[nnz] (may be NULL: original edge id of each
+ * transposed entry).  Rows of S^T ascending, then S's rows ascending (stable: duplicates
+ * keep their order).  workspace: gnn_transpose_workspace_bytes(nnz) bytes, 256-B aligned. */
+GNN_API size_t gnn_transpose_workspace_bytes(int64_t nnz);
+GNN_API gnn_status_t gnn_transpose(const gnn_graph_t *graph, void *workspace, size_t ws_bytes,
+                                   int32_t *row_ptr_t, int32_t *row_ind_t, int32_t *col_ind_t,
+                                   float *val_t, int32_t *edge_perm, gnn_stream_t stream);
 
 /* ------------------------------------------------------------- reorder ---- */
 /* Graph Clustering based Reordering (GCR, Fig. 8) -- optional, HOST side,

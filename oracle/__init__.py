@@ -43,6 +43,7 @@ def _load():
     vp, i64, i32 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32
     lib.oracle_spmm.argtypes = [i64, i64, vp, vp, vp, i64, vp, i64, i64, i64, vp, vp]
     lib.oracle_sddmm.argtypes = [i64, i64, vp, vp, vp, i64, vp, i64, vp, i64, vp, vp]
+    lib.oracle_spmm_agg.argtypes = [i64, i64, vp, vp, vp, i64, vp, i64, i64, i64, i32, vp, vp]
     lib.oracle_plan.argtypes = [i64, vp, i32, i32, i32, i32, i32, i32, i32, i32,
                                 ctypes.POINTER(_PlanInfo), vp, vp, vp]
     lib.oracle_shard_rows.argtypes = [vp, i64, i32, vp]
@@ -50,7 +51,7 @@ def _load():
     lib.oracle_csr_to_coo.argtypes = [vp, i64, vp]
     lib.oracle_modularity.argtypes = [vp, vp, i64, vp, i32]
     lib.oracle_modularity.restype = ctypes.c_double
-    for f in ("oracle_spmm", "oracle_sddmm", "oracle_plan", "oracle_shard_rows",
+    for f in ("oracle_spmm", "oracle_spmm_agg", "oracle_sddmm", "oracle_plan", "oracle_shard_rows",
               "oracle_shard_edges", "oracle_csr_to_coo"):
         getattr(lib, f).restype = ctypes.c_int
     _lib = lib
@@ -89,6 +90,28 @@ def spmm(row_ind, col_ind, val, A, M=None, i0=0, i1=None, r0=0, nrows=None):
                          A.strides[0] // 4, r0, nrows, _ptr(O), _ptr(T))
     if rc != 0:
         raise ValueError("oracle_spmm: invalid arguments")
+    return O, T
+
+
+AGG = {"sum": 0, "mean": 1, "max": 2, "min": 3}
+
+
+def spmm_agg(row_ind, col_ind, val, A, agg, M=None, i0=0, i1=None, r0=0, nrows=None):
+    """Eq. 1 node-wise op with (+) = agg in {sum, mean, max, min}: returns (O, T)."""
+    lib = _load()
+    row_ind, col_ind = _i32(row_ind), _i32(col_ind)
+    val = None if val is None else np.ascontiguousarray(val, np.float32)
+    A = _f32_2d(A)
+    i1 = row_ind.shape[0] if i1 is None else i1
+    if nrows is None:
+        nrows = (M if M is not None else (int(row_ind.max()) + 1 if row_ind.size else 0)) - r0
+    K = A.shape[1]
+    O = np.empty((nrows, K), np.float64)
+    T = np.empty((nrows, K), np.float64)
+    rc = lib.oracle_spmm_agg(i0, i1, _ptr(row_ind), _ptr(col_ind), _ptr(val), K, _ptr(A),
+                             A.strides[0] // 4, r0, nrows, AGG[agg], _ptr(O), _ptr(T))
+    if rc != 0:
+        raise ValueError("oracle_spmm_agg: invalid arguments")
     return O, T
 
 

@@ -7,6 +7,7 @@
 
 #include <math.h>
 #include <stddef.h>
+#include <stdlib.h>
 #include <string.h>
 
 /* ------------------------------------------------------------ SpMM ------ */
@@ -29,6 +30,49 @@ int oracle_spmm(int64_t i0, int64_t i1, const int32_t *row_ind, const int32_t *c
       if (T) T[(r - r0) * K + k] += fabs(term);
     }
   }
+  return 0;
+}
+
+/* ------------------------------------------------ aggregated SpMM ------ */
+/* Eq. 1 with f_n = v * X_u and (+) = sum / mean / max / min. */
+int oracle_spmm_agg(int64_t i0, int64_t i1, const int32_t *row_ind, const int32_t *col_ind,
+                    const float *val, int64_t K, const float *A, int64_t lda, int64_t r0,
+                    int64_t nrows, int32_t agg, double *O, double *T) {
+  if (agg < 0 || agg > 3) return -1;
+  if (agg <= 1) {
+    int rc = oracle_spmm(i0, i1, row_ind, col_ind, val, K, A, lda, r0, nrows, O, T);
+    if (rc != 0 || agg == 0) return rc;
+    /* mean: divide each row by its number of terms */
+    for (int64_t r = 0; r < nrows; ++r) {
+      int64_t cnt = 0;
+      for (int64_t i = i0; i < i1; ++i) cnt += (row_ind[i] == r0 + r);
+      if (cnt == 0) continue;
+      for (int64_t k = 0; k < K; ++k) {
+        O[r * K + k] /= (double)cnt;
+        if (T) T[r * K + k] /= (double)cnt;
+      }
+    }
+    return 0;
+  }
+  if (i0 < 0 || i1 < i0 || K < 1 || lda < K || nrows < 0) return -1;
+  char *seen = (char *)calloc((size_t)nrows + 1, 1);
+  memset(O, 0, sizeof(double) * (size_t)(nrows * K));
+  if (T) memset(T, 0, sizeof(double) * (size_t)(nrows * K));
+  for (int64_t i = i0; i < i1; ++i) {
+    int64_t r = row_ind[i], c = col_ind[i];
+    double v = val ? (double)val[i] : 1.0;
+    if (r < r0 || r >= r0 + nrows || c < 0) { free(seen); return -1; }
+    double *o = O + (r - r0) * K;
+    const float *a = A + c * lda;
+    for (int64_t k = 0; k < K; ++k) {
+      double term = v * (double)a[k];
+      if (!seen[r - r0]) o[k] = term;
+      else if (agg == 2 ? term > o[k] : term < o[k]) o[k] = term;
+      if (T && fabs(term) > T[(r - r0) * K + k]) T[(r - r0) * K + k] = fabs(term);
+    }
+    seen[r - r0] = 1;
+  }
+  free(seen);
   return 0;
 }
 

@@ -66,6 +66,7 @@ class ReorderOpts(ctypes.Structure):
 
 EXPORTS = ["gnn_plan_workspace_bytes", "gnn_plan_create", "gnn_plan_info", "gnn_plan_arrays",
            "gnn_plan_destroy", "gnn_spmm", "gnn_sddmm", "gnn_spmm_bf16", "gnn_sddmm_bf16",
+           "gnn_spmm_ex", "gnn_transpose_workspace_bytes", "gnn_transpose",
            "gnn_shard_rows", "gnn_shard_edges",
            "gnn_reorder_gcr", "gnn_permute_graph", "gnn_permute_rows",
            "gnn_probe_gather", "gnn_csr_to_coo", "gnn_validate", "gnn_last_error",
@@ -96,6 +97,11 @@ def lib():
     if hasattr(L, "gnn_spmm_bf16"):  # (GNN_LIB_PATH may point at an older tuning build)
         L.gnn_spmm_bf16.argtypes = [vp, P(_Graph), vp, i64, vp, i64, vp]
         L.gnn_sddmm_bf16.argtypes = [vp, P(_Graph), vp, i64, vp, i64, vp, vp]
+    if hasattr(L, "gnn_spmm_ex"):
+        L.gnn_spmm_ex.argtypes = [vp, P(_Graph), vp, i64, vp, i64, i32, i32, vp]
+        L.gnn_transpose_workspace_bytes.argtypes = [i64]
+        L.gnn_transpose_workspace_bytes.restype = ctypes.c_size_t
+        L.gnn_transpose.argtypes = [P(_Graph), vp, ctypes.c_size_t, vp, vp, vp, vp, vp, vp]
     L.gnn_shard_rows.argtypes = [vp, i64, i32, vp]
     L.gnn_shard_edges.argtypes = [i64, i32, vp]
     L.gnn_csr_to_coo.argtypes = [vp, i64, i64, vp, vp]
@@ -111,7 +117,7 @@ def lib():
     for f in ("gnn_plan_create", "gnn_plan_info", "gnn_plan_arrays", "gnn_spmm", "gnn_sddmm",
               "gnn_shard_rows", "gnn_shard_edges", "gnn_csr_to_coo", "gnn_validate",
               "gnn_reorder_gcr", "gnn_permute_graph", "gnn_permute_rows", "gnn_probe_gather",
-              "gnn_spmm_bf16", "gnn_sddmm_bf16"):
+              "gnn_spmm_bf16", "gnn_sddmm_bf16", "gnn_spmm_ex", "gnn_transpose"):
         if hasattr(L, f):
             getattr(L, f).restype = st
     _lib = L
@@ -259,19 +265,49 @@ def _dense(t, name, dtypes=(torch.float32,)):
 _FEAT = (torch.float32, torch.bfloat16)
 
 
+AGG = {"sum": 0, "mean": 1, "max": 2, "min": 3}
+
+
 def spmm(p: Plan, graph: DeviceGraph, A: torch.Tensor, out: torch.Tensor | None = None,
-         stream=None) -> torch.Tensor:
-    """gnn_spmm: O = S A (overwrites out; returns it)."""
+         agg: str = "sum", accumulate: bool = False, stream=None) -> torch.Tensor:
+    """gnn_spmm: O = S A (overwrites out; returns it).  agg / accumulate select
+    gnn_spmm_ex: (+) in {sum, mean, max, min}; accumulate=True computes O += S A."""
     K = p.K
     _dense(A, "A", _FEAT)
     if out is None:
+        if accumulate:
+            raise ValueError("accumulate=True needs an existing out")
         out = torch.empty((graph.M, K), dtype=torch.float32, device=A.device)
     _dense(out, "out")
     g = graph.desc()
+    if agg != "sum" or accumulate:
+        _check(lib().gnn_spmm_ex(p.handle, ctypes.byref(g), _ptr(A), A.stride(0), _ptr(out),
+                                 out.stride(0), AGG[agg], int(accumulate), _stream(stream)))
+        return out
     fn = lib().gnn_spmm_bf16 if A.dtype == torch.bfloat16 else lib().gnn_spmm
     _check(fn(p.handle, ctypes.byref(g), _ptr(A), A.stride(0), _ptr(out), out.stride(0),
               _stream(stream)))
     return out
+
+
+def transpose(graph: DeviceGraph, stream=None):
+    """gnn_transpose: (S^T as a DeviceGraph with row_ptr, edge_perm) on the device.
+    edge_perm[j] is the edge id (index into graph's arrays) of transposed entry j."""
+    L = lib()
+    dev = graph.row_ind.device
+    nnz = graph.nnz
+    nbytes = L.gnn_transpose_workspace_bytes(nnz)
+    ws = torch.empty(max(int(nbytes), 1), dtype=torch.uint8, device=dev)
+    rp = torch.empty(graph.N + 1, dtype=torch.int32, device=dev)
+    ri = torch.empty(nnz, dtype=torch.int32, device=dev)
+    ci = torch.empty(nnz, dtype=torch.int32, device=dev)
+    vt = torch.empty(nnz, dtype=torch.float32, device=dev)
+    perm = torch.empty(nnz, dtype=torch.int32, device=dev)
+    g = graph.desc()
+    _check(L.gnn_transpose(ctypes.byref(g), _ptr(ws), int(nbytes), _ptr(rp), _ptr(ri), _ptr(ci),
+                           _ptr(vt), _ptr(perm), _stream(stream)))
+    gt = DeviceGraph(graph.N, graph.M, ri, ci, vt if graph.val is not None else None, rp, 0)
+    return gt, perm
 
 
 def sddmm(p: Plan, graph: DeviceGraph, A1: torch.Tensor, A2T: torch.Tensor,

@@ -48,6 +48,7 @@ struct SparseArgs {
   int32_t K;
   int32_t slices;
   int32_t vecs;
+  int32_t accum;  // 1: O += S A (beta = 1), rows without nonzeros untouched
 };
 
 // Occupancy (active blocks / SM) of the SpMM kernel for a feature width/lane count;

@@ -20,16 +20,19 @@
 #include <atomic>
 #include <climits>
 
+#include <math.h>
+
 #include "spmm_kernel.cuh"
 
 namespace gnn {
 
-// Zero every row shared by several chunks before the atomics land on it: the row
-// is zeroed by the chunk in which it starts (tail flag set, and not a pure
-// continuation of an earlier chunk's row).  One warp per chunk.
+// Initialise every row shared by several chunks before the atomics land on it (0 for
+// sum, -inf / +inf for max / min): the row is initialised by the chunk in which it starts
+// (tail flag set, and not a pure continuation of an earlier chunk's row).  One warp per
+// chunk.
 template <int VW>
 __global__ void spmm_prezero_kernel(const SparseArgs a, float *__restrict__ O,
-                                    const int64_t ldo) {
+                                    const int64_t ldo, const float init) {
   const int64_t c = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int lane = threadIdx.x & 31;
   if (c >= a.num_chunks) return;
@@ -38,11 +41,33 @@ __global__ void spmm_prezero_kernel(const SparseArgs a, float *__restrict__ O,
   const int32_t rf = a.row_first[c], rl = a.row_last[c];
   if ((fl & 1u) && rf == rl) return;
   float *o = O + ((int64_t)rl - a.row_base) * ldo;
-  for (int k = lane * VW; k < a.K; k += 32 * VW) st_zero<VW>(o + k);
+  float z[VW];
+#pragma unroll
+  for (int v = 0; v < VW; ++v) z[v] = init;
+  for (int k = lane * VW; k < a.K; k += 32 * VW) st_vec<VW>(o + k, z);
 }
 
-SpmmFn pick_spmm(int dtype, int vw, int L, int R, int vws) {
-  return dtype == GNN_BF16 ? pick_spmm_bf16(vw, L, R, vws) : pick_spmm_f32(vw, L, R, vws);
+// Mean aggregator: O[r] *= 1 / (nonzeros of row r) for rows with nonzeros (row_ptr read
+// relative to row_ptr[0]).  One warp per row.
+__global__ void spmm_row_mean_kernel(const int32_t *__restrict__ row_ptr, int64_t M, int32_t K,
+                                     float *__restrict__ O, int64_t ldo) {
+  const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t r = warp; r < M; r += nwarps) {
+    const int32_t cnt = row_ptr[r + 1] - row_ptr[r];
+    if (cnt <= 0) continue;
+    const float s = 1.0f / (float)cnt;
+    float *o = O + r * ldo;
+    for (int k = lane; k < K; k += 32) o[k] *= s;
+  }
+}
+
+SpmmFn pick_spmm(int dtype, int vw, int L, int R, int vws, int agg = kAggSum) {
+  if (dtype == GNN_BF16) return agg == kAggSum ? pick_spmm_bf16(vw, L, R, vws) : nullptr;
+  if (agg == kAggMax) return pick_spmm_f32_max(vw, L, R, vws);
+  if (agg == kAggMin) return pick_spmm_f32_min(vw, L, R, vws);
+  return pick_spmm_f32(vw, L, R, vws);
 }
 
 // Cached per (device, dtype, vw, lanes, vecs, wpb): the occupancy API is a host-side
@@ -121,6 +146,7 @@ SparseArgs make_args(const Plan *p, const gnn_graph_t *g) {
   a.K = p->info.K;
   a.slices = p->info.slices;
   a.vecs = p->info.vecs;
+  a.accum = 0;
   return a;
 }
 
@@ -131,12 +157,20 @@ using namespace gnn;
 namespace gnn {
 static gnn_status_t launch_spmm(const Plan *p, const gnn_graph_t *g, const void *A, int64_t lda,
                                 float *O, int64_t ldo, gnn_stream_t stream, int dtype,
-                                const char *who) {
+                                int agg_api, int accumulate, const char *who) {
   if (gnn_status_t st = check_common(p, g, who)) return st;
   const gnn_plan_info_t &in = p->info;
   if (in.feature_dtype != dtype)
     return fail(GNN_ERR_INVALID_ARG, "%s: plan was built for feature_dtype %d", who,
                 in.feature_dtype);
+  if (agg_api < GNN_AGG_SUM || agg_api > GNN_AGG_MIN || (accumulate != 0 && accumulate != 1))
+    return fail(GNN_ERR_INVALID_ARG, "%s: bad aggregator %d / accumulate %d", who, agg_api,
+                accumulate);
+  if (accumulate && agg_api != GNN_AGG_SUM)
+    return fail(GNN_ERR_UNSUPPORTED, "%s: accumulate (beta = 1) is defined for sum only", who);
+  if (agg_api == GNN_AGG_MEAN && g->M > 0 && !g->row_ptr)
+    return fail(GNN_ERR_INVALID_ARG, "%s: the mean aggregator needs graph->row_ptr", who);
+  const int agg = agg_api == GNN_AGG_MAX ? kAggMax : agg_api == GNN_AGG_MIN ? kAggMin : kAggSum;
   const int K = in.K, VW = in.vw_feat;
   const int ES = dtype == GNN_BF16 ? 2 : 4;
   const int VO = VW < 8 ? VW : 8;  // fp32 output vector granule
@@ -151,22 +185,27 @@ static gnn_status_t launch_spmm(const Plan *p, const gnn_graph_t *g, const void 
                 "with a pitch multiple of %d (re-plan with force_vw)",
                 who, ES * VW, VW, 4 * VO, VO);
   cudaStream_t s = (cudaStream_t)stream;
-  if (g->nnz == 0) {  // no chunks: O := 0
+  if (g->nnz == 0) {  // no chunks: O := 0 (beta = 1: unchanged)
+    if (accumulate) return GNN_OK;
     cudaError_t e = cudaMemset2DAsync(O, ldo * sizeof(float), 0, K * sizeof(float), g->M, s);
     return e == cudaSuccess ? GNN_OK : cuda_fail(e, "gnn_spmm memset");
   }
   const int vws = effective_vws(in.vw_sparse, g, nullptr);
-  SpmmFn f = pick_spmm(dtype, VW, in.lanes, in.vecs, vws);
-  if (!f) return fail(GNN_ERR_UNSUPPORTED, "%s: no kernel for vw=%d L=%d", who, VW, in.lanes);
-  const SparseArgs a = make_args(p, g);
+  SpmmFn f = pick_spmm(dtype, VW, in.lanes, in.vecs, vws, agg);
+  if (!f)
+    return fail(GNN_ERR_UNSUPPORTED, "%s: no kernel for vw=%d L=%d agg=%d dtype=%d", who, VW,
+                in.lanes, agg_api, dtype);
+  SparseArgs a = make_args(p, g);
+  a.accum = accumulate;
   const int threads = in.warps_per_block * 32;
-  {
+  if (!accumulate) {
     const int64_t blocks = (a.num_chunks * 32 + 255) / 256;
+    const float init = agg == kAggMax ? -INFINITY : agg == kAggMin ? INFINITY : 0.f;
     switch (VO) {
-      case 1: spmm_prezero_kernel<1><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo); break;
-      case 2: spmm_prezero_kernel<2><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo); break;
-      case 4: spmm_prezero_kernel<4><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo); break;
-      default: spmm_prezero_kernel<8><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo); break;
+      case 1: spmm_prezero_kernel<1><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, init); break;
+      case 2: spmm_prezero_kernel<2><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, init); break;
+      case 4: spmm_prezero_kernel<4><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, init); break;
+      default: spmm_prezero_kernel<8><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, init); break;
     }
   }
   const size_t smem = (size_t)in.warps_per_block * spmm_tile_bytes_per_warp(in.lanes, vws);
@@ -175,6 +214,13 @@ static gnn_status_t launch_spmm(const Plan *p, const gnn_graph_t *g, const void 
     if (e != cudaSuccess) return cuda_fail(e, "gnn_spmm smem attribute");
   }
   f<<<(unsigned)in.num_blocks, threads, smem, s>>>(a, A, lda, O, ldo);
+  if (agg_api == GNN_AGG_MEAN) {
+    DeviceInfo d;
+    device_info(&d);
+    int64_t blocks = (g->M * 32 + 255) / 256;
+    if (blocks > (int64_t)d.num_sms * 16) blocks = (int64_t)d.num_sms * 16;
+    spmm_row_mean_kernel<<<(unsigned)blocks, 256, 0, s>>>(g->row_ptr, g->M, K, O, ldo);
+  }
   cudaError_t e = cudaGetLastError();
   return e == cudaSuccess ? GNN_OK : cuda_fail(e, "gnn_spmm launch");
 }
@@ -184,12 +230,20 @@ extern "C" GNN_API gnn_status_t gnn_spmm(gnn_plan_t plan, const gnn_graph_t *g, 
                                          int64_t lda, float *O, int64_t ldo,
                                          gnn_stream_t stream) {
   return launch_spmm(reinterpret_cast<const Plan *>(plan), g, A, lda, O, ldo, stream, GNN_F32,
-                     "gnn_spmm");
+                     GNN_AGG_SUM, 0, "gnn_spmm");
 }
 
 extern "C" GNN_API gnn_status_t gnn_spmm_bf16(gnn_plan_t plan, const gnn_graph_t *g,
                                               const uint16_t *A, int64_t lda, float *O,
                                               int64_t ldo, gnn_stream_t stream) {
   return launch_spmm(reinterpret_cast<const Plan *>(plan), g, A, lda, O, ldo, stream, GNN_BF16,
-                     "gnn_spmm_bf16");
+                     GNN_AGG_SUM, 0, "gnn_spmm_bf16");
+}
+
+extern "C" GNN_API gnn_status_t gnn_spmm_ex(gnn_plan_t plan, const gnn_graph_t *g, const void *A,
+                                            int64_t lda, float *O, int64_t ldo, int32_t agg,
+                                            int32_t accumulate, gnn_stream_t stream) {
+  const Plan *p = reinterpret_cast<const Plan *>(plan);
+  const int dtype = p ? p->info.feature_dtype : GNN_F32;
+  return launch_spmm(p, g, A, lda, O, ldo, stream, dtype, agg, accumulate, "gnn_spmm_ex");
 }

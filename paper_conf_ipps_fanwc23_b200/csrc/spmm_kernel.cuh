@@ -2,6 +2,7 @@
 // design notes) and its dispatch table; instantiated per feature type in
 // spmm_f32.cu / spmm_bf16.cu so the two halves compile in parallel.
 #pragma once
+#include <math.h>
 #include "device.cuh"
 #include "internal.cuh"
 
@@ -30,22 +31,69 @@ struct FeatDepth {
 #endif
 };
 
+// Aggregators of the node-wise MPP op (Eq. 1): ⊕ = sum (SpMM proper; mean is
+// sum followed by a row scale), max or min of the terms v_i * A[col_i].
+enum : int { kAggSum = 0, kAggMax = 1, kAggMin = 2 };
+
+template <int AGG>
+__device__ __forceinline__ float agg_init() {
+  if constexpr (AGG == kAggSum) return 0.f;
+  else if constexpr (AGG == kAggMax) return -INFINITY;
+  else return INFINITY;
+}
+
+// float atomic max / min through the ordered-integer trick (there is no red.max.f32):
+// non-negative floats order like signed ints, negative ones reversed like unsigned.
+__device__ __forceinline__ void atomic_max_f32(float *p, float v) {
+  if (v >= 0.f) atomicMax(reinterpret_cast<int *>(p), __float_as_int(v));
+  else atomicMin(reinterpret_cast<unsigned *>(p), __float_as_uint(v));
+}
+__device__ __forceinline__ void atomic_min_f32(float *p, float v) {
+  if (v >= 0.f) atomicMin(reinterpret_cast<int *>(p), __float_as_int(v));
+  else atomicMax(reinterpret_cast<unsigned *>(p), __float_as_uint(v));
+}
+
 // Flush the accumulator of row `cur` (Algo 3 line 15, "AtomicStore"): rows shared
-// with a neighbouring chunk are combined with a vector atomic add, rows owned by this
-// chunk get a plain vector store.
-template <int VW>
+// with a neighbouring chunk are combined atomically (vector add, or float max/min), rows
+// owned by this chunk get a plain vector store (or O += acc when accumulating, beta = 1).
+template <int VW, int AGG>
 __device__ __forceinline__ void flush_row(float *Ok, int64_t ldo, int64_t row_base, int32_t cur,
-                                          int32_t rf, int32_t rl, uint32_t fl,
+                                          int32_t rf, int32_t rl, uint32_t fl, bool accum,
                                           const float (&acc)[VW]) {
   float *o = Ok + ((int64_t)cur - row_base) * ldo;
   const bool shared = (cur == rf && (fl & 1u)) || (cur == rl && (fl & 2u));
-  if (shared) red_add<VW>(o, acc);
-  else st_vec<VW>(o, acc);
+  if constexpr (AGG == kAggSum) {
+    if (shared || accum) red_add<VW>(o, acc);
+    else st_vec<VW>(o, acc);
+  } else {
+    if (shared) {
+#pragma unroll
+      for (int v = 0; v < VW; ++v) {
+        if constexpr (AGG == kAggMax) atomic_max_f32(o + v, acc[v]);
+        else atomic_min_f32(o + v, acc[v]);
+      }
+    } else {
+      st_vec<VW>(o, acc);
+    }
+  }
+}
+
+template <int AGG, typename TF, int VW>
+__device__ __forceinline__ void accumulate(float (&acc)[VW], float s, const FeatVec<TF, VW> &x) {
+  if constexpr (AGG == kAggSum) {
+    axpy_f<TF, VW>(acc, s, x);
+  } else {
+#pragma unroll
+    for (int v = 0; v < VW; ++v) {
+      const float t = s * x.get(v);
+      acc[v] = AGG == kAggMax ? fmaxf(acc[v], t) : fminf(acc[v], t);
+    }
+  }
 }
 
 // L lanes per (chunk, K-slice) work item, R VW-wide vectors per lane (plan rule step 2).
 // TF: feature element type (F32 or BF16); accumulation and O are fp32.
-template <typename TF, int VW, int L, int R, int VWS>
+template <typename TF, int VW, int L, int R, int VWS, int AGG>
 __global__ void __launch_bounds__(kMaxThreads, GNN_SPMM_MINB)
     spmm_kernel(const SparseArgs a, const void *__restrict__ A, const int64_t lda,
                 float *__restrict__ O, const int64_t ldo) {
@@ -89,7 +137,8 @@ __global__ void __launch_bounds__(kMaxThreads, GNN_SPMM_MINB)
   const uint32_t ldaB = (uint32_t)lda * (uint32_t)ES;
   float *__restrict__ Ok = O + k0;  // row r at Ok + (r - row_base) * ldo
 
-  auto zero_row = [&](int64_t row) {
+  auto zero_row = [&](int64_t row) {  // rows without nonzeros: 0 (untouched if beta = 1)
+    if (a.accum) return;
 #pragma unroll
     for (int r = 0; r < R; ++r)
       if (col_ok[r]) st_zero<VW>(Ok + (row - a.row_base) * ldo + r * Lg * VW);
@@ -99,7 +148,8 @@ __global__ void __launch_bounds__(kMaxThreads, GNN_SPMM_MINB)
 #pragma unroll
     for (int r = 0; r < R; ++r)
       if (col_ok[r])
-        flush_row<VW>(Ok + r * Lg * VW, ldo, a.row_base, row, rf, rl, fl, acc[r]);
+        flush_row<VW, AGG>(Ok + r * Lg * VW, ldo, a.row_base, row, rf, rl, fl, a.accum != 0,
+                           acc[r]);
   };
 
   // empty rows between the previous chunk's last row and ours are ours to zero
@@ -111,7 +161,7 @@ __global__ void __launch_bounds__(kMaxThreads, GNN_SPMM_MINB)
 #pragma unroll
   for (int r = 0; r < R; ++r)
 #pragma unroll
-    for (int v = 0; v < VW; ++v) acc[r][v] = 0.f;
+    for (int v = 0; v < VW; ++v) acc[r][v] = agg_init<AGG>();
   int32_t cur = -1;
 
   const int32_t *__restrict__ ri = a.row_ind + cs;
@@ -149,7 +199,7 @@ __global__ void __launch_bounds__(kMaxThreads, GNN_SPMM_MINB)
 #pragma unroll
         for (int r = 0; r < R; ++r)
 #pragma unroll
-          for (int v = 0; v < VW; ++v) acc[r][v] = 0.f;
+          for (int v = 0; v < VW; ++v) acc[r][v] = agg_init<AGG>();
       }
 #pragma unroll 1
       for (int jj = 0; jj < T; jj += U) {
@@ -173,7 +223,7 @@ __global__ void __launch_bounds__(kMaxThreads, GNN_SPMM_MINB)
 #pragma unroll
         for (int u = 0; u < U; ++u)
 #pragma unroll
-          for (int r = 0; r < R; ++r) axpy_f<TF, VW>(acc[r], vj[u], x[u][r]);
+          for (int r = 0; r < R; ++r) accumulate<AGG, TF, VW>(acc[r], vj[u], x[u][r]);
       }
     } else {
       // ---- general path: per-nonzero validity and row-switch procedure
@@ -210,10 +260,10 @@ __global__ void __launch_bounds__(kMaxThreads, GNN_SPMM_MINB)
 #pragma unroll
               for (int r = 0; r < R; ++r)
 #pragma unroll
-                for (int v = 0; v < VW; ++v) acc[r][v] = 0.f;
+                for (int v = 0; v < VW; ++v) acc[r][v] = agg_init<AGG>();
             }
 #pragma unroll
-            for (int r = 0; r < R; ++r) axpy_f<TF, VW>(acc[r], vj[u], x[u][r]);
+            for (int r = 0; r < R; ++r) accumulate<AGG, TF, VW>(acc[r], vj[u], x[u][r]);
           }
         }
       }
@@ -229,32 +279,32 @@ __global__ void __launch_bounds__(kMaxThreads, GNN_SPMM_MINB)
 using SpmmFn = void (*)(const SparseArgs, const void *__restrict__, const int64_t,
                         float *__restrict__, const int64_t);
 
-template <typename TF, int VW, int L, int R>
+template <typename TF, int VW, int L, int R, int AGG>
 SpmmFn spmm_pick_vws(int vws) {
   switch (vws) {
-    case 1: return spmm_kernel<TF, VW, L, R, 1>;
-    case 2: return spmm_kernel<TF, VW, L, R, 2>;
-    case 4: return spmm_kernel<TF, VW, L, R, 4>;
+    case 1: return spmm_kernel<TF, VW, L, R, 1, AGG>;
+    case 2: return spmm_kernel<TF, VW, L, R, 2, AGG>;
+    case 4: return spmm_kernel<TF, VW, L, R, 4, AGG>;
   }
   return nullptr;
 }
-template <typename TF, int VW>
+template <typename TF, int VW, int AGG>
 SpmmFn spmm_pick_l(int L, int R, int vws) {
   if (R == 2) {  // the plan uses R = 2 only for rows of >= 16 vectors, i.e. L >= 8
     switch (L) {
-      case 8: return spmm_pick_vws<TF, VW, 8, 2>(vws);
-      case 16: return spmm_pick_vws<TF, VW, 16, 2>(vws);
-      case 32: return spmm_pick_vws<TF, VW, 32, 2>(vws);
+      case 8: return spmm_pick_vws<TF, VW, 8, 2, AGG>(vws);
+      case 16: return spmm_pick_vws<TF, VW, 16, 2, AGG>(vws);
+      case 32: return spmm_pick_vws<TF, VW, 32, 2, AGG>(vws);
     }
     return nullptr;
   }
   switch (L) {
-    case 1: return spmm_pick_vws<TF, VW, 1, 1>(vws);
-    case 2: return spmm_pick_vws<TF, VW, 2, 1>(vws);
-    case 4: return spmm_pick_vws<TF, VW, 4, 1>(vws);
-    case 8: return spmm_pick_vws<TF, VW, 8, 1>(vws);
-    case 16: return spmm_pick_vws<TF, VW, 16, 1>(vws);
-    case 32: return spmm_pick_vws<TF, VW, 32, 1>(vws);
+    case 1: return spmm_pick_vws<TF, VW, 1, 1, AGG>(vws);
+    case 2: return spmm_pick_vws<TF, VW, 2, 1, AGG>(vws);
+    case 4: return spmm_pick_vws<TF, VW, 4, 1, AGG>(vws);
+    case 8: return spmm_pick_vws<TF, VW, 8, 1, AGG>(vws);
+    case 16: return spmm_pick_vws<TF, VW, 16, 1, AGG>(vws);
+    case 32: return spmm_pick_vws<TF, VW, 32, 1, AGG>(vws);
   }
   return nullptr;
 }
@@ -265,8 +315,13 @@ inline int spmm_tile_bytes_per_warp(int L, int vws) {
   return 2 * 3 * (32 / L) * (T + 4) * 4;
 }
 
-// defined in spmm_f32.cu / spmm_bf16.cu
+template <typename TF, int AGG>
+SpmmFn spmm_pick_vw(int vw, int L, int R, int vws);
+
+// defined in spmm_f32*.cu / spmm_bf16.cu (one translation unit per aggregator)
 SpmmFn pick_spmm_f32(int vw, int L, int R, int vws);
+SpmmFn pick_spmm_f32_max(int vw, int L, int R, int vws);
+SpmmFn pick_spmm_f32_min(int vw, int L, int R, int vws);
 SpmmFn pick_spmm_bf16(int vw, int L, int R, int vws);
 
 }  // namespace gnn

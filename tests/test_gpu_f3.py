@@ -1,0 +1,109 @@
+"""GPU parity for the NEXT rows f3/f4: aggregators (Eq. 1 with
+(+) in {sum, mean, max, min}), beta = 1 accumulation, the device transpose, the autograd
+backward pair (dX = S^T dO, dv = SDDMM(dO, X)) and a GCN training smoke test."""
+import numpy as np
+import pytest
+import torch
+
+import gen
+import oracle
+import paper_conf_ipps_fanwc23_b200 as gs
+from paper_conf_ipps_fanwc23_b200 import nn as gnn
+
+from helpers import assert_within, upload
+
+pytestmark = pytest.mark.gpu
+DEV = "cuda"
+
+
+def graphs():
+    rng = np.random.default_rng(7)
+    M, N = 900, 700
+    rows = rng.integers(0, M, 30000)
+    rows = rows[(rows % 9) != 4]                       # empty rows
+    rows = np.concatenate([rows, np.full(6000, 17)])   # a hub split across many chunks
+    cols = rng.integers(0, N, rows.size)
+    vals = rng.uniform(-1, 1, rows.size).astype(np.float32)
+    yield gen.from_coo(M, N, rows, cols, vals)
+    yield gen.powerlaw_graph(5000, 150000, gamma=2.2, n_comm=5, seed=8)
+
+
+@pytest.mark.parametrize("agg", ["sum", "mean", "max", "min"])
+@pytest.mark.parametrize("K", [8, 32, 64, 256])
+@pytest.mark.parametrize("C", [0, 8, 64])
+def test_spmm_aggregators(agg, K, C):
+    for g in graphs():
+        dg = upload(g)
+        p = gs.plan(dg, K, force_chunk=C)
+        X = gen.features(31 + K, g.N, K)
+        O = gs.spmm(p, dg, torch.from_numpy(X).to(DEV), agg=agg).cpu().numpy()
+        ref, T = oracle.spmm_agg(g.row_ind, g.col_ind, g.val, X, agg, M=g.M)
+        tol = 1e-5 if agg in ("sum", "mean") else 1e-6   # max/min: one rounded product
+        assert_within(O, ref, T, tol=tol, what=f"{agg} K={K} C={C}")
+
+
+def test_spmm_accumulate_beta_one():
+    g = gen.powerlaw_graph(3000, 60000, seed=9)
+    dg = upload(g)
+    K = 64
+    p = gs.plan(dg, K)
+    X = gen.features(40, g.N, K)
+    O0 = gen.features(41, g.M, K)
+    O = torch.from_numpy(O0.copy()).to(DEV)
+    gs.spmm(p, dg, torch.from_numpy(X).to(DEV), out=O, accumulate=True)
+    ref, T = oracle.spmm(g.row_ind, g.col_ind, g.val, X, M=g.M)
+    assert_within(O.cpu().numpy(), ref + O0.astype(np.float64), T + np.abs(O0), what="beta=1")
+
+
+def test_transpose_matches_definition():
+    for g in graphs():
+        dg = upload(g)
+        gt, perm = gs.transpose(dg)
+        order = np.lexsort((np.arange(g.nnz), g.row_ind, g.col_ind))  # by col, row, stable
+        assert np.array_equal(perm.cpu().numpy(), order)
+        assert np.array_equal(gt.row_ind.cpu().numpy(), g.col_ind[order])
+        assert np.array_equal(gt.col_ind.cpu().numpy(), g.row_ind[order])
+        assert np.array_equal(gt.val.cpu().numpy(), g.val[order])
+        cnt = np.bincount(g.col_ind, minlength=g.N)
+        assert np.array_equal(gt.row_ptr.cpu().numpy(), np.r_[0, np.cumsum(cnt)])
+
+
+@pytest.mark.parametrize("agg", ["sum", "mean"])
+def test_autograd_backward_pair(agg):
+    """loss = <G, SpMM(S, X)>: dX = S^T G (mean: S^T (G / cnt)) and dv_i = <G_r, X_c>."""
+    for g in graphs():
+        dg = upload(g)
+        op = gnn.SparseOp(dg)
+        K = 32
+        X = torch.from_numpy(gen.features(50, g.N, K)).to(DEV).requires_grad_(True)
+        val = torch.from_numpy(g.val.copy()).to(DEV).requires_grad_(True)
+        G = gen.features(51, g.M, K)
+        O = gnn.spmm_autograd(op, X, val, agg=agg)
+        (O * torch.from_numpy(G).to(DEV)).sum().backward()
+        cnt = np.diff(g.row_ptr).astype(np.float64)
+        Gs = (G / np.maximum(cnt, 1)[:, None]).astype(np.float32) if agg == "mean" else G
+        order = np.lexsort((np.arange(g.nnz), g.row_ind, g.col_ind))
+        dX_ref, TdX = oracle.spmm(g.col_ind[order], g.row_ind[order], g.val[order], Gs, M=g.N)
+        assert_within(X.grad.cpu().numpy(), dX_ref, TdX, what=f"dX ({agg})")
+        dv_ref, Tdv = oracle.sddmm(g.row_ind, g.col_ind, None, Gs, X.detach().cpu().numpy())
+        assert_within(val.grad.cpu().numpy(), dv_ref, Tdv, what=f"dval ({agg})")
+
+
+def test_gcn_training_reduces_loss():
+    g = gen.powerlaw_graph(4000, 80000, gamma=2.4, n_comm=4, mu=0.1, seed=12)
+    dg = upload(g)
+    op = gnn.SparseOp(dg)
+    torch.manual_seed(0)
+    F, C = 32, 4
+    X = torch.from_numpy(gen.features(60, g.N, F)).to(DEV)
+    y = torch.from_numpy(g.comm.astype(np.int64) % C).to(DEV)   # planted communities
+    model = gnn.GCN(F, 64, C).to(DEV)
+    opt = torch.optim.Adam(model.parameters(), lr=0.01)
+    losses = []
+    for _ in range(30):
+        opt.zero_grad()
+        loss = torch.nn.functional.cross_entropy(model(op, X), y)
+        loss.backward()
+        opt.step()
+        losses.append(loss.item())
+    assert losses[-1] < 0.7 * losses[0], losses

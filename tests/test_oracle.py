@@ -386,3 +386,36 @@ def test_plan_bf16_rejects_odd_K_and_bad_force_vw():
         oracle.plan(np.zeros(10, np.int32), 32, 148, 8, feature_dtype=1, force_vw=1)
     with pytest.raises(ValueError):
         oracle.plan(np.zeros(10, np.int32), 32, 148, 8, feature_dtype=0, force_vw=16)
+
+
+# ------------------------------------------------------ aggregators (f3) ----
+@pytest.mark.parametrize("agg", ["sum", "mean", "max", "min"])
+@pytest.mark.parametrize("seed", range(3))
+def test_spmm_aggregators_match_numpy_definition(agg, seed):
+    """Eq. 1 with (+) in {sum, mean, max, min} against a per-row numpy reduction over the
+    row's term matrix (empty rows -> 0)."""
+    rng = np.random.default_rng(300 + seed)
+    M, N, K = 40, 30, 7
+    g, _ = random_coo(rng, M, N, 400)
+    A = rng.uniform(-1, 1, (N, K)).astype(np.float32)
+    O, T = oracle.spmm_agg(g.row_ind, g.col_ind, g.val, A, agg, M=M)
+    terms = g.val[:, None].astype(np.float64) * A[g.col_ind].astype(np.float64)
+    for r in range(M):
+        tr = terms[g.row_ind == r]
+        if tr.shape[0] == 0:
+            assert not O[r].any()
+            continue
+        ref = {"sum": tr.sum(0), "mean": tr.mean(0), "max": tr.max(0), "min": tr.min(0)}[agg]
+        np.testing.assert_allclose(O[r], ref, rtol=0, atol=1e-13)
+        tref = np.abs(tr).sum(0) / (tr.shape[0] if agg == "mean" else 1) if agg in ("sum", "mean") \
+            else np.abs(tr).max(0)
+        np.testing.assert_allclose(T[r], tref, rtol=1e-13, atol=0)
+
+
+def test_spmm_agg_sum_is_algorithm_1():
+    rng = np.random.default_rng(9)
+    g, _ = random_coo(rng, 30, 20, 200)
+    A = rng.uniform(-1, 1, (20, 5)).astype(np.float32)
+    a = oracle.spmm_agg(g.row_ind, g.col_ind, g.val, A, "sum", M=30)
+    b = oracle.spmm(g.row_ind, g.col_ind, g.val, A, M=30)
+    assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1])
