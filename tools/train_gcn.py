@@ -1,0 +1,113 @@
+"""Synthetic end-to-end GCN training step (the analog of the paper's
+Table V): a GCN (SpMM + fully-connected layer) trained full-graph on a
+synthetic graph with random features / labels, our SpMM/SDDMM kernels vs torch.sparse
+(cuSPARSE CSR SpMM) in the same model.  One step = forward + backward + Adam.
+
+    python tools/train_gcn.py --workload C4 --hidden 32,128,256 --steps 20
+"""
+import argparse
+import json
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import gen  # noqa: E402
+import paper_conf_ipps_fanwc23_b200 as gs  # noqa: E402
+from gen import configs  # noqa: E402
+from paper_conf_ipps_fanwc23_b200 import nn as gnn  # noqa: E402
+
+
+class TorchSparseGCN(torch.nn.Module):
+    """Same model with torch.sparse (cuSPARSE) aggregation."""
+
+    def __init__(self, fin, hidden, classes, layers):
+        super().__init__()
+        dims = [fin] + [hidden] * (layers - 1) + [classes]
+        self.lins = torch.nn.ModuleList(torch.nn.Linear(a, b, bias=False) for a, b in zip(dims, dims[1:]))
+        self.biases = torch.nn.ParameterList(torch.nn.Parameter(torch.zeros(b)) for b in dims[1:])
+
+    def forward(self, A, H):
+        for i, (lin, b) in enumerate(zip(self.lins, self.biases)):
+            H = torch.sparse.mm(A, lin(H)) + b
+            if i + 1 < len(self.lins):
+                H = torch.relu(H)
+        return H
+
+
+def time_steps(step, steps, warmup):
+    for _ in range(warmup):
+        step()
+    torch.cuda.synchronize()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record()
+    for _ in range(steps):
+        step()
+    b.record()
+    torch.cuda.synchronize()
+    return a.elapsed_time(b) / steps
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--workload", default="C4")
+    ap.add_argument("--hidden", default="32,128,256")
+    ap.add_argument("--layers", type=int, default=2)
+    ap.add_argument("--features", type=int, default=602)   # Reddit's feature width
+    ap.add_argument("--classes", type=int, default=41)     # Reddit's classes
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--reorder", action="store_true")
+    a = ap.parse_args()
+    dev = torch.device("cuda")
+    g = configs.make_graph(a.workload)
+    if a.reorder:
+        perm, _, _ = gs.reorder_gcr(g.row_ptr, g.col_ind)
+        rp, ri, ci, v = gs.permute_graph(g.row_ptr, g.col_ind, g.val, perm)
+        g = gen.Graph(g.M, g.N, rp, ri, ci, v)
+    dg = gs.DeviceGraph.from_arrays(g.M, g.N, g.row_ind, g.col_ind, g.val, g.row_ptr, device=dev)
+    op = gnn.SparseOp(dg)
+    A = torch.sparse_csr_tensor(torch.from_numpy(g.row_ptr.astype(np.int64)),
+                                torch.from_numpy(g.col_ind.astype(np.int64)),
+                                torch.from_numpy(g.val), size=(g.M, g.N)).to(dev)
+    torch.manual_seed(0)
+    X = torch.randn(g.N, a.features, device=dev)
+    y = torch.randint(0, a.classes, (g.M,), device=dev)
+    res = {"workload": a.workload, "nnz": g.nnz, "features": a.features, "classes": a.classes,
+           "layers": a.layers, "reorder": a.reorder, "runs": []}
+    for h in [int(x) for x in a.hidden.split(",")]:
+        ours = gnn.GCN(a.features, h, a.classes, a.layers).to(dev)
+        base = TorchSparseGCN(a.features, h, a.classes, a.layers).to(dev)
+        o1 = torch.optim.Adam(ours.parameters(), lr=0.01)
+        o2 = torch.optim.Adam(base.parameters(), lr=0.01)
+
+        def step_ours():
+            o1.zero_grad(set_to_none=True)
+            torch.nn.functional.cross_entropy(ours(op, X), y).backward()
+            o1.step()
+
+        def step_base():
+            o2.zero_grad(set_to_none=True)
+            torch.nn.functional.cross_entropy(base(A, X), y).backward()
+            o2.step()
+
+        t_ours = time_steps(step_ours, a.steps, a.warmup)
+        try:
+            t_base = time_steps(step_base, a.steps, a.warmup)
+        except Exception as e:  # noqa: BLE001
+            t_base = None
+            res["baseline_error"] = str(e)[:200]
+        res["runs"].append({"hidden": h, "ours_ms": round(t_ours, 3),
+                            "torch_sparse_ms": None if t_base is None else round(t_base, 3),
+                            "speedup": None if t_base is None else round(t_base / t_ours, 3)})
+        print(json.dumps(res["runs"][-1]), flush=True)
+    print(json.dumps(res), flush=True)
+
+
+if __name__ == "__main__":
+    main()
