@@ -224,9 +224,12 @@ def time_path(args, g, perm, name, Ks, dev, world, rank, dtype="f32"):
     full = gs.DeviceGraph.from_arrays(g.M, g.N, g.row_ind, g.col_ind, g.val, g.row_ptr, device=dev)
     spg, sdg = gdist.local_graphs(full, spec)
     perm_d = None if perm is None else torch.from_numpy(perm).to(dev)
-    X, Xown = {}, {}
+    X, Xown, ov = {}, {}, {}
+    overlap = args.xmode == "overlap" and P > 1
     for K in Ks:
-        if args.xmode == "allgather" and P > 1:
+        if overlap:  # f1: per-block broadcasts overlapped with column-block SpMM
+            ov[K] = gdist.OverlappedSpMM(g.row_ind, g.col_ind, g.val, spec, K, dev)
+        if args.xmode in ("allgather", "overlap") and P > 1:
             own = configs.make_features(name, spec.x1 - spec.x0, K, row0=spec.x0)
             Xown[K] = torch.zeros((spec.xblk, K), dtype=torch.float32, device=dev)
             Xown[K][:own.shape[0]] = torch.from_numpy(own).to(dev)
@@ -251,16 +254,25 @@ def time_path(args, g, perm, name, Ks, dev, world, rank, dtype="f32"):
     def step(ev=None):
         n = 0
         for K in Ks:
+            if ev is not None:
+                ev[K][4].record(stream)  # step start: the X exchange is inside the step
             if args.xmode == "allgather" and P > 1:
                 gdist.gather_features(Xown[K], spec, g.N, out=X[K])
             if ev is not None:
                 ev[K][0].record(stream)
-            pl = gs.plan(spg, K, feature_dtype=dtype)
-            n += 1
-            if ev is not None:
-                ev[K][1].record(stream)
-            gs.spmm(pl, spg, X[K], out=O[K])
-            n += 2 if spg.nnz else 0
+            if overlap:
+                n += P
+                if ev is not None:
+                    ev[K][1].record(stream)
+                X[K] = ov[K](Xown[K], O[K])
+                n += 2 * P
+            else:
+                pl = gs.plan(spg, K, feature_dtype=dtype)
+                n += 1
+                if ev is not None:
+                    ev[K][1].record(stream)
+                gs.spmm(pl, spg, X[K], out=O[K])
+                n += 2 if spg.nnz else 0
             if ev is not None:
                 ev[K][2].record(stream)
             pl2 = pl if same else gs.plan(sdg, K, feature_dtype=dtype)
@@ -276,7 +288,7 @@ def time_path(args, g, perm, name, Ks, dev, world, rank, dtype="f32"):
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
-    ev = [{K: [torch.cuda.Event(enable_timing=True) for _ in range(4)] for K in Ks}
+    ev = [{K: [torch.cuda.Event(enable_timing=True) for _ in range(5)] for K in Ks}
           for _ in range(args.steps)]
     clk = ClockSampler(dev.index)
     clk.start()
@@ -289,17 +301,19 @@ def time_path(args, g, perm, name, Ks, dev, world, rank, dtype="f32"):
         step(ev[s])
         torch.cuda.synchronize()
     clocks = clk.stop()
-    per = {K: {"plan": [], "spmm": [], "sddmm": []} for K in Ks}
+    per = {K: {"comm": [], "plan": [], "spmm": [], "sddmm": []} for K in Ks}
     step_ms = []
     for s in range(args.steps):
         tot = 0.0
         for K in Ks:
             e = ev[s][K]
+            x = e[4].elapsed_time(e[0])
             a, b, c = e[0].elapsed_time(e[1]), e[1].elapsed_time(e[2]), e[2].elapsed_time(e[3])
+            per[K]["comm"].append(x)
             per[K]["plan"].append(a)
             per[K]["spmm"].append(b)
             per[K]["sddmm"].append(c)
-            tot += a + b + c
+            tot += x + a + b + c
         step_ms.append(tot)
     my_bytes, my_flops, detail = 0, 0, {}
     eb = 2 if dtype == "bf16" else 4
@@ -313,6 +327,7 @@ def time_path(args, g, perm, name, Ks, dev, world, rank, dtype="f32"):
         detail[f"K{K}"] = {
             "chunk": info["chunk"], "vw_feat": info["vw_feat"], "lanes": info["lanes"],
             "active_blocks_per_sm": info["active_blocks_per_sm"],
+            "comm_ms": round(statistics.mean(per[K]["comm"]), 4),
             "plan_ms": round(statistics.mean(per[K]["plan"]), 4), "spmm_ms": round(t_sp, 4),
             "sddmm_ms": round(t_sd, 4), "spmm_GBps": round(b_sp / t_sp / 1e6, 1),
             "sddmm_GBps": round(b_sd / t_sd / 1e6, 1),
@@ -378,7 +393,7 @@ def run_ours(args):
     t0 = time.time()
     g0 = build_graph(name)
     gen_s = time.time() - t0
-    reorder = args.reorder and args.xmode != "allgather"
+    reorder = args.reorder and args.xmode == "replicate"
     if reorder:
         g, perm, reorder_info = gcr_reorder(g0)
     else:
@@ -706,7 +721,9 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--workload", default="C4")
     ap.add_argument("--K", default="")
-    ap.add_argument("--xmode", default="replicate", choices=["replicate", "allgather"])
+    ap.add_argument("--xmode", default="replicate", choices=["replicate", "allgather", "overlap"],
+                    help="X replicated on every rank, NCCL all-gathered inside the step, or "
+                         "broadcast per owner block overlapped with column-block SpMM (f1)")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--c3-graphs", type=int, default=20)
     ap.add_argument("--no-cpu", action="store_true")

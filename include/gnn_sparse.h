@@ -241,6 +241,18 @@ GNN_API gnn_status_t gnn_permute_rows(const float *X, int64_t ldx, int64_t n, in
 GNN_API gnn_status_t gnn_probe_gather(const float *X, int64_t ld, const int32_t *idx, int64_t n,
                                       int32_t K, float *sink, gnn_stream_t stream);
 
+/* Split a (row-shard) hybrid CSR/COO by the owner of each column, for overlapping the
+ * X all-gather with SpMM: column c belongs to block c / blk, P blocks.
+ * HOST arrays.  The nonzeros are stably partitioned by block (so every block is again a
+ * hybrid CSR/COO with non-decreasing rows): block q occupies
+ * [bounds[q], bounds[q+1]) of row_ind_out / col_ind_out / val_out (val may be NULL).
+ * Columns keep their global ids.  bounds: [P+1]. */
+GNN_API gnn_status_t gnn_split_col_blocks(const int32_t *row_ind_host, const int32_t *col_ind_host,
+                                          const float *val_host, int64_t nnz, int32_t P,
+                                          int64_t blk, int32_t *row_ind_out,
+                                          int32_t *col_ind_out, float *val_out,
+                                          int64_t *bounds);
+
 /* ------------------------------------------------------------- helpers ---- */
 /* Decode CSR offsets into the hybrid format's RowInd (Fig. 2d):
  * row_ind[i - row_ptr[0]] = r + row_base for row_ptr[r] <= i < row_ptr[r+1]. */

@@ -67,7 +67,7 @@ class ReorderOpts(ctypes.Structure):
 EXPORTS = ["gnn_plan_workspace_bytes", "gnn_plan_create", "gnn_plan_info", "gnn_plan_arrays",
            "gnn_plan_destroy", "gnn_spmm", "gnn_sddmm", "gnn_spmm_bf16", "gnn_sddmm_bf16",
            "gnn_spmm_ex", "gnn_transpose_workspace_bytes", "gnn_transpose",
-           "gnn_shard_rows", "gnn_shard_edges",
+           "gnn_shard_rows", "gnn_shard_edges", "gnn_split_col_blocks",
            "gnn_reorder_gcr", "gnn_permute_graph", "gnn_permute_rows",
            "gnn_probe_gather", "gnn_csr_to_coo", "gnn_validate", "gnn_last_error",
            "gnn_version"]
@@ -104,6 +104,8 @@ def lib():
         L.gnn_transpose.argtypes = [P(_Graph), vp, ctypes.c_size_t, vp, vp, vp, vp, vp, vp]
     L.gnn_shard_rows.argtypes = [vp, i64, i32, vp]
     L.gnn_shard_edges.argtypes = [i64, i32, vp]
+    if hasattr(L, "gnn_split_col_blocks"):
+        L.gnn_split_col_blocks.argtypes = [vp, vp, vp, i64, i32, i64, vp, vp, vp, vp]
     L.gnn_csr_to_coo.argtypes = [vp, i64, i64, vp, vp]
     L.gnn_reorder_gcr.argtypes = [vp, vp, i64, P(ReorderOpts), vp, vp, P(ctypes.c_double)]
     L.gnn_permute_graph.argtypes = [vp, vp, vp, i64, vp, vp, vp, vp, vp]
@@ -117,7 +119,8 @@ def lib():
     for f in ("gnn_plan_create", "gnn_plan_info", "gnn_plan_arrays", "gnn_spmm", "gnn_sddmm",
               "gnn_shard_rows", "gnn_shard_edges", "gnn_csr_to_coo", "gnn_validate",
               "gnn_reorder_gcr", "gnn_permute_graph", "gnn_permute_rows", "gnn_probe_gather",
-              "gnn_spmm_bf16", "gnn_sddmm_bf16", "gnn_spmm_ex", "gnn_transpose"):
+              "gnn_spmm_bf16", "gnn_sddmm_bf16", "gnn_spmm_ex", "gnn_transpose",
+              "gnn_split_col_blocks"):
         if hasattr(L, f):
             getattr(L, f).restype = st
     _lib = L
@@ -331,6 +334,23 @@ def shard_rows(row_ptr, P: int) -> np.ndarray:
     b = np.empty(P + 1, np.int64)
     _check(lib().gnn_shard_rows(rp.ctypes.data, rp.shape[0] - 1, P, b.ctypes.data))
     return b
+
+
+def split_col_blocks(row_ind, col_ind, val, P: int, blk: int):
+    """gnn_split_col_blocks (host): stable partition of the nonzeros by column owner block
+    (col // blk) -> (row_ind, col_ind, val, bounds[P+1])."""
+    ri = np.ascontiguousarray(row_ind, dtype=np.int32)
+    ci = np.ascontiguousarray(col_ind, dtype=np.int32)
+    v = None if val is None else np.ascontiguousarray(val, dtype=np.float32)
+    n = ri.shape[0]
+    ro, co = np.empty(n, np.int32), np.empty(n, np.int32)
+    vo = None if v is None else np.empty(n, np.float32)
+    b = np.empty(P + 1, np.int64)
+    _check(lib().gnn_split_col_blocks(ri.ctypes.data, ci.ctypes.data,
+                                      None if v is None else v.ctypes.data, n, P, blk,
+                                      ro.ctypes.data, co.ctypes.data,
+                                      None if vo is None else vo.ctypes.data, b.ctypes.data))
+    return ro, co, vo, b
 
 
 def shard_edges(nnz: int, P: int) -> np.ndarray:

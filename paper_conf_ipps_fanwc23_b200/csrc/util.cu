@@ -140,6 +140,34 @@ GNN_API gnn_status_t gnn_shard_edges(int64_t nnz, int32_t P, int64_t *bounds) {
   return GNN_OK;
 }
 
+GNN_API gnn_status_t gnn_split_col_blocks(const int32_t *row_ind, const int32_t *col_ind,
+                                          const float *val, int64_t nnz, int32_t P, int64_t blk,
+                                          int32_t *row_out, int32_t *col_out, float *val_out,
+                                          int64_t *bounds) {
+  if (nnz < 0 || P < 1 || blk < 1 || !bounds ||
+      (nnz > 0 && (!row_ind || !col_ind || !row_out || !col_out || (val && !val_out))))
+    return fail(GNN_ERR_INVALID_ARG, "gnn_split_col_blocks: bad arguments");
+  for (int32_t q = 0; q <= P; ++q) bounds[q] = 0;
+  for (int64_t i = 0; i < nnz; ++i) {  // counting pass
+    const int64_t q = col_ind[i] / blk;
+    if (col_ind[i] < 0 || q >= P)
+      return fail(GNN_ERR_INVALID_ARG, "gnn_split_col_blocks: column %d outside %d blocks of %lld",
+                  col_ind[i], P, (long long)blk);
+    bounds[q + 1]++;
+  }
+  for (int32_t q = 0; q < P; ++q) bounds[q + 1] += bounds[q];
+  int64_t fill[1024];
+  if (P > 1024) return fail(GNN_ERR_INVALID_ARG, "gnn_split_col_blocks: P > 1024");
+  for (int32_t q = 0; q < P; ++q) fill[q] = bounds[q];
+  for (int64_t i = 0; i < nnz; ++i) {  // stable scatter
+    const int64_t j = fill[col_ind[i] / blk]++;
+    row_out[j] = row_ind[i];
+    col_out[j] = col_ind[i];
+    if (val) val_out[j] = val[i];
+  }
+  return GNN_OK;
+}
+
 GNN_API gnn_status_t gnn_csr_to_coo(const int32_t *row_ptr, int64_t M, int64_t row_base,
                                     int32_t *row_ind, gnn_stream_t stream) {
   if (M < 0 || (M > 0 && (!row_ptr || !row_ind)))

@@ -69,3 +69,68 @@ def gather_features(own: torch.Tensor, s: ShardSpec, N: int, out: torch.Tensor |
         out = torch.empty((s.xblk * s.world, K), dtype=own.dtype, device=own.device)
     dist.all_gather_into_tensor(out, own.contiguous(), group=group)
     return out
+
+
+# ------------------------------------------------------------------------------
+# f1: overlap the X all-gather with SpMM.  Each rank splits its row shard
+# by column owner block (gnn_split_col_blocks), computes the block whose X rows it owns
+# while the other blocks are still being broadcast, then each remaining block as soon as
+# its broadcast lands, accumulating into O (gnn_spmm_ex with beta = 1) in a fixed order.
+
+def block_order(P: int, p: int):
+    """Compute order on rank p: the local block first, then the others in the order
+    their broadcasts are issued (0..P-1, skipping p)."""
+    return [p] + [q for q in range(P) if q != p]
+
+
+def start_block_broadcasts(X_full: torch.Tensor, s: ShardSpec, group=None):
+    """Issue one broadcast per owner block (the same order on every rank) and return the
+    async works; works[q].wait() makes the current stream wait for block q."""
+    works = []
+    for q in range(s.world):
+        blk = X_full[q * s.xblk:(q + 1) * s.xblk]
+        works.append(dist.broadcast(blk, src=q, group=group, async_op=True))
+    return works
+
+
+class OverlappedSpMM:
+    """Row-shard SpMM whose feature rows arrive block by block (f1)."""
+
+    def __init__(self, row_ind, col_ind, val, s: ShardSpec, K: int, device, group=None):
+        from . import DeviceGraph, plan, split_col_blocks
+        import numpy as _np
+        self.s, self.K, self.group = s, K, group
+        ro, co, vo, b = split_col_blocks(_np.asarray(row_ind)[s.e0:s.e1],
+                                         _np.asarray(col_ind)[s.e0:s.e1],
+                                         None if val is None else _np.asarray(val)[s.e0:s.e1],
+                                         s.world, s.xblk)
+        self.bounds = b
+        t = lambda a, dt: torch.from_numpy(a).to(device=device, dtype=dt)
+        self.ri, self.ci = t(ro, torch.int32), t(co, torch.int32)
+        self.vi = None if vo is None else t(vo, torch.float32)
+        self.blocks, self.plans = [], []
+        for q in range(s.world):
+            a, z = int(b[q]), int(b[q + 1])
+            g = DeviceGraph(s.r1 - s.r0, s.xblk * s.world, self.ri[a:z], self.ci[a:z],
+                            None if self.vi is None else self.vi[a:z], None, s.r0)
+            self.blocks.append(g)
+            self.plans.append(plan(g, K))
+        self.X_full = torch.empty((s.xblk * s.world, K), dtype=torch.float32, device=device)
+
+    def __call__(self, X_own: torch.Tensor, O: torch.Tensor, replan: bool = True) -> torch.Tensor:
+        """X_own: this rank's xblk x K rows (padded); O: (r1 - r0) x K output.  Returns
+        the gathered X (complete on the current stream when this returns).  replan=True
+        rebuilds the per-block plans (GPU plan kernel) as part of the step."""
+        from . import plan, spmm
+        s = self.s
+        if replan:
+            self.plans = [plan(g, self.K) for g in self.blocks]
+        self.X_full[s.rank * s.xblk:(s.rank + 1) * s.xblk].copy_(X_own)
+        works = start_block_broadcasts(self.X_full, s, self.group)
+        first = True
+        for q in block_order(s.world, s.rank):
+            if q != s.rank:
+                works[q].wait()
+            spmm(self.plans[q], self.blocks[q], self.X_full, out=O, accumulate=not first)
+            first = False
+        return self.X_full

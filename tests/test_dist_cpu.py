@@ -98,3 +98,59 @@ def test_shard_spec_covers_everything():
         assert sum(s.x1 - s.x0 for s in specs) == g.N
         for a, b in zip(specs, specs[1:]):
             assert a.r1 == b.r0 and a.f1 == b.f0 and a.e1 == b.e0
+
+
+def _overlap_worker(rank, world, port, q):
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    sys.path.insert(0, root)
+    import gen
+    import oracle
+    import paper_conf_ipps_fanwc23_b200 as gs
+    from paper_conf_ipps_fanwc23_b200 import dist as gdist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        g = gen.powerlaw_graph(2501, 50000, gamma=2.2, n_comm=5, seed=93)
+        K = 16
+        s = gdist.shard_spec(g.row_ptr, g.N, rank, world)
+        X = gen.features(94, g.N, K)
+        Xf = torch.zeros((s.xblk * world, K))
+        own = torch.from_numpy(gen.features(94, s.x1 - s.x0, K, row0=s.x0))
+        Xf[s.x0:s.x1] = own
+        works = gdist.start_block_broadcasts(Xf, s)
+        ro, co, vo, b = gs.split_col_blocks(g.row_ind[s.e0:s.e1], g.col_ind[s.e0:s.e1],
+                                            g.val[s.e0:s.e1], world, s.xblk)
+        O = np.zeros((s.r1 - s.r0, K))
+        for qq in gdist.block_order(world, rank):
+            if qq != rank:
+                works[qq].wait()
+            a, z = int(b[qq]), int(b[qq + 1])
+            part, _ = oracle.spmm(ro, co, vo, Xf.numpy(), i0=a, i1=z, r0=s.r0,
+                                  nrows=s.r1 - s.r0)
+            O += part
+        ref, _ = oracle.spmm(g.row_ind, g.col_ind, g.val, X, i0=s.e0, i1=s.e1, r0=s.r0,
+                             nrows=s.r1 - s.r0)
+        ok = bool(np.allclose(O, ref, rtol=0, atol=1e-12)) and bool(
+            np.array_equal(Xf[:g.N].numpy(), X))
+        res = [None] * world
+        dist.all_gather_object(res, ok)
+        if rank == 0:
+            q.put(all(res))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_gloo_overlapped_block_broadcast_spmm():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    world = 2
+    procs = [ctx.Process(target=_overlap_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    for p in procs:
+        p.join(timeout=240)
+        assert p.exitcode == 0
+    assert q.get(timeout=10)

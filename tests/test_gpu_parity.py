@@ -452,3 +452,33 @@ def test_bf16_plan_dtype_mismatch_rejected():
     p = gs.plan(dg, 32)  # fp32 plan
     with pytest.raises(gs.GnnError):
         gs.spmm(p, dg, torch.zeros((g.N, 32), dtype=torch.bfloat16, device=DEV))
+
+
+@pytest.mark.parametrize("P", [2, 4, 8])
+def test_column_block_accumulation_equals_spmm(P):
+    """f1 building block: a row shard split by column owner block (gnn_split_col_blocks),
+    SpMM of the local block (beta = 0) then the others accumulated (beta = 1) in
+    block_order, equals the shard's SpMM."""
+    from paper_conf_ipps_fanwc23_b200 import dist as gdist
+    g = gen.powerlaw_graph(6000, 300000, gamma=2.2, n_comm=6, seed=90 + P)
+    K = 64
+    X = _x(91, g.N, K)
+    for rank in range(P):
+        s = gdist.shard_spec(g.row_ptr, g.N, rank, P)
+        ro, co, vo, b = gs.split_col_blocks(g.row_ind[s.e0:s.e1], g.col_ind[s.e0:s.e1],
+                                            g.val[s.e0:s.e1], P, s.xblk)
+        Xf = np.zeros((s.xblk * P, K), np.float32)
+        Xf[:g.N] = X
+        Xd = torch.from_numpy(Xf).to(DEV)
+        O = torch.full((s.r1 - s.r0, K), float("nan"), device=DEV)
+        first = True
+        for q in gdist.block_order(P, rank):
+            a, z = int(b[q]), int(b[q + 1])
+            bg = gs.DeviceGraph.from_arrays(s.r1 - s.r0, s.xblk * P, ro[a:z], co[a:z], vo[a:z],
+                                            row_base=s.r0)
+            gs.spmm(gs.plan(bg, K), bg, Xd, out=O, accumulate=not first)
+            first = False
+        ref, T = oracle.spmm(g.row_ind, g.col_ind, g.val, X, i0=s.e0, i1=s.e1, r0=s.r0,
+                             nrows=s.r1 - s.r0)
+        torch.cuda.synchronize()
+        assert_within(O.cpu().numpy(), ref, T, what=f"column blocks P={P} rank={rank}")
