@@ -180,8 +180,16 @@ class DeviceGraph:
                            self.row_base + r0)
 
     def desc(self) -> _Graph:
-        return _Graph(self.M, self.N, self.nnz, _ptr(self.row_ptr), _ptr(self.row_ind),
-                      _ptr(self.col_ind), _ptr(self.val), self.row_base)
+        # cached: the descriptor is rebuilt only if an array was replaced
+        key = (self.M, self.N, self.row_base,
+               *(None if t is None else (t.data_ptr(), t.numel())
+                 for t in (self.row_ptr, self.row_ind, self.col_ind, self.val)))
+        if self._keep and self._keep[0] == key:
+            return self._keep[1]
+        d = _Graph(self.M, self.N, self.nnz, _ptr(self.row_ptr), _ptr(self.row_ind),
+                   _ptr(self.col_ind), _ptr(self.val), self.row_base)
+        self._keep[:] = [key, d]
+        return d
 
 
 # ------------------------------------------------------------------ plan ----

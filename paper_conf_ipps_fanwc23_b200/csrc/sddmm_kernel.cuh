@@ -40,7 +40,7 @@ struct SddmmShape {
 // slot i of lane l with u = l * (U/L) + i.  Then S_O = sum * v (Algo 2 line 6) is
 // stored for the first `valid` of the U nonzeros at out[0..U).
 template <int U, int L>
-__device__ __forceinline__ void reduce_scale_store(float (&part)[U], const float (&vj)[U],
+__device__ __forceinline__ void reduce_scale_store(float (&part)[U], const float *sval,
                                                    const int l, float *__restrict__ out,
                                                    const int valid) {
   constexpr int P = U > L ? U / L : 1;  // values left per lane after the halving steps
@@ -64,25 +64,16 @@ __device__ __forceinline__ void reduce_scale_store(float (&part)[U], const float
       part[0] += __shfl_xor_sync(kFull, part[0], o, L);
     }
   }
+  // the owner lane of nonzero u reads its value straight from the shared-memory tile
   if constexpr (U <= L) {
     constexpr int R = L / U;
     const int u = l / R;
-    if (l % R == 0 && u < valid) {
-      float v = vj[0];
-#pragma unroll
-      for (int w = 1; w < U; ++w) v = (w == u) ? vj[w] : v;
-      out[u] = part[0] * v;
-    }
+    if (l % R == 0 && u < valid) out[u] = part[0] * (sval ? sval[u] : 1.f);
   } else {
 #pragma unroll
     for (int i = 0; i < P; ++i) {
       const int u = l * P + i;
-      if (u < valid) {
-        float v = vj[0];
-#pragma unroll
-        for (int w = 1; w < U; ++w) v = (w == u) ? vj[w] : v;
-        out[u] = part[i] * v;
-      }
+      if (u < valid) out[u] = part[i] * (sval ? sval[u] : 1.f);
     }
   }
 }
@@ -172,11 +163,10 @@ __global__ void __launch_bounds__(kMaxThreads, (SddmmShape<VW, L, SMAX>::minb))
       for (int jj = 0; jj < T; jj += U) {
         int32_t rj[U];
         uint32_t cj[U];
-        float vj[U], part[U];
+        float part[U];
 #pragma unroll
         for (int u = 0; u < U; ++u) {
           cj[u] = (uint32_t)s_col[jj + u];
-          vj[u] = vi ? s_val[jj + u] : 1.f;
           if constexpr (!FAST) rj[u] = s_row[jj + u];
           part[u] = 0.f;
         }
@@ -212,7 +202,8 @@ __global__ void __launch_bounds__(kMaxThreads, (SddmmShape<VW, L, SMAX>::minb))
             }
           }
         }
-        reduce_scale_store<U, Lg>(part, vj, l, oc + tb + jj, item_ok ? (FAST ? U : valid) : 0);
+        reduce_scale_store<U, Lg>(part, vi ? s_val + jj : nullptr, l, oc + tb + jj,
+                                  item_ok ? (FAST ? U : valid) : 0);
       }
     };
     if (fast) run_tile(std::true_type{});
