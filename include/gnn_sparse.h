@@ -232,6 +232,25 @@ GNN_API gnn_status_t gnn_permute_rows(const float *X, int64_t ldx, int64_t n, in
                                       const int32_t *perm, float *Y, int64_t ldy,
                                       gnn_stream_t stream);
 
+/* ------------------------------------------------------------ end to end ---- */
+/* The whole path on HOST buffers (bench.py's "e2e" number): copies the hybrid CSR/COO
+ * arrays (if upload_graph) and X from host memory into the caller's device workspace,
+ * builds the plan (GPU plan kernel), runs SpMM (O = S X, if O_host) and SDDMM
+ * (S_O[i] = v_i <X_r, X_c>, i.e. A1 = A2T = X, if out_host), and copies O (M x K, pitch K)
+ * and S_O (nnz) back.  Everything is enqueued on `stream` and returns without waiting:
+ * synchronise the stream before reading O_host / out_host or reusing X_host (pinned host
+ * memory gives asynchronous DMA; pageable memory works but copies synchronously).
+ * graph_host: square (M == N), row_base 0, host pointers (row_ptr unused).  fp32 only.
+ * upload_graph = 0 reuses the graph already in this workspace from an earlier call (the
+ * graph's offsets do not depend on K, so one workspace sized for the largest K serves all).
+ * workspace: gnn_run_host_workspace_bytes(M, N, nnz, K, opts) bytes, 256-B aligned, device. */
+GNN_API size_t gnn_run_host_workspace_bytes(int64_t M, int64_t N, int64_t nnz, int32_t K,
+                                            const gnn_plan_opts_t *opts);
+GNN_API gnn_status_t gnn_run_host(const gnn_graph_t *graph_host, int32_t upload_graph,
+                                  const float *X_host, int32_t K, float *O_host,
+                                  float *out_host, const gnn_plan_opts_t *opts, void *workspace,
+                                  size_t ws_bytes, gnn_stream_t stream);
+
 /* ----------------------------------------------------------- measurement --- */
 /* Roofline probe (not part of the method): gathers rows X[idx[i]][0:K] for i in [0, n)
  * with the same 256-bit row loads the kernels use and no other work (sums are folded

@@ -69,7 +69,7 @@ EXPORTS = ["gnn_plan_workspace_bytes", "gnn_plan_create", "gnn_plan_info", "gnn_
            "gnn_spmm_ex", "gnn_transpose_workspace_bytes", "gnn_transpose",
            "gnn_shard_rows", "gnn_shard_edges", "gnn_split_col_blocks",
            "gnn_reorder_gcr", "gnn_permute_graph", "gnn_permute_rows",
-           "gnn_probe_gather", "gnn_csr_to_coo", "gnn_validate", "gnn_last_error",
+           "gnn_probe_gather", "gnn_run_host_workspace_bytes", "gnn_run_host", "gnn_csr_to_coo", "gnn_validate", "gnn_last_error",
            "gnn_version"]
 
 _lib = None
@@ -104,6 +104,11 @@ def lib():
         L.gnn_transpose.argtypes = [P(_Graph), vp, ctypes.c_size_t, vp, vp, vp, vp, vp, vp]
     L.gnn_shard_rows.argtypes = [vp, i64, i32, vp]
     L.gnn_shard_edges.argtypes = [i64, i32, vp]
+    if hasattr(L, "gnn_run_host"):
+        L.gnn_run_host_workspace_bytes.argtypes = [i64, i64, i64, i32, P(PlanOpts)]
+        L.gnn_run_host_workspace_bytes.restype = ctypes.c_size_t
+        L.gnn_run_host.argtypes = [P(_Graph), i32, vp, i32, vp, vp, P(PlanOpts), vp,
+                                   ctypes.c_size_t, vp]
     if hasattr(L, "gnn_split_col_blocks"):
         L.gnn_split_col_blocks.argtypes = [vp, vp, vp, i64, i32, i64, vp, vp, vp, vp]
     L.gnn_csr_to_coo.argtypes = [vp, i64, i64, vp, vp]
@@ -120,7 +125,7 @@ def lib():
               "gnn_shard_rows", "gnn_shard_edges", "gnn_csr_to_coo", "gnn_validate",
               "gnn_reorder_gcr", "gnn_permute_graph", "gnn_permute_rows", "gnn_probe_gather",
               "gnn_spmm_bf16", "gnn_sddmm_bf16", "gnn_spmm_ex", "gnn_transpose",
-              "gnn_split_col_blocks"):
+              "gnn_split_col_blocks", "gnn_run_host"):
         if hasattr(L, f):
             getattr(L, f).restype = st
     _lib = L
@@ -434,3 +439,42 @@ def probe_gather(X: torch.Tensor, idx: torch.Tensor, sink: torch.Tensor | None =
         sink = torch.zeros(1, device=X.device)
     _check(lib().gnn_probe_gather(_ptr(X), X.stride(0), _ptr(idx), idx.numel(), X.shape[1],
                                   _ptr(sink), _stream(stream)))
+
+
+class HostRunner:
+    """gnn_run_host: the end-to-end call on HOST buffers.  Holds the device workspace
+    (sized for the largest K) and the host graph descriptor; run() enqueues H2D copies,
+    plan, SpMM, SDDMM and D2H copies on the current stream (synchronise before reading)."""
+
+    def __init__(self, M, N, row_ind, col_ind, val, Kmax, device="cuda", **opts):
+        self._keep = [np.ascontiguousarray(row_ind, np.int32),
+                      np.ascontiguousarray(col_ind, np.int32),
+                      None if val is None else np.ascontiguousarray(val, np.float32)]
+        self.M, self.N, self.nnz = int(M), int(N), int(row_ind.shape[0] if hasattr(row_ind, "shape") else len(row_ind))
+        self.opts = _opts(**opts)
+        nbytes = lib().gnn_run_host_workspace_bytes(self.M, self.N, self.nnz, Kmax,
+                                                    ctypes.byref(self.opts))
+        if nbytes == ctypes.c_size_t(-1).value:
+            _check(GNN_ERR_INVALID_ARG)
+        self.ws = torch.empty(max(int(nbytes), 1), dtype=torch.uint8, device=device)
+        self.ws_bytes = int(nbytes)
+        self.desc = _Graph(self.M, self.N, self.nnz, None, self._keep[0].ctypes.data,
+                           self._keep[1].ctypes.data,
+                           None if self._keep[2] is None else self._keep[2].ctypes.data, 0)
+
+    def pin(self):
+        """Re-point the graph at pinned copies (asynchronous H2D)."""
+        pinned = [None if a is None else torch.from_numpy(a).pin_memory() for a in self._keep]
+        self._pinned = pinned
+        self.desc = _Graph(self.M, self.N, self.nnz, None, pinned[0].data_ptr(),
+                           pinned[1].data_ptr(), None if pinned[2] is None else pinned[2].data_ptr(), 0)
+        return self
+
+    def run(self, X_host: torch.Tensor, K: int, O_host=None, out_host=None, upload_graph=True,
+            stream=None):
+        for t in (X_host, O_host, out_host):
+            if t is not None and (t.is_cuda or not t.is_contiguous() or t.dtype != torch.float32):
+                raise ValueError("host buffers must be contiguous fp32 CPU tensors")
+        _check(lib().gnn_run_host(ctypes.byref(self.desc), int(upload_graph), _ptr(X_host), K,
+                                  _ptr(O_host), _ptr(out_host), ctypes.byref(self.opts),
+                                  _ptr(self.ws), self.ws_bytes, _stream(stream)))

@@ -482,3 +482,20 @@ def test_column_block_accumulation_equals_spmm(P):
                              nrows=s.r1 - s.r0)
         torch.cuda.synchronize()
         assert_within(O.cpu().numpy(), ref, T, what=f"column blocks P={P} rank={rank}")
+
+
+def test_run_host_end_to_end_matches_oracle():
+    """gnn_run_host (HOST buffers in, HOST results out) for several K with one workspace
+    and one graph upload."""
+    g = configs.make_graph("C2")
+    runner = gs.HostRunner(g.M, g.N, g.row_ind, g.col_ind, g.val, 128, device=DEV).pin()
+    for j, K in enumerate((32, 64, 128)):
+        X = torch.from_numpy(_x(800 + K, g.N, K)).pin_memory()
+        O = torch.empty((g.M, K)).pin_memory()
+        E = torch.empty(g.nnz).pin_memory()
+        runner.run(X, K, O, E, upload_graph=(j == 0))
+        torch.cuda.synchronize()
+        ref, T = oracle.spmm(g.row_ind, g.col_ind, g.val, X.numpy(), M=g.M)
+        assert_within(O.numpy(), ref, T, what=f"run_host spmm K={K}")
+        r2, T2 = oracle.sddmm(g.row_ind, g.col_ind, g.val, X.numpy(), X.numpy())
+        assert_within(E.numpy(), r2, T2, what=f"run_host sddmm K={K}")
