@@ -89,8 +89,11 @@ int spmm_active_blocks_per_sm(int dtype, int vw, int lanes, int vecs, int wpb) {
   if (!f) return 0;
   // the plan's vw_sparse is not known yet: size the tiles for the widest (4)
   const size_t smem = (size_t)wpb * spmm_tile_bytes_per_warp(lanes, 4);
-  if (cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
-      cudaSuccess)
+  // only ever raise the per-function limit above the 48 KB default (a smaller value would
+  // make later launches with more warps per block fail); launches re-raise it as needed
+  if (smem > 48 * 1024 &&
+      cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
+          cudaSuccess)
     return 0;
   if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, f, wpb * 32, smem) != cudaSuccess)
     return 0;

@@ -107,3 +107,56 @@ def test_gcn_training_reduces_loss():
         opt.step()
         losses.append(loss.item())
     assert losses[-1] < 0.7 * losses[0], losses
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_randomized_configurations(seed):
+    """Seeded fuzz over shapes and every plan/kernel knob: random sparsity with empty rows
+    and hubs, K (odd/even, > 512), forced chunk / vector width, warps per block, alpha,
+    val None, bf16 features, aggregators; every output against the oracle."""
+    rng = np.random.default_rng(10_000 + seed)
+    M = int(rng.integers(1, 3000))
+    N = int(rng.integers(1, 3000))
+    nnz = int(rng.integers(0, 40000))
+    rows = np.sort(rng.integers(0, M, nnz))
+    if nnz > 10 and rng.random() < 0.5:
+        rows[: nnz // 3] = rows[0]                       # a hub row
+    cols = rng.integers(0, N, nnz)
+    vals = rng.uniform(-1, 1, nnz).astype(np.float32)
+    g = gen.from_coo(M, N, rows, cols, vals)
+    K = int(rng.choice([1, 2, 3, 7, 8, 16, 24, 40, 64, 96, 128, 200, 256, 520, 1024]))
+    bf16 = K % 2 == 0 and rng.random() < 0.3
+    kw = {}
+    if rng.random() < 0.4:
+        kw["force_chunk"] = int(rng.choice([1, 3, 8, 17, 32, 64, 100, 128, 256, 512]))
+    if rng.random() < 0.3:
+        choices = [v for v in ((2, 4, 8, 16) if bf16 else (1, 2, 4, 8)) if K % v == 0]
+        if choices:
+            kw["force_vw"] = int(rng.choice(choices))
+    if rng.random() < 0.3:
+        kw["warps_per_block"] = int(rng.choice([1, 2, 4, 16]))
+    if rng.random() < 0.3:
+        kw["alpha"] = int(rng.choice([1, 3, 8]))
+    with_val = rng.random() < 0.8
+    dg = upload(g, with_val=with_val)
+    p = gs.plan(dg, K, feature_dtype="bf16" if bf16 else "f32", **kw)
+    info = p.info()
+    ref_plan = oracle.plan(g.row_ind, K, info["num_sms"], info["active_blocks_per_sm"],
+                           alpha=kw.get("alpha", 2), warps_per_block=kw.get("warps_per_block", 8),
+                           force_chunk=kw.get("force_chunk", 0), force_vw=kw.get("force_vw", 0),
+                           feature_dtype=1 if bf16 else 0)
+    assert info == ref_plan.info
+    X = torch.from_numpy(gen.features(seed, N, K)).to(DEV)
+    A1 = torch.from_numpy(gen.features(seed + 1, M, K)).to(DEV)
+    if bf16:
+        X, A1 = X.to(torch.bfloat16), A1.to(torch.bfloat16)
+    Xh, A1h = X.float().cpu().numpy(), A1.float().cpu().numpy()
+    val = g.val if with_val else None
+    agg = "sum" if bf16 else str(rng.choice(["sum", "sum", "mean", "max", "min"]))
+    O = gs.spmm(p, dg, X, agg=agg).cpu().numpy()
+    ref, T = oracle.spmm_agg(g.row_ind, g.col_ind, val, Xh, agg, M=M)
+    assert_within(O, ref, T, tol=1e-5 if agg in ("sum", "mean") else 1e-6, what=f"spmm {agg}")
+    if p.info()["slices"] <= 4:
+        E = gs.sddmm(p, dg, A1, X).cpu().numpy()
+        r2, T2 = oracle.sddmm(g.row_ind, g.col_ind, val, A1h, Xh)
+        assert_within(E, r2, T2, what="sddmm")
