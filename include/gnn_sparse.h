@@ -76,7 +76,9 @@ typedef struct {
   int32_t warps_per_block; /* WarpsPerBlock; 1..16, default 8               */
   int32_t force_chunk;     /* 0 = DTP choice; >0 forces NnzPerWarp (ablation/tests) */
   int32_t force_vw;        /* 0 = from K; 1/2/4/8 forces the feature vector width   */
-  int32_t deterministic;   /* reserved (must be 0 in this version)                  */
+  int32_t deterministic;   /* 1: SpMM sums rows split across chunks in chunk order
+                              through per-chunk partials in the workspace (no atomics:
+                              bit-reproducible; workspace grows by 8*K B per chunk)     */
   int32_t feature_dtype;   /* gnn_dtype_t of the feature matrices; default GNN_F32   */
 } gnn_plan_opts_t;
 

@@ -250,16 +250,20 @@ def _dtype_code(d):
     raise ValueError(f"unsupported feature dtype {d!r}")
 
 
-def _opts(alpha=0, warps_per_block=0, force_chunk=0, force_vw=0, feature_dtype=0):
-    return PlanOpts(alpha, warps_per_block, force_chunk, force_vw, 0, _dtype_code(feature_dtype))
+def _opts(alpha=0, warps_per_block=0, force_chunk=0, force_vw=0, feature_dtype=0,
+          deterministic=False):
+    return PlanOpts(alpha, warps_per_block, force_chunk, force_vw, int(bool(deterministic)),
+                    _dtype_code(feature_dtype))
 
 
 def plan(graph: DeviceGraph, K: int, alpha: int = 0, warps_per_block: int = 0,
-         force_chunk: int = 0, force_vw: int = 0, feature_dtype=GNN_F32, stream=None) -> Plan:
+         force_chunk: int = 0, force_vw: int = 0, feature_dtype=GNN_F32,
+         deterministic: bool = False, stream=None) -> Plan:
     """gnn_plan_create: DTP/HVMA chunking + the GPU plan kernel (no host sync).
-    feature_dtype: fp32 (default) or bf16 feature matrices."""
+    feature_dtype: fp32 (default) or bf16 feature matrices.
+    deterministic: split rows summed in chunk order without atomics (bit-reproducible)."""
     L = lib()
-    o = _opts(alpha, warps_per_block, force_chunk, force_vw, feature_dtype)
+    o = _opts(alpha, warps_per_block, force_chunk, force_vw, feature_dtype, deterministic)
     nbytes = L.gnn_plan_workspace_bytes(graph.nnz, K, ctypes.byref(o))
     if nbytes == ctypes.c_size_t(-1).value:
         _check(GNN_ERR_INVALID_ARG)

@@ -28,6 +28,7 @@ struct Plan {
   int32_t *row_first;
   int32_t *row_last;
   uint8_t *flags;
+  float *carry;  // deterministic plans: [num_chunks][2][K] split-row partials, else null
   int64_t M;
   int64_t row_base;
 };
@@ -49,6 +50,7 @@ struct SparseArgs {
   int32_t slices;
   int32_t vecs;
   int32_t accum;  // 1: O += S A (beta = 1), rows without nonzeros untouched
+  float *carry;   // deterministic: split-row partials [chunk][first|last][K] (no atomics)
 };
 
 // Occupancy (active blocks / SM) of the SpMM kernel for a feature width/lane count;

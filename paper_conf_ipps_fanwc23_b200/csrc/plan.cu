@@ -32,7 +32,8 @@ gnn_status_t make_info(int64_t nnz, int32_t K, const gnn_plan_opts_t *opts,
   const int32_t alpha = o.alpha ? o.alpha : 2;
   const int32_t wpb = o.warps_per_block ? o.warps_per_block : 8;
   if (nnz < 0 || nnz >= (int64_t(1) << 31) || K < 1 || alpha < 1 || wpb < 1 ||
-      wpb * 32 > kMaxThreads || o.force_chunk < 0 || o.deterministic != 0)
+      wpb * 32 > kMaxThreads || o.force_chunk < 0 || o.deterministic < 0 ||
+      o.deterministic > 1)
     return fail(GNN_ERR_INVALID_ARG,
                 "plan: bad arguments (nnz=%lld K=%d alpha=%d wpb=%d force_chunk=%d det=%d)",
                 (long long)nnz, K, alpha, wpb, o.force_chunk, o.deterministic);
@@ -98,9 +99,14 @@ gnn_status_t make_info(int64_t nnz, int32_t K, const gnn_plan_opts_t *opts,
   return GNN_OK;
 }
 
-size_t ws_bytes_for(int64_t nch) {
+// row_first | row_last | flags [| carry: 2 partial rows of K fp32 per chunk when the
+// plan is deterministic (split rows are summed in chunk order by a fix-up pass instead of
+// with atomics)]
+size_t ws_bytes_for(int64_t nch, int32_t K, int32_t deterministic) {
   if (nch == 0) return 0;
-  return 2 * align256(sizeof(int32_t) * nch) + align256(nch);
+  size_t b = 2 * align256(sizeof(int32_t) * nch) + align256(nch);
+  if (deterministic) b += align256(sizeof(float) * 2 * (size_t)nch * K);
+  return b;
 }
 
 // One thread per chunk: Algo 3 lines 2-3 (warp_start = id * NnzPerWarp, end
@@ -131,7 +137,7 @@ extern "C" {
 GNN_API size_t gnn_plan_workspace_bytes(int64_t nnz, int32_t K, const gnn_plan_opts_t *opts) {
   gnn_plan_info_t info;
   if (make_info(nnz, K, opts, &info) != GNN_OK) return (size_t)-1;
-  return ws_bytes_for(info.num_chunks);
+  return ws_bytes_for(info.num_chunks, K, opts ? opts->deterministic : 0);
 }
 
 GNN_API gnn_status_t gnn_plan_create(const gnn_graph_t *g, int32_t K,
@@ -145,7 +151,8 @@ GNN_API gnn_status_t gnn_plan_create(const gnn_graph_t *g, int32_t K,
   gnn_plan_info_t info;
   if (gnn_status_t st = make_info(g->nnz, K, opts, &info)) return st;
   const int64_t nch = info.num_chunks;
-  const size_t need = ws_bytes_for(nch);
+  const int32_t det = opts ? opts->deterministic : 0;
+  const size_t need = ws_bytes_for(nch, K, det);
   if (ws_bytes < need || (need > 0 && (!workspace || !aligned(workspace, 256))))
     return fail(GNN_ERR_WORKSPACE, "gnn_plan_create: workspace %zu B (need %zu B, 256-B aligned)",
                 ws_bytes, need);
@@ -159,6 +166,8 @@ GNN_API gnn_status_t gnn_plan_create(const gnn_graph_t *g, int32_t K,
   p->row_first = (int32_t *)w;
   p->row_last = (int32_t *)(w + align256(sizeof(int32_t) * nch));
   p->flags = (uint8_t *)(w + 2 * align256(sizeof(int32_t) * nch));
+  p->carry = det && nch > 0 ? (float *)(w + 2 * align256(sizeof(int32_t) * nch) + align256(nch))
+                            : nullptr;
   DeviceInfo d;
   device_info(&d);
   p->device = d.device;

@@ -47,6 +47,31 @@ __global__ void spmm_prezero_kernel(const SparseArgs a, float *__restrict__ O,
   for (int k = lane * VW; k < a.K; k += 32 * VW) st_vec<VW>(o + k, z);
 }
 
+// Deterministic plans: every row split across chunks is combined from the per-chunk
+// partials in chunk order (no atomics): one warp per chunk in which such a row starts,
+// lanes over the K columns.  AGG: 0 sum, 1 max, 2 min.
+template <int AGG>
+__global__ void spmm_fixup_kernel(const SparseArgs a, float *__restrict__ O, const int64_t ldo) {
+  const int64_t c0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  if (c0 >= a.num_chunks) return;
+  const uint32_t f0 = a.flags[c0];
+  if (!(f0 & 2u)) return;
+  const int32_t rf0 = a.row_first[c0], r = a.row_last[c0];
+  if ((f0 & 1u) && rf0 == r) return;  // the row started in an earlier chunk
+  const int K = a.K;
+  float *o = O + ((int64_t)r - a.row_base) * ldo;
+  for (int k = lane; k < K; k += 32) {
+    float acc = a.carry[(c0 * 2 + (r == rf0 ? 0 : 1)) * (int64_t)K + k];
+    for (int64_t c = c0 + 1; c < a.num_chunks; ++c) {  // chunk c starts with row r
+      const float v = a.carry[(c * 2) * (int64_t)K + k];
+      acc = AGG == 0 ? acc + v : (AGG == 1 ? fmaxf(acc, v) : fminf(acc, v));
+      if (!((a.flags[c] & 2u) && a.row_last[c] == r)) break;
+    }
+    o[k] = (AGG == 0 && a.accum) ? o[k] + acc : acc;
+  }
+}
+
 // Mean aggregator: O[r] *= 1 / (nonzeros of row r) for rows with nonzeros (row_ptr read
 // relative to row_ptr[0]).  One warp per row.
 __global__ void spmm_row_mean_kernel(const int32_t *__restrict__ row_ptr, int64_t M, int32_t K,
@@ -150,6 +175,7 @@ SparseArgs make_args(const Plan *p, const gnn_graph_t *g) {
   a.slices = p->info.slices;
   a.vecs = p->info.vecs;
   a.accum = 0;
+  a.carry = nullptr;
   return a;
 }
 
@@ -200,8 +226,9 @@ static gnn_status_t launch_spmm(const Plan *p, const gnn_graph_t *g, const void 
                 in.lanes, agg_api, dtype);
   SparseArgs a = make_args(p, g);
   a.accum = accumulate;
+  a.carry = p->carry;
   const int threads = in.warps_per_block * 32;
-  if (!accumulate) {
+  if (!accumulate && !a.carry) {
     const int64_t blocks = (a.num_chunks * 32 + 255) / 256;
     const float init = agg == kAggMax ? -INFINITY : agg == kAggMin ? INFINITY : 0.f;
     switch (VO) {
@@ -217,6 +244,12 @@ static gnn_status_t launch_spmm(const Plan *p, const gnn_graph_t *g, const void 
     if (e != cudaSuccess) return cuda_fail(e, "gnn_spmm smem attribute");
   }
   f<<<(unsigned)in.num_blocks, threads, smem, s>>>(a, A, lda, O, ldo);
+  if (a.carry) {
+    const int64_t blocks = (a.num_chunks * 32 + 255) / 256;
+    if (agg == kAggMax) spmm_fixup_kernel<1><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo);
+    else if (agg == kAggMin) spmm_fixup_kernel<2><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo);
+    else spmm_fixup_kernel<0><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo);
+  }
   if (agg_api == GNN_AGG_MEAN) {
     DeviceInfo d;
     device_info(&d);

@@ -145,6 +145,16 @@ __global__ void __launch_bounds__(kMaxThreads, GNN_SPMM_MINB)
   };
   float acc[R][VW];
   auto flush = [&](int32_t row) {
+    if (a.carry) {  // deterministic plan: split rows go to this chunk's partial slots
+      const bool shared = (row == rf && (fl & 1u)) || (row == rl && (fl & 2u));
+      if (shared) {
+        float *cp = a.carry + (c * 2 + (row == rf ? 0 : 1)) * (int64_t)a.K + k0;
+#pragma unroll
+        for (int r = 0; r < R; ++r)
+          if (col_ok[r]) st_vec<VW>(cp + r * Lg * VW, acc[r]);
+        return;
+      }
+    }
 #pragma unroll
     for (int r = 0; r < R; ++r)
       if (col_ok[r])

@@ -160,3 +160,23 @@ def test_randomized_configurations(seed):
         E = gs.sddmm(p, dg, A1, X).cpu().numpy()
         r2, T2 = oracle.sddmm(g.row_ind, g.col_ind, val, A1h, Xh)
         assert_within(E, r2, T2, what="sddmm")
+
+
+@pytest.mark.parametrize("agg", ["sum", "max", "mean"])
+@pytest.mark.parametrize("C", [0, 8, 64])
+def test_deterministic_spmm_bitwise_reproducible(agg, C):
+    """deterministic plans (no atomics: split-row partials summed in chunk order) give the
+    same bits on every run, and match the oracle."""
+    for g in graphs():
+        dg = upload(g)
+        K = 64
+        p = gs.plan(dg, K, force_chunk=C, deterministic=True)
+        X = torch.from_numpy(gen.features(70, g.N, K)).to(DEV)
+        outs = [gs.spmm(p, dg, X, agg=agg).cpu().numpy() for _ in range(3)]
+        assert all(np.array_equal(outs[0], o) for o in outs[1:])
+        ref, T = oracle.spmm_agg(g.row_ind, g.col_ind, g.val, X.cpu().numpy(), agg, M=g.M)
+        assert_within(outs[0], ref, T, tol=1e-5 if agg != "max" else 1e-6, what=f"det {agg}")
+        O = torch.from_numpy(outs[0].copy()).to(DEV)
+        if agg == "sum":  # beta = 1 through the fix-up pass as well
+            gs.spmm(p, dg, X, out=O, accumulate=True)
+            assert_within(O.cpu().numpy(), 2 * ref, 2 * T, what="det accumulate")
