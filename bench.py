@@ -355,8 +355,10 @@ def init_dist(world, local):
             dist.init_process_group("nccl", device_id=dev)
         else:
             dist.init_process_group(backend)
+        # torchrun pins OMP_NUM_THREADS=1; the host-side graph generator / reorder use
+        # OpenMP, so give each rank its share of the cores (read when gen/ first loads)
         ncores = os.cpu_count() or 1
-        os.environ.setdefault("OMP_NUM_THREADS", str(max(1, ncores // world)))
+        os.environ["OMP_NUM_THREADS"] = str(max(1, ncores // world))
     return dev
 
 

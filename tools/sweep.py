@@ -20,7 +20,7 @@ import numpy as np, torch
 import gen, oracle
 import paper_conf_ipps_fanwc23_b200 as gs
 from gen import configs
-res = {"lib": os.environ["GNN_LIB_PATH"], "dtype": DTYPE}
+res = {"lib": os.environ["GNN_LIB_PATH"], "dtype": DTYPE, "force_chunk": FCHUNK}
 # parity on a small graph
 g = gen.powerlaw_graph(4000, 200000, gamma=2.2, n_comm=5, seed=3)
 dg = gs.DeviceGraph.from_arrays(g.M, g.N, g.row_ind, g.col_ind, g.val, g.row_ptr)
@@ -51,7 +51,7 @@ for K, fvw in [(k, 0) for k in KS] + [(k, 8) for k in KS if VW8 and k % 8 == 0 a
     if DTYPE == "bf16":
         X = X.to(torch.bfloat16)
     O = torch.empty((g.M, K), device="cuda"); E = torch.empty(g.nnz, device="cuda")
-    p = gs.plan(dg, K, force_vw=fvw, feature_dtype=DTYPE)
+    p = gs.plan(dg, K, force_vw=fvw, feature_dtype=DTYPE, force_chunk=FCHUNK)
     ts, td = [], []
     for it in range(REPS + 2):
         flush.fill_(it)
@@ -74,10 +74,11 @@ def main():
     ap.add_argument("--vw8", action="store_true")
     ap.add_argument("--reorder", action="store_true")
     ap.add_argument("--dtype", default="f32", choices=["f32", "bf16"])
+    ap.add_argument("--force-chunk", type=int, default=0)
     ap.add_argument("libs", nargs="+")
     a = ap.parse_args()
     code = CHILD.replace("ROOT", repr(ROOT)).replace("WL", repr(a.workload)).replace(
-        "KS", repr([int(k) for k in a.K.split(",")])).replace("REPS", str(a.reps)).replace("VW8", str(a.vw8)).replace("REORDER", str(a.reorder)).replace("DTYPE", repr(a.dtype))
+        "KS", repr([int(k) for k in a.K.split(",")])).replace("REPS", str(a.reps)).replace("VW8", str(a.vw8)).replace("REORDER", str(a.reorder)).replace("DTYPE", repr(a.dtype)).replace("FCHUNK", str(a.force_chunk))
     for lib in a.libs:
         env = dict(os.environ, GNN_LIB_PATH=os.path.abspath(lib))
         r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
