@@ -239,9 +239,16 @@ GNN_API gnn_status_t gnn_permute_rows(const float *X, int64_t ldx, int64_t n, in
  * arrays (if upload_graph) and X from host memory into the caller's device workspace,
  * builds the plan (GPU plan kernel), runs SpMM (O = S X, if O_host) and SDDMM
  * (S_O[i] = v_i <X_r, X_c>, i.e. A1 = A2T = X, if out_host), and copies O (M x K, pitch K)
- * and S_O (nnz) back.  Everything is enqueued on `stream` and returns without waiting:
- * synchronise the stream before reading O_host / out_host or reusing X_host (pinned host
- * memory gives asynchronous DMA; pageable memory works but copies synchronously).
+ * and S_O (nnz) back.  Everything is enqueued asynchronously and the call returns without
+ * waiting; `stream` is ordered after every copy of the call, so synchronise it before
+ * reading O_host / out_host or reusing X_host (pinned host memory gives asynchronous DMA;
+ * pageable memory works but copies synchronously).  Internally the plan's chunks are cut
+ * into pieces (about one per 4 Mi nonzeros, at most 32; env GNN_HOST_PIECES overrides):
+ * ColInd/Value of later pieces upload on a copy-in stream while earlier pieces compute
+ * (alternating between `stream` and a second compute stream) and finished O rows / S_O
+ * values download on a copy-out stream, so the call costs about max(upload, compute,
+ * download) instead of their sum.  Deterministic plans run as one piece.  Reads the host
+ * row_ind to find the rows each piece completes.
  * graph_host: square (M == N), row_base 0, host pointers (row_ptr unused).  fp32 only.
  * upload_graph = 0 reuses the graph already in this workspace from an earlier call (the
  * graph's offsets do not depend on K, so one workspace sized for the largest K serves all).

@@ -51,6 +51,8 @@ struct SparseArgs {
   int32_t vecs;
   int32_t accum;  // 1: O += S A (beta = 1), rows without nonzeros untouched
   float *carry;   // deterministic: split-row partials [chunk][first|last][K] (no atomics)
+  int64_t c_begin, c_end;  // chunk range of this launch (default [0, num_chunks)); the
+                           // pipelined host path launches a plan piece by piece
 };
 
 // Occupancy (active blocks / SM) of the SpMM kernel for a feature width/lane count;
@@ -61,6 +63,16 @@ int spmm_active_blocks_per_sm(int dtype, int vw, int lanes, int vecs, int warps_
 gnn_status_t check_common(const Plan *p, const gnn_graph_t *g, const char *who);
 int effective_vws(int vws, const gnn_graph_t *g, const void *extra);
 SparseArgs make_args(const Plan *p, const gnn_graph_t *g);
+
+// Launchers (spmm.cu / sddmm.cu); c0 < 0 = every chunk of the plan, else chunks [c0, c1).
+gnn_status_t launch_spmm(const Plan *p, const gnn_graph_t *g, const void *A, int64_t lda,
+                         float *O, int64_t ldo, gnn_stream_t stream, int dtype, int agg_api,
+                         int accumulate, const char *who, int64_t c0, int64_t c1);
+gnn_status_t launch_spmm_prezero(const Plan *p, const gnn_graph_t *g, float *O, int64_t ldo,
+                                 gnn_stream_t stream);
+gnn_status_t launch_sddmm(const Plan *p, const gnn_graph_t *g, const void *A1, int64_t lda1,
+                          const void *A2T, int64_t lda2, float *out, gnn_stream_t stream,
+                          int dtype, const char *who, int64_t c0, int64_t c1);
 
 // Valid warps_per_block range; block size = 32 * wpb <= kMaxThreads.
 constexpr int kMaxThreads = 512;

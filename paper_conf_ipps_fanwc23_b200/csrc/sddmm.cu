@@ -16,9 +16,10 @@
 #include "sddmm_kernel.cuh"
 
 namespace gnn {
-static gnn_status_t launch_sddmm(const Plan *p, const gnn_graph_t *g, const void *A1,
-                                 int64_t lda1, const void *A2T, int64_t lda2, float *out,
-                                 gnn_stream_t stream, int dtype, const char *who) {
+// c0 < 0: the whole plan; else chunks [c0, c1) only (the pipelined host path).
+gnn_status_t launch_sddmm(const Plan *p, const gnn_graph_t *g, const void *A1, int64_t lda1,
+                          const void *A2T, int64_t lda2, float *out, gnn_stream_t stream,
+                          int dtype, const char *who, int64_t c0, int64_t c1) {
   if (gnn_status_t st = check_common(p, g, who)) return st;
   const gnn_plan_info_t &in = p->info;
   if (in.feature_dtype != dtype)
@@ -40,11 +41,19 @@ static gnn_status_t launch_sddmm(const Plan *p, const gnn_graph_t *g, const void
   if (!f)
     return fail(GNN_ERR_UNSUPPORTED, "%s: K=%d needs %d slices (max 4 at vw=%d)", who, K,
                 in.slices, VW);
-  const SparseArgs a = make_args(p, g);
+  SparseArgs a = make_args(p, g);
+  if (c0 >= 0) {
+    if (c1 < c0 || c1 > a.num_chunks)
+      return fail(GNN_ERR_INVALID_ARG, "%s: bad chunk range [%lld, %lld)", who, (long long)c0,
+                  (long long)c1);
+    if (c1 == c0) return GNN_OK;
+    a.c_begin = c0;
+    a.c_end = c1;
+  }
   const int threads = in.warps_per_block * 32;
   const int lg = sddmm_group_lanes(V, in.slices);
   const int64_t per_block = (int64_t)(32 / lg) * in.warps_per_block;
-  const int64_t blocks = (a.num_chunks + per_block - 1) / per_block;
+  const int64_t blocks = (a.c_end - a.c_begin + per_block - 1) / per_block;
   const size_t smem = (size_t)in.warps_per_block *
                       sddmm_tile_bytes_per_warp(lg, sddmm_effective_vws(V, in.slices, vws));
   if (smem > 48 * 1024) {
@@ -63,7 +72,7 @@ extern "C" GNN_API gnn_status_t gnn_sddmm(gnn_plan_t plan, const gnn_graph_t *g,
                                           const float *A1, int64_t lda1, const float *A2T,
                                           int64_t lda2, float *out, gnn_stream_t stream) {
   return launch_sddmm(reinterpret_cast<const Plan *>(plan), g, A1, lda1, A2T, lda2, out, stream,
-                      GNN_F32, "gnn_sddmm");
+                      GNN_F32, "gnn_sddmm", -1, 0);
 }
 
 extern "C" GNN_API gnn_status_t gnn_sddmm_bf16(gnn_plan_t plan, const gnn_graph_t *g,
@@ -71,5 +80,5 @@ extern "C" GNN_API gnn_status_t gnn_sddmm_bf16(gnn_plan_t plan, const gnn_graph_
                                                const uint16_t *A2T, int64_t lda2, float *out,
                                                gnn_stream_t stream) {
   return launch_sddmm(reinterpret_cast<const Plan *>(plan), g, A1, lda1, A2T, lda2, out, stream,
-                      GNN_BF16, "gnn_sddmm_bf16");
+                      GNN_BF16, "gnn_sddmm_bf16", -1, 0);
 }

@@ -94,8 +94,9 @@ __global__ void __launch_bounds__(kMaxThreads, (SddmmShape<VW, L, SMAX>::minb))
   const int lane = threadIdx.x & 31;
   const int g = lane / Lg;
   const int l = lane & (Lg - 1);
-  const int64_t c = ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * G + g;
-  const bool item_ok = c < a.num_chunks;
+  const int64_t c =
+      a.c_begin + ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * G + g;
+  const bool item_ok = c < a.c_end;
   if (!__any_sync(kFull, item_ok)) return;
   const int64_t cs = c * a.chunk;
   const int n = item_ok ? (int)(min(cs + (int64_t)a.chunk, a.nnz) - cs) : 0;

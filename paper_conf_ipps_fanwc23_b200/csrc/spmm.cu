@@ -33,9 +33,9 @@ namespace gnn {
 template <int VW>
 __global__ void spmm_prezero_kernel(const SparseArgs a, float *__restrict__ O,
                                     const int64_t ldo, const float init) {
-  const int64_t c = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t c = a.c_begin + (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5);
   const int lane = threadIdx.x & 31;
-  if (c >= a.num_chunks) return;
+  if (c >= a.c_end) return;
   const uint32_t fl = a.flags[c];
   if (!(fl & 2u)) return;
   const int32_t rf = a.row_first[c], rl = a.row_last[c];
@@ -176,6 +176,8 @@ SparseArgs make_args(const Plan *p, const gnn_graph_t *g) {
   a.vecs = p->info.vecs;
   a.accum = 0;
   a.carry = nullptr;
+  a.c_begin = 0;
+  a.c_end = a.num_chunks;
   return a;
 }
 
@@ -184,9 +186,12 @@ SparseArgs make_args(const Plan *p, const gnn_graph_t *g) {
 using namespace gnn;
 
 namespace gnn {
-static gnn_status_t launch_spmm(const Plan *p, const gnn_graph_t *g, const void *A, int64_t lda,
-                                float *O, int64_t ldo, gnn_stream_t stream, int dtype,
-                                int agg_api, int accumulate, const char *who) {
+// c0 < 0: the whole plan; else chunks [c0, c1) only (sum, overwrite, atomic plans: the
+// pipelined host path), without the pre-zero pass: the caller runs launch_spmm_prezero
+// over the whole plan first, so ranges may then run concurrently.
+gnn_status_t launch_spmm(const Plan *p, const gnn_graph_t *g, const void *A, int64_t lda,
+                         float *O, int64_t ldo, gnn_stream_t stream, int dtype, int agg_api,
+                         int accumulate, const char *who, int64_t c0, int64_t c1) {
   if (gnn_status_t st = check_common(p, g, who)) return st;
   const gnn_plan_info_t &in = p->info;
   if (in.feature_dtype != dtype)
@@ -227,9 +232,18 @@ static gnn_status_t launch_spmm(const Plan *p, const gnn_graph_t *g, const void 
   SparseArgs a = make_args(p, g);
   a.accum = accumulate;
   a.carry = p->carry;
+  if (c0 >= 0) {
+    if (c1 < c0 || c1 > a.num_chunks || a.carry || agg_api != GNN_AGG_SUM)
+      return fail(GNN_ERR_INVALID_ARG, "%s: bad chunk range [%lld, %lld)", who, (long long)c0,
+                  (long long)c1);
+    if (c1 == c0) return GNN_OK;
+    a.c_begin = c0;
+    a.c_end = c1;
+  }
+  const int64_t nch = a.c_end - a.c_begin;
   const int threads = in.warps_per_block * 32;
-  if (!accumulate && !a.carry) {
-    const int64_t blocks = (a.num_chunks * 32 + 255) / 256;
+  if (!accumulate && !a.carry && c0 < 0) {
+    const int64_t blocks = (nch * 32 + 255) / 256;
     const float init = agg == kAggMax ? -INFINITY : agg == kAggMin ? INFINITY : 0.f;
     switch (VO) {
       case 1: spmm_prezero_kernel<1><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, init); break;
@@ -243,7 +257,9 @@ static gnn_status_t launch_spmm(const Plan *p, const gnn_graph_t *g, const void 
     cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return cuda_fail(e, "gnn_spmm smem attribute");
   }
-  f<<<(unsigned)in.num_blocks, threads, smem, s>>>(a, A, lda, O, ldo);
+  const int64_t per_block = (int64_t)(32 / in.lanes) * in.warps_per_block;  // items / block
+  const int64_t grid = (nch * in.slices + per_block - 1) / per_block;
+  f<<<(unsigned)grid, threads, smem, s>>>(a, A, lda, O, ldo);
   if (a.carry) {
     const int64_t blocks = (a.num_chunks * 32 + 255) / 256;
     if (agg == kAggMax) spmm_fixup_kernel<1><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo);
@@ -262,18 +278,38 @@ static gnn_status_t launch_spmm(const Plan *p, const gnn_graph_t *g, const void 
 }
 }  // namespace gnn
 
+namespace gnn {
+gnn_status_t launch_spmm_prezero(const Plan *p, const gnn_graph_t *g, float *O, int64_t ldo,
+                                 gnn_stream_t stream) {
+  if (gnn_status_t st = check_common(p, g, "spmm prezero")) return st;
+  if (p->info.num_chunks == 0) return GNN_OK;
+  SparseArgs a = make_args(p, g);
+  const int VW = p->info.vw_feat, VO = VW < 8 ? VW : 8;
+  const int64_t blocks = (a.num_chunks * 32 + 255) / 256;
+  cudaStream_t s = (cudaStream_t)stream;
+  switch (VO) {
+    case 1: spmm_prezero_kernel<1><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, 0.f); break;
+    case 2: spmm_prezero_kernel<2><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, 0.f); break;
+    case 4: spmm_prezero_kernel<4><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, 0.f); break;
+    default: spmm_prezero_kernel<8><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, 0.f); break;
+  }
+  cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? GNN_OK : cuda_fail(e, "spmm prezero launch");
+}
+}  // namespace gnn
+
 extern "C" GNN_API gnn_status_t gnn_spmm(gnn_plan_t plan, const gnn_graph_t *g, const float *A,
                                          int64_t lda, float *O, int64_t ldo,
                                          gnn_stream_t stream) {
   return launch_spmm(reinterpret_cast<const Plan *>(plan), g, A, lda, O, ldo, stream, GNN_F32,
-                     GNN_AGG_SUM, 0, "gnn_spmm");
+                     GNN_AGG_SUM, 0, "gnn_spmm", -1, 0);
 }
 
 extern "C" GNN_API gnn_status_t gnn_spmm_bf16(gnn_plan_t plan, const gnn_graph_t *g,
                                               const uint16_t *A, int64_t lda, float *O,
                                               int64_t ldo, gnn_stream_t stream) {
   return launch_spmm(reinterpret_cast<const Plan *>(plan), g, A, lda, O, ldo, stream, GNN_BF16,
-                     GNN_AGG_SUM, 0, "gnn_spmm_bf16");
+                     GNN_AGG_SUM, 0, "gnn_spmm_bf16", -1, 0);
 }
 
 extern "C" GNN_API gnn_status_t gnn_spmm_ex(gnn_plan_t plan, const gnn_graph_t *g, const void *A,
@@ -281,5 +317,5 @@ extern "C" GNN_API gnn_status_t gnn_spmm_ex(gnn_plan_t plan, const gnn_graph_t *
                                             int32_t accumulate, gnn_stream_t stream) {
   const Plan *p = reinterpret_cast<const Plan *>(plan);
   const int dtype = p ? p->info.feature_dtype : GNN_F32;
-  return launch_spmm(p, g, A, lda, O, ldo, stream, dtype, agg, accumulate, "gnn_spmm_ex");
+  return launch_spmm(p, g, A, lda, O, ldo, stream, dtype, agg, accumulate, "gnn_spmm_ex", -1, 0);
 }

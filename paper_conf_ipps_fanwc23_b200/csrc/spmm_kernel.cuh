@@ -108,8 +108,9 @@ __global__ void __launch_bounds__(kMaxThreads, GNN_SPMM_MINB)
   const int lane = threadIdx.x & 31;
   const int g = lane / Lg;
   const int l = lane & (Lg - 1);
-  const int64_t item = ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * G + g;
-  const bool item_ok = item < a.num_chunks * a.slices;
+  const int64_t item =
+      a.c_begin * a.slices + ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * G + g;
+  const bool item_ok = item < a.c_end * a.slices;
   if (!__any_sync(kFull, item_ok)) return;  // warp-uniform exit
 
   int64_t c = 0;

@@ -499,3 +499,79 @@ def test_run_host_end_to_end_matches_oracle():
         assert_within(O.numpy(), ref, T, what=f"run_host spmm K={K}")
         r2, T2 = oracle.sddmm(g.row_ind, g.col_ind, g.val, X.numpy(), X.numpy())
         assert_within(E.numpy(), r2, T2, what=f"run_host sddmm K={K}")
+
+
+def _run_host_check(g, Ks, pieces, seed=900, opts=None):
+    """gnn_run_host with GNN_HOST_PIECES=pieces against the oracle everywhere."""
+    import os
+    old = os.environ.get("GNN_HOST_PIECES")
+    os.environ["GNN_HOST_PIECES"] = str(pieces)
+    try:
+        runner = gs.HostRunner(g.M, g.N, g.row_ind, g.col_ind, g.val, max(Ks), device=DEV,
+                               **(opts or {})).pin()
+        for j, K in enumerate(Ks):
+            X = torch.from_numpy(_x(seed + K, g.N, K)).pin_memory()
+            O = torch.full((g.M, K), float("nan")).pin_memory()
+            E = torch.full((g.nnz,), float("nan")).pin_memory()
+            runner.run(X, K, O, E, upload_graph=(j == 0))
+            torch.cuda.synchronize()
+            ref, T = oracle.spmm(g.row_ind, g.col_ind, g.val, X.numpy(), M=g.M)
+            assert_within(O.numpy(), ref, T, what=f"run_host pieces={pieces} spmm K={K}")
+            r2, T2 = oracle.sddmm(g.row_ind, g.col_ind, g.val, X.numpy(), X.numpy())
+            assert_within(E.numpy(), r2, T2, what=f"run_host pieces={pieces} sddmm K={K}")
+    finally:
+        if old is None:
+            del os.environ["GNN_HOST_PIECES"]
+        else:
+            os.environ["GNN_HOST_PIECES"] = old
+
+
+@pytest.mark.parametrize("pieces", [2, 3, 7, 32])
+def test_run_host_pipelined_pieces(pieces):
+    """The copy/compute pipeline of gnn_run_host (pieces of the plan's chunks on two
+    compute streams, O rows downloaded as they become final): every output element
+    matches the oracle for any piece count, including pieces whose boundaries fall
+    inside a row, before runs of empty rows and inside a hub row."""
+    g = configs.make_graph("C2")
+    _run_host_check(g, (32, 64, 256), pieces)
+    rng = np.random.default_rng(17)
+    M = 3000
+    rows = rng.integers(0, M, 60000)
+    rows = rows[(rows % 11) > 2]  # runs of empty rows
+    rows = np.concatenate([rows, np.full(20000, 1500), [0, M - 1]])  # hub + first/last row
+    cols = rng.integers(0, M, rows.size)
+    g2 = gen.from_coo(M, M, rows, cols, gen.uniform_values(5, rows.size))
+    _run_host_check(g2, (8, 32, 128), pieces)
+
+
+def test_run_host_pipelined_deterministic_and_no_values():
+    """Deterministic plans run unpipelined; a NULL value array means all ones."""
+    g = configs.make_graph("C2")
+    _run_host_check(g, (64,), 8, opts={"deterministic": 1})
+    g1 = gen.Graph(g.M, g.N, g.row_ptr, g.row_ind, g.col_ind, None)
+    _run_host_check(g1, (32, 128), 5)
+
+
+@pytest.mark.slow
+def test_run_host_full_size_sampled_parity():
+    """bench.py's e2e call at full C4 size (default piece count, graph uploaded by the
+    first K, reused by the second): sampled rows / edges against the oracle."""
+    g = configs.make_graph("C4")
+    runner = gs.HostRunner(g.M, g.N, g.row_ind, g.col_ind, g.val, 256, device=DEV).pin()
+    rows = _sampled_rows(g, 200, 3)
+    edges = np.unique(np.r_[np.random.default_rng(4).choice(g.nnz, 5000, replace=False),
+                            g.row_ptr[rows[:50]], g.nnz - 1])
+    for j, K in enumerate((32, 256)):
+        X = configs.make_features("C4", g.N, K)
+        O = torch.empty((g.M, K)).pin_memory()
+        E = torch.empty(g.nnz).pin_memory()
+        runner.run(torch.from_numpy(X).pin_memory(), K, O, E, upload_graph=(j == 0))
+        torch.cuda.synchronize()
+        ref, T = oracle.spmm_rows(g, X, rows)
+        assert_within(O.numpy()[rows], ref, T, what=f"run_host C4 spmm K={K}")
+        r2 = np.empty(edges.size)
+        T2 = np.empty(edges.size)
+        for i, e in enumerate(edges):
+            a, b = oracle.sddmm(g.row_ind, g.col_ind, g.val, X, X, i0=int(e), i1=int(e) + 1)
+            r2[i], T2[i] = a[0], b[0]
+        assert_within(E.numpy()[edges], r2, T2, what=f"run_host C4 sddmm K={K}")
