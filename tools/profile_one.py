@@ -22,6 +22,7 @@ def main():
     ap.add_argument("--reps", type=int, default=1)
     ap.add_argument("--scale", type=float, default=1.0)
     ap.add_argument("--reorder", action="store_true")
+    ap.add_argument("--dtype", default="f32", choices=["f32", "bf16"])
     a = ap.parse_args()
     g = configs.make_graph(a.workload, a.scale)
     perm = None
@@ -35,10 +36,12 @@ def main():
         X = torch.from_numpy(configs.make_features(a.workload, g.N, K)).cuda()
         if perm is not None:
             X = gs.permute_rows(X, torch.from_numpy(perm))
+        if a.dtype == "bf16":
+            X = X.to(torch.bfloat16)
         O = torch.empty((g.M, K), device="cuda")
         E = torch.empty(g.nnz, device="cuda")
         for _ in range(a.reps):
-            p = gs.plan(dg, K)
+            p = gs.plan(dg, K, feature_dtype=gs.GNN_BF16 if a.dtype == "bf16" else gs.GNN_F32)
             gs.spmm(p, dg, X, out=O)
             gs.sddmm(p, dg, X, X, out=E)
         torch.cuda.synchronize()
