@@ -11,6 +11,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <type_traits>
+
 namespace gnn {
 
 constexpr unsigned kFull = 0xffffffffu;
@@ -375,4 +377,179 @@ struct SparseTiles {
   }
 };
 
+
+// ------------------------------------------------- TMA-staged sparse tiles ----
+// ncu on the cp.async ring (C4, K = 32) showed the LDGSTS copies costing ~27 L1 data-pipe
+// wavefronts per warp instruction -- ~40% of the wavefronts of a data pipe running at
+// 70-83% of its peak, the busiest unit of both kernels.  With vw_sparse = 4 (16-byte
+// aligned chunk bases) the tiles can instead be filled by the TMA unit: one bulk copy
+// (cp.async.bulk, global -> shared, completion counted on a per-warp mbarrier) per
+// (group, array) and tile, issued by one lane each, which bypasses the LSU data pipe.
+// Tile T = L * 4 * TM nonzeros per group (TM: tile multiplier), stride T + 4 words
+// (bank padding, keeps 16-byte destination alignment).  Entries past the chunk end are
+// left stale (the kernels never use them); a tail that is not a multiple of 16 bytes is
+// copied with plain loads by the issuing lane.
+// MEASURED SLOWER (profiles/r01_sweep31_tma_tiles.txt, C4 GCR): SpMM K=32 0.93 -> 1.16 ms,
+// SDDMM 1.06 -> 1.24 ms at TM = 1, no gain at K = 256 either: the many small (64-256 B)
+// bulk copies and the mbarrier round trip one tile ahead cost more than the LDGSTS
+// wavefronts they remove, so the data pipe is busy but not the binding limit (the L2 ->
+// SM return path is).  Kept as an opt-in build (-DGNN_TMA_TILES=1) for that record.
+#ifndef GNN_TMA_TILES
+#define GNN_TMA_TILES 0  // measured slower (profiles/r01_sweep31_tma_tiles.txt): opt-in
+#endif
+#ifndef GNN_TILE_MULT
+#define GNN_TILE_MULT 1
+#endif
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_fence_init() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // (a cluster-scope fence would emit CCTL.IVALL: an L1 flush per warp)
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t *bar, uint32_t tx) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
+               "r"(tx)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait_parity(uint64_t *bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred P1;\n"
+      "LAB_WAIT:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
+      "@P1 bra DONE;\n\t"
+      "bra LAB_WAIT;\n"
+      "DONE:\n\t}" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes,
+                                         uint64_t *bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::
+          "r"(smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
+template <int L, int TM>
+struct TmaTiles {
+  static constexpr int G = 32 / L;
+  static constexpr int T = L * 4 * TM;       // nonzeros per tile per lane group
+  static constexpr int STRIDE = T + 4;       // words per group
+  static constexpr int WORDS = G * STRIDE;   // words per array per stage
+  static constexpr int SLOTS = (3 * G + 31) / 32;  // copies issued per lane per tile
+  static constexpr int WARP_WORDS = 4 + 2 * 3 * WORDS;  // 2 mbarriers + ring
+  static constexpr int BYTES_PER_WARP = WARP_WORDS * 4;
+  int32_t *w;
+  const int32_t *src[SLOTS];  // this lane's copy slots: source of (array, group) at tile 0
+  int doff[SLOTS];            // ... destination (words into the warp region, stage 0)
+  int n[SLOTS];               // ... valid entries of that group's chunk (0: no copy)
+  __device__ __forceinline__ uint64_t *bar(int st) const { return reinterpret_cast<uint64_t *>(w) + st; }
+  __device__ __forceinline__ int32_t *arr(int st, int a, int g) const {
+    return w + 4 + (st * 3 + a) * WORDS + g * STRIDE;
+  }
+  __device__ __forceinline__ int32_t *rows(int st, int g) const { return arr(st, 0, g); }
+  __device__ __forceinline__ int32_t *cols(int st, int g) const { return arr(st, 1, g); }
+  __device__ __forceinline__ float *vals(int st, int g) const {
+    return reinterpret_cast<float *>(arr(st, 2, g));
+  }
+  // chunk_of(gg, &cs, &n): first nonzero and count of group gg's chunk (n = 0: none).
+  template <typename ChunkOf>
+  __device__ __forceinline__ void init(int32_t *warp_smem, int lane, const int32_t *ri0,
+                                       const int32_t *ci0, const float *vi0, ChunkOf chunk_of) {
+    w = warp_smem;
+#pragma unroll
+    for (int q = 0; q < SLOTS; ++q) {
+      const int j = lane + 32 * q;
+      const int a = j / G, gg = j % G;
+      n[q] = 0;
+      src[q] = ri0;
+      doff[q] = 4 + ((a < 3 ? a : 0) * WORDS + gg * STRIDE);
+      if (j < 3 * G && (a != 2 || vi0)) {
+        int64_t cs;
+        int cnt;
+        chunk_of(gg, cs, cnt);
+        n[q] = cnt;
+        src[q] = (a == 0 ? ri0 : a == 1 ? ci0 : reinterpret_cast<const int32_t *>(vi0)) + cs;
+      }
+    }
+    if (lane == 0) {
+      mbar_init(bar(0), 1);
+      mbar_init(bar(1), 1);
+      mbar_fence_init();
+    }
+    __syncwarp();
+  }
+  // fill stage st with entries [tb, tb + T) of every group's chunk
+  __device__ __forceinline__ void issue(int st, int tb, int lane) const {
+    uint32_t bulk[SLOTS], mine = 0;
+#pragma unroll
+    for (int q = 0; q < SLOTS; ++q) {
+      int cnt = n[q] - tb;
+      cnt = cnt < 0 ? 0 : (cnt > T ? T : cnt);
+      bulk[q] = (uint32_t)(cnt * 4) & ~15u;
+      mine += bulk[q];
+    }
+    const uint32_t total = __reduce_add_sync(kFull, mine);
+    if (lane == 0) mbar_arrive_expect_tx(bar(st), total);
+    const int soff = st * 3 * WORDS;
+#pragma unroll
+    for (int q = 0; q < SLOTS; ++q) {
+      int32_t *d = w + doff[q] + soff;
+      if (bulk[q]) bulk_g2s(d, src[q] + tb, bulk[q], bar(st));
+      int cnt = n[q] - tb;
+      cnt = cnt > T ? T : cnt;
+      for (int e = (int)(bulk[q] >> 2); e < cnt; ++e) d[e] = __ldg(src[q] + tb + e);
+    }
+  }
+  __device__ __forceinline__ void skip() const {}
+  __device__ __forceinline__ void wait(int st, int t) const {
+    mbar_wait_parity(bar(st), (uint32_t)((t >> 1) & 1));
+  }
+};
+
+// The cp.async ring behind the same interface (vw_sparse < 4: misaligned sub-views,
+// small chunks).
+template <int L, int VWS>
+struct AsyncTiles : SparseTiles<L, VWS> {
+  using Base = SparseTiles<L, VWS>;
+  int g, l, cnt;
+  const int32_t *ri, *ci;
+  const float *vi;
+  template <typename ChunkOf>
+  __device__ __forceinline__ void init(int32_t *warp_smem, int lane, const int32_t *ri0,
+                                       const int32_t *ci0, const float *vi0, ChunkOf chunk_of) {
+    this->w = warp_smem;
+    g = lane / L;
+    l = lane & (L - 1);
+    int64_t cs;
+    chunk_of(g, cs, cnt);
+    ri = ri0 + cs;
+    ci = ci0 + cs;
+    vi = vi0 ? vi0 + cs : nullptr;
+  }
+  __device__ __forceinline__ void issue(int st, int tb, int) const {
+    Base::load(st, g, l, ri, ci, vi, tb, cnt);
+    cp_async_commit();
+  }
+  __device__ __forceinline__ void skip() const { cp_async_commit(); }  // (empty group)
+  __device__ __forceinline__ void wait(int, int) const {
+    cp_async_wait<1>();  // all but the most recent group: tile t has landed
+  }
+};
+
+template <int L, int VWS>
+using TilesFor = typename std::conditional<(VWS == 4 && GNN_TMA_TILES), TmaTiles<L, GNN_TILE_MULT>,
+                                           AsyncTiles<L, VWS>>::type;
+
+// dynamic shared memory per warp of the tiles of a lane-group width L at vw_sparse vws
+inline int tile_bytes_per_warp(int L, int vws) {
+  if (vws == 4 && GNN_TMA_TILES) return (4 + 2 * 3 * (32 / L) * (L * 4 * GNN_TILE_MULT + 4)) * 4;
+  return 2 * 3 * (32 / L) * (L * vws + 4) * 4;
+}
 }  // namespace gnn

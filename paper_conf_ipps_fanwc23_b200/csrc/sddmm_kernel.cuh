@@ -87,7 +87,8 @@ __global__ void __launch_bounds__(kMaxThreads, (SddmmShape<VW, L, SMAX>::minb))
   using Sh = SddmmShape<VW, L, SMAX>;
   constexpr int R = Sh::R, Lg = Sh::Lg;
   constexpr int G = 32 / Lg;
-  constexpr int T = Lg * VWS;
+  using Tiles = TilesFor<Lg, VWS>;
+  constexpr int T = Tiles::T;
   constexpr int U0 = Sh::depth > VWS ? Sh::depth : VWS;
   constexpr int U = U0 < T ? U0 : T;
   static_assert(T % U == 0 && U % VWS == 0, "tile / prefetch shape");
@@ -114,16 +115,27 @@ __global__ void __launch_bounds__(kMaxThreads, (SddmmShape<VW, L, SMAX>::minb))
     for (int r = 0; r < R; ++r) a1[sl][r].zero();
   }
 
-  const int32_t *__restrict__ ri = a.row_ind + cs;
-  const int32_t *__restrict__ ci = a.col_ind + cs;
   const float *__restrict__ vi = a.val ? a.val + cs : nullptr;
   float *__restrict__ oc = out + cs;
-  // sparse tiles: per-warp double-buffered shared-memory ring filled with cp.async
+  // sparse tiles: per-warp double-buffered shared-memory ring (TMA bulk copies, or
+  // cp.async for narrow sparse vectors), one tile ahead of use
   extern __shared__ int32_t gnn_smem[];
-  using Tiles = SparseTiles<Lg, VWS>;
-  const Tiles tiles{gnn_smem + (threadIdx.x >> 5) * Tiles::WARP_WORDS};
-  tiles.load(0, g, l, ri, ci, vi, 0, n);
-  cp_async_commit();
+  Tiles tiles;
+  {
+    const int64_t c0 =
+        a.c_begin + ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * G;
+    tiles.init(gnn_smem + (threadIdx.x >> 5) * Tiles::WARP_WORDS, lane, a.row_ind, a.col_ind,
+               a.val, [&](int gg, int64_t &cs_, int &n_) {
+                 const int64_t cc = c0 + gg;
+                 cs_ = 0;
+                 n_ = 0;
+                 if (cc < a.c_end) {
+                   cs_ = cc * a.chunk;
+                   n_ = (int)(min(cs_ + (int64_t)a.chunk, a.nnz) - cs_);
+                 }
+               });
+  }
+  tiles.issue(0, 0, lane);
 
   auto load_a1_slice = [&](int sl, int32_t row) {
     const char *base = reinterpret_cast<const char *>(A1) +
@@ -141,9 +153,9 @@ __global__ void __launch_bounds__(kMaxThreads, (SddmmShape<VW, L, SMAX>::minb))
     const int tb = t * T;
     const int st = t & 1;
     __syncwarp();  // every lane is done with the stage the next copy overwrites
-    if (t + 1 < ntiles) tiles.load(st ^ 1, g, l, ri, ci, vi, tb + T, n);
-    cp_async_commit();
-    cp_async_wait<1>();
+    if (t + 1 < ntiles) tiles.issue(st ^ 1, tb + T, lane);
+    else tiles.skip();
+    tiles.wait(st, t);  // tile t has landed
     __syncwarp();
     const int32_t *s_row = tiles.rows(st, g);
     const int32_t *s_col = tiles.cols(st, g);
@@ -246,9 +258,7 @@ SddmmFn pick_sddmm_f32(int vw, int V, int vws, int S);
 SddmmFn pick_sddmm_bf16(int vw, int V, int vws, int S);
 
 // dynamic shared memory per warp of the instantiation with Lg lanes per dot product
-inline int sddmm_tile_bytes_per_warp(int lg, int vws) {
-  return 2 * 3 * (32 / lg) * (lg * vws + 4) * 4;
-}
+inline int sddmm_tile_bytes_per_warp(int lg, int vws) { return tile_bytes_per_warp(lg, vws); }
 // the vw_sparse the dispatcher actually instantiates (a batch must cover whole vectors)
 inline int sddmm_effective_vws(int V, int S, int vws) {
   const int r = S > 1 ? 2 : ((V >= GNN_SDDMM_R2_FROM && V >= 2) ? 2 : 1);

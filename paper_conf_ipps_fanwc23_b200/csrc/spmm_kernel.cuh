@@ -100,7 +100,8 @@ __global__ void __launch_bounds__(kMaxThreads, GNN_SPMM_MINB)
   constexpr int ES = TF::bytes;
   constexpr int Lg = L;
   constexpr int G = 32 / Lg;
-  constexpr int T = Lg * VWS;  // nonzeros per tile per group
+  using Tiles = TilesFor<L, VWS>;
+  constexpr int T = Tiles::T;  // nonzeros per tile per group
   // U nonzeros per batch: FeatDepth vectors in flight per lane, whole sparse vectors
   constexpr int D = FeatDepth<TF, VW, L, R>::value / R;
   constexpr int U = D > T ? T : (D < VWS ? VWS : D);
@@ -175,25 +176,36 @@ __global__ void __launch_bounds__(kMaxThreads, GNN_SPMM_MINB)
     for (int v = 0; v < VW; ++v) acc[r][v] = agg_init<AGG>();
   int32_t cur = -1;
 
-  const int32_t *__restrict__ ri = a.row_ind + cs;
-  const int32_t *__restrict__ ci = a.col_ind + cs;
   const float *__restrict__ vi = a.val ? a.val + cs : nullptr;
-  // sparse tiles: per-warp double-buffered shared-memory ring filled with cp.async
+  // sparse tiles: per-warp double-buffered shared-memory ring (TMA bulk copies, or
+  // cp.async for narrow sparse vectors), one tile ahead of use
   extern __shared__ int32_t gnn_smem[];
-  using Tiles = SparseTiles<L, VWS>;
-  const Tiles tiles{gnn_smem + (threadIdx.x >> 5) * Tiles::WARP_WORDS};
-  tiles.load(0, g, l, ri, ci, vi, 0, n);
-  cp_async_commit();
+  Tiles tiles;
+  {
+    const int64_t item0 =
+        a.c_begin * a.slices + ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * G;
+    tiles.init(gnn_smem + (threadIdx.x >> 5) * Tiles::WARP_WORDS, lane, a.row_ind, a.col_ind,
+               a.val, [&](int gg, int64_t &cs_, int &n_) {
+                 const int64_t it = item0 + gg;
+                 cs_ = 0;
+                 n_ = 0;
+                 if (it < a.c_end * a.slices) {
+                   cs_ = (it / a.slices) * a.chunk;
+                   n_ = (int)(min(cs_ + (int64_t)a.chunk, a.nnz) - cs_);
+                 }
+               });
+  }
+  tiles.issue(0, 0, lane);
 
   const int ntiles = (a.chunk + T - 1) / T;  // warp-uniform trip count
   for (int t = 0; t < ntiles; ++t) {
     const int tb = t * T;
     const int st = t & 1;
     __syncwarp();  // every lane is done with the stage the next copy overwrites
-    if (t + 1 < ntiles) tiles.load(st ^ 1, g, l, ri, ci, vi, tb + T, n);
-    cp_async_commit();
-    cp_async_wait<1>();  // this lane's copies of tile t have landed
-    __syncwarp();        // ... and every other lane's
+    if (t + 1 < ntiles) tiles.issue(st ^ 1, tb + T, lane);
+    else tiles.skip();
+    tiles.wait(st, t);  // tile t has landed
+    __syncwarp();       // (and the plain-load tails written by other lanes are visible)
     const int32_t *s_row = tiles.rows(st, g);
     const int32_t *s_col = tiles.cols(st, g);
     const float *s_val = tiles.vals(st, g);
@@ -321,10 +333,7 @@ SpmmFn spmm_pick_l(int L, int R, int vws) {
 }
 
 // dynamic shared memory of spmm_kernel<.., L, .., VWS> per warp
-inline int spmm_tile_bytes_per_warp(int L, int vws) {
-  const int T = L * vws;
-  return 2 * 3 * (32 / L) * (T + 4) * 4;
-}
+inline int spmm_tile_bytes_per_warp(int L, int vws) { return tile_bytes_per_warp(L, vws); }
 
 template <typename TF, int AGG>
 SpmmFn spmm_pick_vw(int vw, int L, int R, int vws);
