@@ -260,6 +260,24 @@ GNN_API gnn_status_t gnn_run_host(const gnn_graph_t *graph_host, int32_t upload_
                                   float *out_host, const gnn_plan_opts_t *opts, void *workspace,
                                   size_t ws_bytes, gnn_stream_t stream);
 
+/* gnn_run_host for nk feature widths K[0..nk) on one graph in ONE pipelined call
+ * (1 <= nk <= 16): X_host[k] (N x K[k]), O_host[k] (M x K[k], or O_host / O_host[k] NULL
+ * to skip that SpMM), out_host[k] (nnz, or NULL to skip that SDDMM).  The graph uploads
+ * with the first width; X_host[k+1] uploads and every download overlap the kernels of
+ * earlier widths, so the call costs about max(total upload, total compute, total
+ * download).  Each width has its own plan and workspace region, so no width waits for
+ * an earlier width's download.  Same ordering, ownership and error rules as gnn_run_host
+ * (gnn_run_host is this call with nk = 1).  workspace:
+ * gnn_run_host_multi_workspace_bytes(M, N, nnz, nk, K, opts) bytes ((size_t)-1 on
+ * invalid arguments), 256-B aligned, device. */
+GNN_API size_t gnn_run_host_multi_workspace_bytes(int64_t M, int64_t N, int64_t nnz, int32_t nk,
+                                                  const int32_t *K, const gnn_plan_opts_t *opts);
+GNN_API gnn_status_t gnn_run_host_multi(const gnn_graph_t *graph_host, int32_t upload_graph,
+                                        int32_t nk, const int32_t *K,
+                                        const float *const *X_host, float *const *O_host,
+                                        float *const *out_host, const gnn_plan_opts_t *opts,
+                                        void *workspace, size_t ws_bytes, gnn_stream_t stream);
+
 /* ----------------------------------------------------------- measurement --- */
 /* Roofline probe (not part of the method): gathers rows X[idx[i]][0:K] for i in [0, n)
  * with the same 256-bit row loads the kernels use and no other work (sums are folded

@@ -69,7 +69,8 @@ EXPORTS = ["gnn_plan_workspace_bytes", "gnn_plan_create", "gnn_plan_info", "gnn_
            "gnn_spmm_ex", "gnn_transpose_workspace_bytes", "gnn_transpose",
            "gnn_shard_rows", "gnn_shard_edges", "gnn_split_col_blocks",
            "gnn_reorder_gcr", "gnn_permute_graph", "gnn_permute_rows",
-           "gnn_probe_gather", "gnn_run_host_workspace_bytes", "gnn_run_host", "gnn_csr_to_coo", "gnn_validate", "gnn_last_error",
+           "gnn_probe_gather", "gnn_run_host_workspace_bytes", "gnn_run_host",
+           "gnn_run_host_multi_workspace_bytes", "gnn_run_host_multi", "gnn_csr_to_coo", "gnn_validate", "gnn_last_error",
            "gnn_version"]
 
 _lib = None
@@ -107,6 +108,12 @@ def lib():
     if hasattr(L, "gnn_run_host"):
         L.gnn_run_host_workspace_bytes.argtypes = [i64, i64, i64, i32, P(PlanOpts)]
         L.gnn_run_host_workspace_bytes.restype = ctypes.c_size_t
+        if hasattr(L, "gnn_run_host_multi"):  # (GNN_LIB_PATH may point at an older build)
+            L.gnn_run_host_multi_workspace_bytes.argtypes = [i64, i64, i64, i32, vp,
+                                                             P(PlanOpts)]
+            L.gnn_run_host_multi_workspace_bytes.restype = ctypes.c_size_t
+            L.gnn_run_host_multi.argtypes = [P(_Graph), i32, i32, vp, vp, vp, vp, P(PlanOpts),
+                                             vp, ctypes.c_size_t, vp]
         L.gnn_run_host.argtypes = [P(_Graph), i32, vp, i32, vp, vp, P(PlanOpts), vp,
                                    ctypes.c_size_t, vp]
     if hasattr(L, "gnn_split_col_blocks"):
@@ -125,7 +132,7 @@ def lib():
               "gnn_shard_rows", "gnn_shard_edges", "gnn_csr_to_coo", "gnn_validate",
               "gnn_reorder_gcr", "gnn_permute_graph", "gnn_permute_rows", "gnn_probe_gather",
               "gnn_spmm_bf16", "gnn_sddmm_bf16", "gnn_spmm_ex", "gnn_transpose",
-              "gnn_split_col_blocks", "gnn_run_host"):
+              "gnn_split_col_blocks", "gnn_run_host", "gnn_run_host_multi"):
         if hasattr(L, f):
             getattr(L, f).restype = st
     _lib = L
@@ -447,10 +454,11 @@ def probe_gather(X: torch.Tensor, idx: torch.Tensor, sink: torch.Tensor | None =
 
 class HostRunner:
     """gnn_run_host: the end-to-end call on HOST buffers.  Holds the device workspace
-    (sized for the largest K) and the host graph descriptor; run() enqueues H2D copies,
-    plan, SpMM, SDDMM and D2H copies on the current stream (synchronise before reading)."""
+    (sized for the largest K, and for run_multi over Ks if given) and the host graph
+    descriptor; run() / run_multi() enqueue H2D copies, plans, SpMM, SDDMM and D2H copies
+    ordered on the current stream (synchronise before reading)."""
 
-    def __init__(self, M, N, row_ind, col_ind, val, Kmax, device="cuda", **opts):
+    def __init__(self, M, N, row_ind, col_ind, val, Kmax, device="cuda", Ks=None, **opts):
         self._keep = [np.ascontiguousarray(row_ind, np.int32),
                       np.ascontiguousarray(col_ind, np.int32),
                       None if val is None else np.ascontiguousarray(val, np.float32)]
@@ -460,6 +468,13 @@ class HostRunner:
                                                     ctypes.byref(self.opts))
         if nbytes == ctypes.c_size_t(-1).value:
             _check(GNN_ERR_INVALID_ARG)
+        if Ks is not None:
+            karr = (ctypes.c_int32 * len(Ks))(*Ks)
+            mb = lib().gnn_run_host_multi_workspace_bytes(self.M, self.N, self.nnz, len(Ks),
+                                                          karr, ctypes.byref(self.opts))
+            if mb == ctypes.c_size_t(-1).value:
+                _check(GNN_ERR_INVALID_ARG)
+            nbytes = max(int(nbytes), int(mb))
         self.ws = torch.empty(max(int(nbytes), 1), dtype=torch.uint8, device=device)
         self.ws_bytes = int(nbytes)
         self.desc = _Graph(self.M, self.N, self.nnz, None, self._keep[0].ctypes.data,
@@ -482,3 +497,22 @@ class HostRunner:
         _check(lib().gnn_run_host(ctypes.byref(self.desc), int(upload_graph), _ptr(X_host), K,
                                   _ptr(O_host), _ptr(out_host), ctypes.byref(self.opts),
                                   _ptr(self.ws), self.ws_bytes, _stream(stream)))
+
+    def run_multi(self, X_hosts, Ks, O_hosts=None, out_hosts=None, upload_graph=True,
+                  stream=None):
+        """gnn_run_host_multi: several feature widths on one graph in one pipelined call
+        (later X uploads and every download overlap the kernels of earlier widths)."""
+        n = len(Ks)
+        O_hosts = O_hosts or [None] * n
+        out_hosts = out_hosts or [None] * n
+        for t in list(X_hosts) + list(O_hosts) + list(out_hosts):
+            if t is not None and (t.is_cuda or not t.is_contiguous() or t.dtype != torch.float32):
+                raise ValueError("host buffers must be contiguous fp32 CPU tensors")
+        vp = ctypes.c_void_p
+        karr = (ctypes.c_int32 * n)(*Ks)
+        xa = (vp * n)(*[_ptr(t) for t in X_hosts])
+        oa = (vp * n)(*[_ptr(t) for t in O_hosts])
+        ea = (vp * n)(*[_ptr(t) for t in out_hosts])
+        _check(lib().gnn_run_host_multi(ctypes.byref(self.desc), int(upload_graph), n, karr, xa,
+                                        oa, ea, ctypes.byref(self.opts), _ptr(self.ws),
+                                        self.ws_bytes, _stream(stream)))

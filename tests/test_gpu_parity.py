@@ -575,3 +575,61 @@ def test_run_host_full_size_sampled_parity():
             a, b = oracle.sddmm(g.row_ind, g.col_ind, g.val, X, X, i0=int(e), i1=int(e) + 1)
             r2[i], T2[i] = a[0], b[0]
         assert_within(E.numpy()[edges], r2, T2, what=f"run_host C4 sddmm K={K}")
+
+
+def _run_multi_check(g, Ks, pieces=None, skip_o=(), seed=950):
+    """gnn_run_host_multi over several widths in one call, every output vs the oracle."""
+    import os
+    old = os.environ.get("GNN_HOST_PIECES")
+    if pieces is not None:
+        os.environ["GNN_HOST_PIECES"] = str(pieces)
+    try:
+        runner = gs.HostRunner(g.M, g.N, g.row_ind, g.col_ind, g.val, max(Ks), device=DEV,
+                               Ks=Ks).pin()
+        Xs = [torch.from_numpy(_x(seed + K, g.N, K)).pin_memory() for K in Ks]
+        Os = [None if j in skip_o else torch.full((g.M, K), float("nan")).pin_memory()
+              for j, K in enumerate(Ks)]
+        Es = [torch.full((g.nnz,), float("nan")).pin_memory() for _ in Ks]
+        for rep in range(2):  # the second call reuses the uploaded graph
+            runner.run_multi(Xs, Ks, Os, Es, upload_graph=(rep == 0))
+            torch.cuda.synchronize()
+            for j, K in enumerate(Ks):
+                X = Xs[j].numpy()
+                if Os[j] is not None:
+                    ref, T = oracle.spmm(g.row_ind, g.col_ind, g.val, X, M=g.M)
+                    assert_within(Os[j].numpy(), ref, T, what=f"multi spmm K={K} rep={rep}")
+                r2, T2 = oracle.sddmm(g.row_ind, g.col_ind, g.val, X, X)
+                assert_within(Es[j].numpy(), r2, T2, what=f"multi sddmm K={K} rep={rep}")
+                Es[j].fill_(float("nan"))
+                if Os[j] is not None:
+                    Os[j].fill_(float("nan"))
+    finally:
+        if old is None:
+            os.environ.pop("GNN_HOST_PIECES", None)
+        else:
+            os.environ["GNN_HOST_PIECES"] = old
+
+
+@pytest.mark.parametrize("pieces", [None, 3, 32])
+def test_run_host_multi_widths(pieces):
+    """Several feature widths in one pipelined gnn_run_host_multi call (per-width plans,
+    pieces alternating over two compute streams across widths, one width's SpMM skipped)."""
+    g = configs.make_graph("C2")
+    _run_multi_check(g, (32, 8, 256, 64), pieces, skip_o=(1,))
+    rng = np.random.default_rng(23)
+    M = 2500
+    rows = rng.integers(0, M, 50000)
+    rows = rows[(rows % 13) > 3]
+    rows = np.concatenate([rows, np.full(15000, 700), [M - 1]])
+    g2 = gen.from_coo(M, M, rows, rng.integers(0, M, rows.size), gen.uniform_values(6, rows.size))
+    _run_multi_check(g2, (16, 128), pieces)
+
+
+def test_run_host_multi_rejects_bad_arguments():
+    g = configs.make_graph("C1")
+    runner = gs.HostRunner(g.M, g.N, g.row_ind, g.col_ind, g.val, 32, device=DEV, Ks=(32,))
+    X = torch.zeros((g.N, 32))
+    with pytest.raises(gs.GnnError):
+        runner.run_multi([X], [0])
+    with pytest.raises(gs.GnnError):
+        runner.run_multi([X] * 17, [32] * 17)
