@@ -325,7 +325,7 @@ def time_path(args, g, perm, name, Ks, dev, world, rank, dtype="f32"):
         my_flops += spmm_flops(spg.nnz, K) + sddmm_flops(sdg.nnz, K)
         t_sp, t_sd = statistics.mean(per[K]["spmm"]), statistics.mean(per[K]["sddmm"])
         detail[f"K{K}"] = {
-            "chunk": info["chunk"], "vw_feat": info["vw_feat"], "lanes": info["lanes"],
+            "chunk": info["chunk"], "chunk_dtp": info["chunk_dtp"], "vw_feat": info["vw_feat"], "lanes": info["lanes"],
             "active_blocks_per_sm": info["active_blocks_per_sm"],
             "comm_ms": round(statistics.mean(per[K]["comm"]), 4),
             "plan_ms": round(statistics.mean(per[K]["plan"]), 4), "spmm_ms": round(t_sp, 4),

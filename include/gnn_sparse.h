@@ -80,6 +80,8 @@ typedef struct {
                               through per-chunk partials in the workspace (no atomics:
                               bit-reproducible; workspace grows by 8*K B per chunk)     */
   int32_t feature_dtype;   /* gnn_dtype_t of the feature matrices; default GNN_F32   */
+  int32_t no_locality;     /* 1: plain DTP, skip the L2 locality cap (DESIGN.md §3
+                              step 5b); 0 (default) applies it                       */
 } gnn_plan_opts_t;
 
 /* What the plan decided (all integers; bit-exact with the oracle's plan). */
@@ -97,22 +99,29 @@ typedef struct {
   int32_t alpha;
   int32_t K;
   int32_t feature_dtype;   /* gnn_dtype_t the plan was built for                    */
+  int32_t chunk_dtp;       /* the plain-DTP choice before the locality cap           */
   int64_t nnz;
   int64_t num_chunks;      /* ceil(nnz / chunk)                                     */
   int64_t num_blocks;      /* SpMM grid size (integer form of InEq. (5) RHS)         */
+  int64_t M;               /* rows of the planned graph (locality cap input)        */
+  int64_t l2_bytes;        /* device L2 size the locality cap used (0: cap off)     */
 } gnn_plan_info_t;
 
 typedef struct gnn_plan *gnn_plan_t;
 
 /* ---------------------------------------------------------------- plan ---- */
-/* Bytes of device workspace gnn_plan_create needs for (nnz, K, opts) on the current
- * device (exact; 0 when nnz == 0).  Returns (size_t)-1 on invalid arguments. */
-GNN_API size_t gnn_plan_workspace_bytes(int64_t nnz, int32_t K, const gnn_plan_opts_t *opts);
+/* Bytes of device workspace gnn_plan_create needs for a graph of M rows and nnz
+ * nonzeros at width K with opts on the current device (exact; 0 when nnz == 0).
+ * Returns (size_t)-1 on invalid arguments. */
+GNN_API size_t gnn_plan_workspace_bytes(int64_t M, int64_t nnz, int32_t K,
+                                        const gnn_plan_opts_t *opts);
 
 /* Dynamic Task Partition + Hierarchical Vectorized Memory Access and the
  * per-chunk boundary table of the hybrid-parallel strategy (Algo 3 lines
  * 2-3 P:175-176).  Host part: C* from InEq. (5) over the candidate set
- * {8,32,64,128,256,512}, scalar integer arithmetic only -- no device read, no sync.
+ * {8,32,64,128,256,512}, capped so that the feature rows of the rows in flight fit a
+ * quarter of L2 (DESIGN.md §3 step 5b, a B200 addition to DTP), scalar integer
+ * arithmetic only -- no device read, no sync.
  * Device part: one launch writing, for every chunk c (nnz [c*C*, min((c+1)*C*, nnz))),
  *   row_first[c] = row_ind[start], row_last[c] = row_ind[end-1],
  *   flags[c] = (head row continues from chunk c-1) | (tail row continues into c+1) << 1.

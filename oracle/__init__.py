@@ -26,9 +26,9 @@ class _PlanInfo(ctypes.Structure):
     _fields_ = [(n, ctypes.c_int32) for n in (
         "chunk", "vw_feat", "vw_sparse", "lanes", "vecs", "slices", "groups",
         "warps_per_block", "active_blocks_per_sm", "num_sms", "alpha", "K",
-        "feature_dtype")] + [
+        "feature_dtype", "chunk_dtp")] + [
         ("nnz", ctypes.c_int64), ("num_chunks", ctypes.c_int64),
-        ("num_blocks", ctypes.c_int64)]
+        ("num_blocks", ctypes.c_int64), ("M", ctypes.c_int64), ("l2_bytes", ctypes.c_int64)]
 
 
 def _load():
@@ -44,7 +44,7 @@ def _load():
     lib.oracle_spmm.argtypes = [i64, i64, vp, vp, vp, i64, vp, i64, i64, i64, vp, vp]
     lib.oracle_sddmm.argtypes = [i64, i64, vp, vp, vp, i64, vp, i64, vp, i64, vp, vp]
     lib.oracle_spmm_agg.argtypes = [i64, i64, vp, vp, vp, i64, vp, i64, i64, i64, i32, vp, vp]
-    lib.oracle_plan.argtypes = [i64, vp, i32, i32, i32, i32, i32, i32, i32, i32,
+    lib.oracle_plan.argtypes = [i64, vp, i32, i32, i32, i32, i32, i32, i32, i32, i64, i64,
                                 ctypes.POINTER(_PlanInfo), vp, vp, vp]
     lib.oracle_shard_rows.argtypes = [vp, i64, i32, vp]
     lib.oracle_shard_edges.argtypes = [i64, i32, vp]
@@ -156,15 +156,17 @@ class Plan:
 
 
 def plan(row_ind, K, num_sms, active_blocks_per_sm, alpha=2, warps_per_block=8,
-         force_chunk=0, force_vw=0, feature_dtype=0) -> Plan:
-    """DTP/HVMA plan; device parameters are inputs."""
+         force_chunk=0, force_vw=0, feature_dtype=0, M=0, l2_bytes=0) -> Plan:
+    """DTP/HVMA plan; device parameters are inputs.  M (graph
+    rows) and l2_bytes (device L2) feed the locality cap, step 5b; l2_bytes = 0 is the
+    plain DTP rule."""
     lib = _load()
     row_ind = _i32(row_ind)
     nnz = row_ind.shape[0]
     info = _PlanInfo()
     # first call sizes the arrays (chunk depends on the rule)
     rc = lib.oracle_plan(nnz, _ptr(row_ind), K, alpha, warps_per_block, force_chunk,
-                         force_vw, feature_dtype, num_sms, active_blocks_per_sm,
+                         force_vw, feature_dtype, num_sms, active_blocks_per_sm, M, l2_bytes,
                          ctypes.byref(info), None, None, None)
     if rc != 0:
         raise ValueError("oracle_plan: invalid arguments")
@@ -173,7 +175,7 @@ def plan(row_ind, K, num_sms, active_blocks_per_sm, alpha=2, warps_per_block=8,
     rl = np.empty(nch, np.int32)
     fl = np.empty(nch, np.uint8)
     lib.oracle_plan(nnz, _ptr(row_ind), K, alpha, warps_per_block, force_chunk,
-                    force_vw, feature_dtype, num_sms, active_blocks_per_sm,
+                    force_vw, feature_dtype, num_sms, active_blocks_per_sm, M, l2_bytes,
                     ctypes.byref(info), _ptr(rf), _ptr(rl), _ptr(fl))
     d = {name: getattr(info, name) for name, _ in _PlanInfo._fields_}
     return Plan(d, rf, rl, fl)

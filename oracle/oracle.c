@@ -118,10 +118,11 @@ static int64_t blocks_for(int64_t nnz, int64_t C, int64_t S, int64_t G, int64_t 
 
 int oracle_plan(int64_t nnz, const int32_t *row_ind, int32_t K, int32_t alpha,
                 int32_t warps_per_block, int32_t force_chunk, int32_t force_vw,
-                int32_t feature_dtype, int32_t num_sms, int32_t active_blocks_per_sm, oracle_plan_info_t *info,
+                int32_t feature_dtype, int32_t num_sms, int32_t active_blocks_per_sm,
+                int64_t M, int64_t l2_bytes, oracle_plan_info_t *info,
                 int32_t *row_first, int32_t *row_last, uint8_t *flags) {
   if (nnz < 0 || K < 1 || alpha < 1 || warps_per_block < 1 || num_sms < 1 ||
-      active_blocks_per_sm < 1 || force_chunk < 0 || !info)
+      active_blocks_per_sm < 1 || force_chunk < 0 || M < 0 || l2_bytes < 0 || !info)
     return -1;
   /* step 1: feature vector width in elements of the feature dtype (0 fp32: 8,4,2,1;
    * 1 bf16: 16,8,4,2): the widest that divides K, or forced */
@@ -154,6 +155,29 @@ int oracle_plan(int64_t nnz, const int32_t *row_ind, int32_t K, int32_t alpha,
     if (blocks_for(nnz, kCandidates[j], S, G, warps_per_block) >= (int64_t)alpha * FW)
       C = kCandidates[j];
   }
+  int32_t C_dtp = C;
+  /* step 5b (a B200 reading -- not in the paper): the locality
+   * cap.  One full wave holds FW x WarpsPerBlock x G / S chunks; with C nonzeros each
+   * that is (FW x WPB x G x C) / S nonzeros in flight, covering about
+   * nonzeros x M / nnz rows (at most M).  Their feature rows, rows x K x eb bytes
+   * (eb = 4 fp32, 2 bf16), must fit a quarter of L2: compared without overflow as
+   * rows <= floor(floor(L2 / 4) / (K x eb)).  The largest candidate <= C_dtp that fits
+   * wins; if none fits, 8.  l2_bytes == 0 switches the cap off. */
+  if (l2_bytes > 0 && nnz > 0 && M > 0) {
+    int64_t eb = feature_dtype == 1 ? 2 : 4;
+    int64_t rows_that_fit = (l2_bytes / 4) / ((int64_t)K * eb);
+    int32_t capped = 8;
+    for (int j = 0; j < 6; ++j) {
+      int32_t cand = kCandidates[j];
+      if (cand > C_dtp) continue;
+      int64_t chunks_in_flight_x_C = FW * warps_per_block * G * cand;
+      int64_t nnz_in_flight = chunks_in_flight_x_C / S;
+      int64_t rows_in_flight = nnz_in_flight * M / nnz;
+      if (rows_in_flight > M) rows_in_flight = M;
+      if (rows_in_flight <= rows_that_fit) capped = cand;
+    }
+    C = capped;
+  }
   if (force_chunk > 0) C = force_chunk;
   /* step 6: sparse-load vector width (HVMA) */
   int32_t vws = 1;
@@ -174,6 +198,9 @@ int oracle_plan(int64_t nnz, const int32_t *row_ind, int32_t K, int32_t alpha,
   info->alpha = alpha;
   info->K = K;
   info->feature_dtype = feature_dtype;
+  info->chunk_dtp = C_dtp;
+  info->M = M;
+  info->l2_bytes = l2_bytes;
   info->nnz = nnz;
   info->num_chunks = nch;
   info->num_blocks = nnz > 0 ? blocks_for(nnz, C, S, G, warps_per_block) : 0;

@@ -48,14 +48,16 @@ class PlanOpts(ctypes.Structure):
     """gnn_plan_opts_t; zero fields take the library defaults (alpha 2, 8 warps/block)."""
     _fields_ = [("alpha", ctypes.c_int32), ("warps_per_block", ctypes.c_int32),
                 ("force_chunk", ctypes.c_int32), ("force_vw", ctypes.c_int32),
-                ("deterministic", ctypes.c_int32), ("feature_dtype", ctypes.c_int32)]
+                ("deterministic", ctypes.c_int32), ("feature_dtype", ctypes.c_int32),
+                ("no_locality", ctypes.c_int32)]
 
 
 class _PlanInfo(ctypes.Structure):
     _fields_ = [(n, ctypes.c_int32) for n in (
         "chunk", "vw_feat", "vw_sparse", "lanes", "vecs", "slices", "groups", "warps_per_block",
-        "active_blocks_per_sm", "num_sms", "alpha", "K", "feature_dtype")] + [
-        ("nnz", ctypes.c_int64), ("num_chunks", ctypes.c_int64), ("num_blocks", ctypes.c_int64)]
+        "active_blocks_per_sm", "num_sms", "alpha", "K", "feature_dtype", "chunk_dtp")] + [
+        ("nnz", ctypes.c_int64), ("num_chunks", ctypes.c_int64), ("num_blocks", ctypes.c_int64),
+        ("M", ctypes.c_int64), ("l2_bytes", ctypes.c_int64)]
 
 
 class ReorderOpts(ctypes.Structure):
@@ -86,7 +88,7 @@ def lib():
     L = ctypes.CDLL(LIB_PATH)
     vp, i64, i32, st = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_int
     P = ctypes.POINTER
-    L.gnn_plan_workspace_bytes.argtypes = [i64, i32, P(PlanOpts)]
+    L.gnn_plan_workspace_bytes.argtypes = [i64, i64, i32, P(PlanOpts)]
     L.gnn_plan_workspace_bytes.restype = ctypes.c_size_t
     L.gnn_plan_create.argtypes = [P(_Graph), i32, P(PlanOpts), vp, ctypes.c_size_t, vp, P(vp)]
     L.gnn_plan_info.argtypes = [vp, P(_PlanInfo)]
@@ -258,20 +260,22 @@ def _dtype_code(d):
 
 
 def _opts(alpha=0, warps_per_block=0, force_chunk=0, force_vw=0, feature_dtype=0,
-          deterministic=False):
+          deterministic=False, no_locality=False):
     return PlanOpts(alpha, warps_per_block, force_chunk, force_vw, int(bool(deterministic)),
-                    _dtype_code(feature_dtype))
+                    _dtype_code(feature_dtype), int(bool(no_locality)))
 
 
 def plan(graph: DeviceGraph, K: int, alpha: int = 0, warps_per_block: int = 0,
          force_chunk: int = 0, force_vw: int = 0, feature_dtype=GNN_F32,
-         deterministic: bool = False, stream=None) -> Plan:
+         deterministic: bool = False, no_locality: bool = False, stream=None) -> Plan:
     """gnn_plan_create: DTP/HVMA chunking + the GPU plan kernel (no host sync).
     feature_dtype: fp32 (default) or bf16 feature matrices.
-    deterministic: split rows summed in chunk order without atomics (bit-reproducible)."""
+    deterministic: split rows summed in chunk order without atomics (bit-reproducible).
+    no_locality: plain DTP, without the L2 locality cap (DESIGN.md §3 step 5b)."""
     L = lib()
-    o = _opts(alpha, warps_per_block, force_chunk, force_vw, feature_dtype, deterministic)
-    nbytes = L.gnn_plan_workspace_bytes(graph.nnz, K, ctypes.byref(o))
+    o = _opts(alpha, warps_per_block, force_chunk, force_vw, feature_dtype, deterministic,
+              no_locality)
+    nbytes = L.gnn_plan_workspace_bytes(graph.M, graph.nnz, K, ctypes.byref(o))
     if nbytes == ctypes.c_size_t(-1).value:
         _check(GNN_ERR_INVALID_ARG)
     dev = graph.row_ind.device

@@ -30,7 +30,7 @@ bool layout(int64_t M, int64_t N, int64_t nnz, int32_t nk, const int32_t *K,
   l->col_ind = o; o += a256(4 * (size_t)nnz);
   l->val = o;     o += a256(4 * (size_t)nnz);
   for (int k = 0; k < nk; ++k) {
-    const size_t pb = gnn_plan_workspace_bytes(nnz, K[k], opts);
+    const size_t pb = gnn_plan_workspace_bytes(M, nnz, K[k], opts);
     if (pb == (size_t)-1) return false;
     l->X[k] = o;    o += a256(4 * (size_t)N * K[k]);
     l->O[k] = o;    o += a256(4 * (size_t)M * K[k]);
@@ -159,7 +159,7 @@ GNN_API gnn_status_t gnn_run_host_multi(const gnn_graph_t *gh, int32_t upload_gr
   const bool det = opts && opts->deterministic;
   for (int k = 0; k < nk; ++k) {
     if (gnn_status_t st = gnn_plan_create(&gd, Ks[k], opts, w + l.plan[k],
-                                          gnn_plan_workspace_bytes(nnz, Ks[k], opts), stream,
+                                          gnn_plan_workspace_bytes(M, nnz, Ks[k], opts), stream,
                                           &plans.p[k]))
       return st;
     if (O_host && O_host[k] && !det && nnz > 0)

@@ -17,6 +17,7 @@ struct DeviceInfo {
   int device;
   int num_sms;
   int cc_major, cc_minor;
+  int64_t l2_bytes;
 };
 gnn_status_t device_info(DeviceInfo *out);
 

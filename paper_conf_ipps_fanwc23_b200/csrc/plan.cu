@@ -25,15 +25,15 @@ inline int64_t blocks_for(int64_t nnz, int64_t C, int64_t S, int64_t G, int64_t 
   return cdiv(cdiv(cdiv(nnz, C) * S, G), WPB);
 }
 
-gnn_status_t make_info(int64_t nnz, int32_t K, const gnn_plan_opts_t *opts,
+gnn_status_t make_info(int64_t M, int64_t nnz, int32_t K, const gnn_plan_opts_t *opts,
                        gnn_plan_info_t *info) {
   gnn_plan_opts_t o{};
   if (opts) o = *opts;
   const int32_t alpha = o.alpha ? o.alpha : 2;
   const int32_t wpb = o.warps_per_block ? o.warps_per_block : 8;
-  if (nnz < 0 || nnz >= (int64_t(1) << 31) || K < 1 || alpha < 1 || wpb < 1 ||
+  if (M < 0 || nnz < 0 || nnz >= (int64_t(1) << 31) || K < 1 || alpha < 1 || wpb < 1 ||
       wpb * 32 > kMaxThreads || o.force_chunk < 0 || o.deterministic < 0 ||
-      o.deterministic > 1)
+      o.deterministic > 1 || o.no_locality < 0 || o.no_locality > 1)
     return fail(GNN_ERR_INVALID_ARG,
                 "plan: bad arguments (nnz=%lld K=%d alpha=%d wpb=%d force_chunk=%d det=%d)",
                 (long long)nnz, K, alpha, wpb, o.force_chunk, o.deterministic);
@@ -74,6 +74,24 @@ gnn_status_t make_info(int64_t nnz, int32_t K, const gnn_plan_opts_t *opts,
   int32_t C = 8;
   for (int32_t c : kCand)
     if (blocks_for(nnz, c, S, G, wpb) >= alpha * FW) C = c;
+  const int32_t C_dtp = C;
+  // step 5b (B200 addition): locality cap.  A full wave holds FW*WPB*G/S chunks, i.e.
+  // about that many * C / (nnz / M) rows in flight; after a clustering reorder their
+  // feature rows are the L2 working set, so C* is the largest candidate <= C_dtp whose
+  // rows in flight fit a quarter of L2 (else 8).
+  const int64_t l2 = o.no_locality ? 0 : d.l2_bytes;  // 0: cap off (reported in the info)
+  if (l2 > 0 && nnz > 0 && M > 0) {
+    const int64_t eb = dt == GNN_BF16 ? 2 : 4;
+    const int64_t rows_fit = (l2 / 4) / ((int64_t)K * eb);
+    int32_t Cl = kCand[0];
+    for (int32_t c : kCand) {
+      if (c > C_dtp) break;
+      int64_t rows = ((FW * wpb * G * c) / S) * M / nnz;
+      if (rows > M) rows = M;
+      if (rows <= rows_fit) Cl = c;
+    }
+    C = Cl;
+  }
   if (o.force_chunk > 0) C = o.force_chunk;
   // step 6: sparse vector width (HVMA)
   int32_t vws = 1;
@@ -93,6 +111,9 @@ gnn_status_t make_info(int64_t nnz, int32_t K, const gnn_plan_opts_t *opts,
   info->alpha = alpha;
   info->K = K;
   info->feature_dtype = dt;
+  info->chunk_dtp = C_dtp;
+  info->M = M;
+  info->l2_bytes = l2;
   info->nnz = nnz;
   info->num_chunks = nnz > 0 ? cdiv(nnz, C) : 0;
   info->num_blocks = nnz > 0 ? blocks_for(nnz, C, S, G, wpb) : 0;
@@ -134,9 +155,10 @@ using namespace gnn;
 
 extern "C" {
 
-GNN_API size_t gnn_plan_workspace_bytes(int64_t nnz, int32_t K, const gnn_plan_opts_t *opts) {
+GNN_API size_t gnn_plan_workspace_bytes(int64_t M, int64_t nnz, int32_t K,
+                                        const gnn_plan_opts_t *opts) {
   gnn_plan_info_t info;
-  if (make_info(nnz, K, opts, &info) != GNN_OK) return (size_t)-1;
+  if (make_info(M, nnz, K, opts, &info) != GNN_OK) return (size_t)-1;
   return ws_bytes_for(info.num_chunks, K, opts ? opts->deterministic : 0);
 }
 
@@ -149,7 +171,7 @@ GNN_API gnn_status_t gnn_plan_create(const gnn_graph_t *g, int32_t K,
       (g->nnz > 0 && (!g->row_ind || !g->col_ind)))
     return fail(GNN_ERR_INVALID_ARG, "gnn_plan_create: bad graph descriptor");
   gnn_plan_info_t info;
-  if (gnn_status_t st = make_info(g->nnz, K, opts, &info)) return st;
+  if (gnn_status_t st = make_info(g->M, g->nnz, K, opts, &info)) return st;
   const int64_t nch = info.num_chunks;
   const int32_t det = opts ? opts->deterministic : 0;
   const size_t need = ws_bytes_for(nch, K, det);

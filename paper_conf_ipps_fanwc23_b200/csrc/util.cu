@@ -43,6 +43,9 @@ gnn_status_t device_info(DeviceInfo *out) {
       return cuda_fail(e, "cudaDeviceGetAttribute(SM count)");
     cudaDeviceGetAttribute(&d.cc_major, cudaDevAttrComputeCapabilityMajor, dev);
     cudaDeviceGetAttribute(&d.cc_minor, cudaDevAttrComputeCapabilityMinor, dev);
+    int l2 = 0;
+    cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, dev);
+    d.l2_bytes = l2;
     if (d.cc_major != 10 || d.cc_minor != 0)
       return fail(GNN_ERR_CUDA, "device %d is sm_%d%d; this library is built for sm_100a only",
                   dev, d.cc_major, d.cc_minor);

@@ -49,9 +49,9 @@ static int run_graph(int64_t n, int64_t nnz_target, int32_t n_comm, uint64_t see
       const int64_t nch_max = nnz / 8 + 2;
       int32_t *rf = malloc(sizeof(int32_t) * nch_max), *rl = malloc(sizeof(int32_t) * nch_max);
       uint8_t *fl = malloc(nch_max);
-      CHECK(oracle_plan(nnz, ri, K, 2, 8, 0, 0, dt, 148, 2, &info, rf, rl, fl) == 0);
+      CHECK(oracle_plan(nnz, ri, K, 2, 8, 0, 0, dt, 148, 2, n, 132644864, &info, rf, rl, fl) == 0);
       CHECK(info.num_chunks <= nch_max);
-      CHECK(oracle_plan(nnz, ri, K, 2, 8, 8, 0, dt, 148, 2, &info, rf, rl, fl) == 0);
+      CHECK(oracle_plan(nnz, ri, K, 2, 8, 8, 0, dt, 148, 2, n, 0, &info, rf, rl, fl) == 0);
       free(rf); free(rl); free(fl);
     }
     free(X); free(O); free(T); free(E); free(TE);

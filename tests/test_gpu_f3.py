@@ -137,6 +137,8 @@ def test_randomized_configurations(seed):
         kw["warps_per_block"] = int(rng.choice([1, 2, 4, 16]))
     if rng.random() < 0.3:
         kw["alpha"] = int(rng.choice([1, 3, 8]))
+    if rng.random() < 0.2:
+        kw["no_locality"] = True
     with_val = rng.random() < 0.8
     dg = upload(g, with_val=with_val)
     p = gs.plan(dg, K, feature_dtype="bf16" if bf16 else "f32", **kw)
@@ -144,7 +146,8 @@ def test_randomized_configurations(seed):
     ref_plan = oracle.plan(g.row_ind, K, info["num_sms"], info["active_blocks_per_sm"],
                            alpha=kw.get("alpha", 2), warps_per_block=kw.get("warps_per_block", 8),
                            force_chunk=kw.get("force_chunk", 0), force_vw=kw.get("force_vw", 0),
-                           feature_dtype=1 if bf16 else 0)
+                           feature_dtype=1 if bf16 else 0, M=M,
+                           l2_bytes=0 if kw.get("no_locality") else info["l2_bytes"])
     assert info == ref_plan.info
     X = torch.from_numpy(gen.features(seed, N, K)).to(DEV)
     A1 = torch.from_numpy(gen.features(seed + 1, M, K)).to(DEV)

@@ -28,10 +28,14 @@ def _x(seed, rows, K, ld=None):
 
 def check_plan(p, g, K, **kw):
     info = p.info()
+    # the locality cap reads the device's L2 size (0 when switched off)
+    l2 = 0 if kw.get("no_locality") else torch.cuda.get_device_properties(0).L2_cache_size
+    assert info["l2_bytes"] == l2 and info["M"] == g.M
     ref = oracle.plan(g.row_ind, K, info["num_sms"], info["active_blocks_per_sm"],
                       alpha=kw.get("alpha", 2) or 2,
                       warps_per_block=kw.get("warps_per_block", 8) or 8,
-                      force_chunk=kw.get("force_chunk", 0), force_vw=kw.get("force_vw", 0))
+                      force_chunk=kw.get("force_chunk", 0), force_vw=kw.get("force_vw", 0),
+                      M=g.M, l2_bytes=l2)
     assert info == ref.info, (info, ref.info)
     rf, rl, fl = (t.cpu().numpy() for t in p.arrays())
     assert np.array_equal(rf, ref.row_first)
@@ -269,7 +273,7 @@ def test_plan_spmm_sddmm_capture_in_cuda_graph():
     X = torch.from_numpy(_x(5, g.N, K)).to(DEV)
     O = torch.empty((g.M, K), device=DEV)
     E = torch.empty(g.nnz, device=DEV)
-    nbytes = gs.lib().gnn_plan_workspace_bytes(g.nnz, K, None)
+    nbytes = gs.lib().gnn_plan_workspace_bytes(g.M, g.nnz, K, None)
     s = torch.cuda.Stream()
     s.wait_stream(torch.cuda.current_stream())
     holder = []
@@ -430,7 +434,7 @@ def test_bf16_features_parity(K):
     p = gs.plan(dg, K, feature_dtype="bf16")
     info = p.info()
     ref = oracle.plan(g.row_ind, K, info["num_sms"], info["active_blocks_per_sm"],
-                      feature_dtype=1)
+                      feature_dtype=1, M=g.M, l2_bytes=info["l2_bytes"])
     assert info == ref.info
     Xb, Xexact, X32 = _bf16_pair(600 + K, g.N, K)
     A1b, A1exact, A132 = _bf16_pair(700 + K, g.M, K)
@@ -633,3 +637,20 @@ def test_run_host_multi_rejects_bad_arguments():
         runner.run_multi([X], [0])
     with pytest.raises(gs.GnnError):
         runner.run_multi([X] * 17, [32] * 17)
+
+
+@pytest.mark.parametrize("no_locality", [False, True])
+def test_locality_cap_plan_and_parity(no_locality):
+    """A low-degree graph with wide rows, where the L2 locality cap (DESIGN.md §3 step
+    5b) lowers C* below the DTP choice: plan info and arrays bit-exact with the oracle
+    (which is given the device's L2 size), outputs within the fp32 bar; with
+    no_locality the plain DTP choice is kept."""
+    rng = np.random.default_rng(31)
+    M = 200_000
+    rows = np.sort(rng.integers(0, M, 800_000))
+    g = gen.from_coo(M, M, rows, rng.integers(0, M, rows.size), gen.uniform_values(8, rows.size))
+    info, _ = run_full(g, 256, no_locality=no_locality)
+    if no_locality:
+        assert info["chunk"] == info["chunk_dtp"]
+    else:
+        assert info["chunk"] < info["chunk_dtp"]

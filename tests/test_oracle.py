@@ -283,6 +283,57 @@ def test_plan_dtp_maximality_bruteforce(nnz, K, alpha, abs_):
     assert p.info["vw_sparse"] == {8: 1, 32: 1, 64: 2, 128: 4, 256: 4, 512: 4}[C]
 
 
+# ---- step 5b, the locality cap: hand-worked examples ----
+# 148 SMs x 2 blocks/SM -> FW = 296; WPB 8; K = 256 fp32 -> L 16, R 2, G 2, S 1.
+# nnz = 10,000,000, M = 200,000 (degree 50): DTP alone -> 512 (blocks(512) = 1221 >= 592).
+# L2 = 64 MiB: rows that fit = (67,108,864 / 4) / (256 * 4) = 16,384.
+#   C = 512: 296*8*2*512 = 2,424,832 nnz in flight * 200,000 / 10^7 = 48,496 rows  > 16,384
+#   C = 256: 1,212,416 -> 24,248 rows > 16,384;  C = 128: 606,208 -> 12,124 rows <= 16,384
+# bf16: VW 16 -> L 8, R 2, G 4 (twice the chunks in flight) and 2 B per element (twice
+#   the rows fit, 32,768): C = 256 -> 48,496 rows > 32,768; C = 128 -> 24,248 -> 128.
+# Degree 100 (M = 100,000), fp32: C = 512 -> 24,248 > 16,384; C = 256 -> 12,124 -> 256.
+# Degree 500 (M = 20,000): C = 512 -> 4,849 rows -> 512.  L2 off -> 512.
+# L2 = 1 MiB: 256 rows fit; even C = 8 (37,888 nnz -> 757 rows) does not -> 8.
+@pytest.mark.parametrize("M,dtype,l2,expect", [
+    (200_000, 0, 64 << 20, 128), (200_000, 1, 64 << 20, 128), (100_000, 0, 64 << 20, 256),
+    (200_000, 0, 0, 512), (20_000, 0, 64 << 20, 512), (200_000, 0, 1 << 20, 8)])
+def test_plan_locality_cap_worked_examples(M, dtype, l2, expect):
+    p = oracle.plan(np.zeros(10_000_000, np.int32), 256, num_sms=148, active_blocks_per_sm=2,
+                    feature_dtype=dtype, M=M, l2_bytes=l2)
+    assert p.info["chunk_dtp"] == 512
+    assert p.info["chunk"] == expect
+    assert p.info["num_chunks"] == -(-10_000_000 // expect)
+
+
+def test_plan_locality_cap_monotone():
+    """More L2 never shrinks C*, more rows per nonzero never grows it, the cap never
+    exceeds the DTP choice, and an unbounded L2 (or none) gives DTP exactly."""
+    rng = np.random.default_rng(77)
+    cands = [8, 32, 64, 128, 256, 512]
+    for _ in range(60):
+        nnz = int(rng.integers(1, 3_000_000))
+        K = int(rng.choice([8, 32, 64, 128, 256, 512, 1024]))
+        abs_ = int(rng.integers(1, 9))
+        dt = int(rng.integers(0, 2)) if K % 2 == 0 else 0
+        row_ind = np.zeros(nnz, np.int32)
+
+        def chunk(M, l2):
+            return oracle.plan(row_ind, K, 148, abs_, feature_dtype=dt, M=M,
+                               l2_bytes=l2).info
+
+        M = int(rng.integers(1, 2 * nnz + 2))
+        base = chunk(M, 0)
+        assert base["chunk"] == base["chunk_dtp"]
+        prev = 0
+        for l2 in (1 << 16, 1 << 20, 16 << 20, 64 << 20, 126 << 20, 1 << 40):
+            c = chunk(M, l2)["chunk"]
+            assert c in cands and c <= base["chunk"] and c >= prev
+            prev = c
+        assert prev == base["chunk"]
+        c_small_m = chunk(max(1, M // 4), 64 << 20)["chunk"]
+        assert c_small_m >= chunk(M, 64 << 20)["chunk"]
+
+
 def test_plan_matches_survey_dtp_table():
     """SURVEY.md §8(a1) table (WPB 8, 8 blocks/SM, 148 SMs, alpha 2)."""
     for nnz, K, C in [(10_000, 32, 8), (100_000, 64, 8), (114_848_857, 32, 512),
