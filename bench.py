@@ -456,8 +456,8 @@ def run_ours(args):
         del r2
         torch.cuda.empty_cache()
     e2e = None
-    if world == 1 and not args.no_e2e:
-        e2e = run_e2e(args, g, Ks, dev, perm)
+    if not args.no_e2e:
+        e2e = run_e2e(args, g, Ks, dev, perm, world, rank)
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
         cpu = cpu_baseline(g, Ks, args.cpu_seconds, name)
@@ -606,13 +606,16 @@ def run_c3(args, dev, world, rank):
         dist.destroy_process_group()
 
 
-def run_e2e(args, g, Ks, dev, perm=None):
+def run_e2e(args, g, Ks, dev, perm=None, world=1, rank=0):
     """Same metric end to end through the C-ABI call on HOST buffers: every step copies
     the graph arrays (once) and X (per K) from pinned host memory, plans, runs SpMM +
     SDDMM and copies O and S_O back to pinned host memory -- all inside the CUDA-event
     timed region.  Headline: one gnn_run_host_multi call per step (all widths pipelined
-    together); also reported: one gnn_run_host call per width."""
+    together); also reported: one gnn_run_host call per width.  With N ranks each rank
+    runs its nnz-balanced row shard (graph rows, its O rows and S_O entries; X whole)
+    and the time is the max over ranks."""
     import torch
+    import torch.distributed as dist
 
     import paper_conf_ipps_fanwc23_b200 as gs
     from gen import configs
@@ -624,13 +627,18 @@ def run_e2e(args, g, Ks, dev, perm=None):
             Xp[perm] = X
             X = Xp
         return torch.from_numpy(X).pin_memory()
-    runner = gs.HostRunner(g.M, g.N, g.row_ind, g.col_ind, g.val, max(Ks), device=dev,
-                           Ks=Ks).pin()
+    b = gs.shard_rows(g.row_ptr, world) if world > 1 else np.array([0, g.M])
+    r0, r1 = int(b[rank]), int(b[rank + 1])
+    e0, e1 = int(g.row_ptr[r0]), int(g.row_ptr[r1])
+    M, nnz = r1 - r0, e1 - e0
+    runner = gs.HostRunner(M, g.N, g.row_ind[e0:e1], g.col_ind[e0:e1],
+                           None if g.val is None else g.val[e0:e1], max(Ks), device=dev,
+                           Ks=Ks, row_base=r0).pin()
     h_X = {K: feats(K) for K in Ks}
-    h_O = {K: torch.empty((g.M, K), dtype=torch.float32).pin_memory() for K in Ks}
-    h_E = {K: torch.empty(g.nnz, dtype=torch.float32).pin_memory() for K in Ks}
-    h2d = 12 * g.nnz + sum(4 * g.N * K for K in Ks)
-    d2h = sum(4 * g.M * K for K in Ks) + 4 * g.nnz * len(Ks)
+    h_O = {K: torch.empty((M, K), dtype=torch.float32).pin_memory() for K in Ks}
+    h_E = {K: torch.empty(nnz, dtype=torch.float32).pin_memory() for K in Ks}
+    h2d = 12 * nnz + sum(4 * g.N * K for K in Ks)      # this rank's copies
+    d2h = sum(4 * M * K for K in Ks) + 4 * nnz * len(Ks)
 
     def step_multi():
         runner.run_multi([h_X[K] for K in Ks], list(Ks), [h_O[K] for K in Ks],
@@ -644,6 +652,8 @@ def run_e2e(args, g, Ks, dev, perm=None):
         for _ in range(max(1, min(args.warmup, 2))):
             step()
         torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
         steps = max(1, min(args.steps, 5))
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record()
@@ -651,14 +661,26 @@ def run_e2e(args, g, Ks, dev, perm=None):
             step()
         b.record()
         torch.cuda.synchronize()
-        return a.elapsed_time(b) / steps, steps
+        ms_ = a.elapsed_time(b) / steps
+        if world > 1:  # max over ranks
+            t = torch.tensor([ms_], dtype=torch.float64,
+                             device=dev if dist.get_backend() == "nccl" else "cpu")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ms_ = float(t[0])
+        return ms_, steps
 
     ms, steps = timed(step_multi)
     ms_calls, _ = timed(step_calls)
-    nbytes = sum(spmm_bytes(g.nnz, g.M, K) + sddmm_bytes(g.nnz, g.M, K) for K in Ks)
+    nbytes = sum(spmm_bytes(g.nnz, g.M, K) + sddmm_bytes(g.nnz, g.M, K) for K in Ks)  # all ranks
+    if world > 1:
+        t = torch.tensor([float(h2d), float(d2h)], dtype=torch.float64,
+                         device=dev if dist.get_backend() == "nccl" else "cpu")
+        dist.all_reduce(t)
+        h2d, d2h = float(t[0]), float(t[1])
     return {"value": round(nbytes / (ms * 1e-3) / 1e9, 2), "unit": "GB/s",
             "ms_per_step": round(ms, 3), "h2d_bytes_per_step": int(h2d),
             "d2h_bytes_per_step": int(d2h), "steps": steps, "api": "gnn_run_host_multi",
+            "ranks": world, "sharding": "nnz-balanced row shards (X whole on every rank)",
             "per_width_calls": {"api": "gnn_run_host (one call per K)",
                                 "ms_per_step": round(ms_calls, 3),
                                 "value": round(nbytes / (ms_calls * 1e-3) / 1e9, 2)}}

@@ -258,7 +258,9 @@ GNN_API gnn_status_t gnn_permute_rows(const float *X, int64_t ldx, int64_t n, in
  * values download on a copy-out stream, so the call costs about max(upload, compute,
  * download) instead of their sum.  Deterministic plans run as one piece.  Reads the host
  * row_ind to find the rows each piece completes.
- * graph_host: square (M == N), row_base 0, host pointers (row_ptr unused).  fp32 only.
+ * graph_host: host pointers (row_ptr unused), a square N-node graph or a row shard of one
+ * (rows [row_base, row_base + M) with row_base + M <= N; SDDMM then uses A1 = those rows
+ * of X, O holds the shard's M rows).  fp32 only.
  * upload_graph = 0 reuses the graph already in this workspace from an earlier call (the
  * graph's offsets do not depend on K, so one workspace sized for the largest K serves all).
  * workspace: gnn_run_host_workspace_bytes(M, N, nnz, K, opts) bytes, 256-B aligned, device. */

@@ -462,11 +462,14 @@ class HostRunner:
     descriptor; run() / run_multi() enqueue H2D copies, plans, SpMM, SDDMM and D2H copies
     ordered on the current stream (synchronise before reading)."""
 
-    def __init__(self, M, N, row_ind, col_ind, val, Kmax, device="cuda", Ks=None, **opts):
+    def __init__(self, M, N, row_ind, col_ind, val, Kmax, device="cuda", Ks=None, row_base=0,
+                 **opts):
+        """M rows [row_base, row_base + M) of an N-node graph (a row shard when M < N)."""
         self._keep = [np.ascontiguousarray(row_ind, np.int32),
                       np.ascontiguousarray(col_ind, np.int32),
                       None if val is None else np.ascontiguousarray(val, np.float32)]
         self.M, self.N, self.nnz = int(M), int(N), int(row_ind.shape[0] if hasattr(row_ind, "shape") else len(row_ind))
+        self.row_base = int(row_base)
         self.opts = _opts(**opts)
         nbytes = lib().gnn_run_host_workspace_bytes(self.M, self.N, self.nnz, Kmax,
                                                     ctypes.byref(self.opts))
@@ -483,14 +486,15 @@ class HostRunner:
         self.ws_bytes = int(nbytes)
         self.desc = _Graph(self.M, self.N, self.nnz, None, self._keep[0].ctypes.data,
                            self._keep[1].ctypes.data,
-                           None if self._keep[2] is None else self._keep[2].ctypes.data, 0)
+                           None if self._keep[2] is None else self._keep[2].ctypes.data, self.row_base)
 
     def pin(self):
         """Re-point the graph at pinned copies (asynchronous H2D)."""
         pinned = [None if a is None else torch.from_numpy(a).pin_memory() for a in self._keep]
         self._pinned = pinned
         self.desc = _Graph(self.M, self.N, self.nnz, None, pinned[0].data_ptr(),
-                           pinned[1].data_ptr(), None if pinned[2] is None else pinned[2].data_ptr(), 0)
+                           pinned[1].data_ptr(), None if pinned[2] is None else pinned[2].data_ptr(),
+                           self.row_base)
         return self
 
     def run(self, X_host: torch.Tensor, K: int, O_host=None, out_host=None, upload_graph=True,

@@ -458,10 +458,12 @@ struct TmaTiles {
   __device__ __forceinline__ float *vals(int st, int g) const {
     return reinterpret_cast<float *>(arr(st, 2, g));
   }
-  // chunk_of(gg, &cs, &n): first nonzero and count of group gg's chunk (n = 0: none).
+  // chunk_of(gg, &cs, &n): first nonzero and count of group gg's chunk (n = 0: none);
+  // (own_cs, own_n: the calling lane's own group's, unused here)
   template <typename ChunkOf>
   __device__ __forceinline__ void init(int32_t *warp_smem, int lane, const int32_t *ri0,
-                                       const int32_t *ci0, const float *vi0, ChunkOf chunk_of) {
+                                       const int32_t *ci0, const float *vi0, ChunkOf chunk_of,
+                                       int64_t, int) {
     w = warp_smem;
 #pragma unroll
     for (int q = 0; q < SLOTS; ++q) {
@@ -521,17 +523,19 @@ struct AsyncTiles : SparseTiles<L, VWS> {
   int g, l, cnt;
   const int32_t *ri, *ci;
   const float *vi;
+  // each lane copies for its own group only: (own_cs, own_n) = its chunk's first nonzero
+  // and count, as the kernel already computed them
   template <typename ChunkOf>
   __device__ __forceinline__ void init(int32_t *warp_smem, int lane, const int32_t *ri0,
-                                       const int32_t *ci0, const float *vi0, ChunkOf chunk_of) {
+                                       const int32_t *ci0, const float *vi0, ChunkOf,
+                                       int64_t own_cs, int own_n) {
     this->w = warp_smem;
     g = lane / L;
     l = lane & (L - 1);
-    int64_t cs;
-    chunk_of(g, cs, cnt);
-    ri = ri0 + cs;
-    ci = ci0 + cs;
-    vi = vi0 ? vi0 + cs : nullptr;
+    cnt = own_n;
+    ri = ri0 + own_cs;
+    ci = ci0 + own_cs;
+    vi = vi0 ? vi0 + own_cs : nullptr;
   }
   __device__ __forceinline__ void issue(int st, int tb, int) const {
     Base::load(st, g, l, ri, ci, vi, tb, cnt);

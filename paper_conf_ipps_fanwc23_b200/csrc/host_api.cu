@@ -97,9 +97,11 @@ GNN_API gnn_status_t gnn_run_host_multi(const gnn_graph_t *gh, int32_t upload_gr
                                         const gnn_plan_opts_t *opts, void *workspace,
                                         size_t ws_bytes, gnn_stream_t stream) {
   if (!gh || gh->M < 0 || gh->N < 0 || gh->nnz < 0 || nk < 1 || nk > kMaxK || !Ks || !X_host ||
-      gh->M != gh->N || gh->row_base != 0 || (gh->nnz > 0 && (!gh->row_ind || !gh->col_ind)))
+      gh->row_base < 0 || gh->row_base + gh->M > gh->N ||
+      (gh->nnz > 0 && (!gh->row_ind || !gh->col_ind)))
     return fail(GNN_ERR_INVALID_ARG,
-                "gnn_run_host: bad arguments (square graph with host arrays, 1 <= nk <= %d)",
+                "gnn_run_host: bad arguments (host arrays, rows [row_base, row_base + M) of an "
+                "N-node graph, 1 <= nk <= %d)",
                 kMaxK);
   for (int k = 0; k < nk; ++k)
     if (Ks[k] < 1 || !X_host[k])
@@ -115,7 +117,7 @@ GNN_API gnn_status_t gnn_run_host_multi(const gnn_graph_t *gh, int32_t upload_gr
                 ws_bytes, l.total);
   char *w = (char *)workspace;
   cudaStream_t s = (cudaStream_t)stream;  // compute runs on the caller's stream (+ s2)
-  const int64_t nnz = gh->nnz, M = gh->M, N = gh->N;
+  const int64_t nnz = gh->nnz, M = gh->M, N = gh->N, r0 = gh->row_base;
   const bool up = upload_graph && nnz > 0;
   // Events are re-recorded for every piece: a stream wait captures the event's most recent
   // record at the time it is enqueued, so a fixed set of 8 serves the whole call.
@@ -211,10 +213,10 @@ GNN_API gnn_status_t gnn_run_host_multi(const gnn_graph_t *gh, int32_t upload_gr
         // rows final once pieces 0..p are done: up to this piece's last row, minus that
         // row if it continues into the next piece (whose first chunk also zeroes the empty
         // rows before it).  The copy-out stream waits for every piece in order.
-        int64_t done = M;
+        int64_t done = M;  // (local rows: global row id - row_base)
         if (p + 1 < P) {
           const int32_t rl = gh->row_ind[en - 1];
-          done = gh->row_ind[en] == rl ? rl : (int64_t)rl + 1;
+          done = (gh->row_ind[en] == rl ? rl : (int64_t)rl + 1) - r0;
         }
         e = cudaEventRecord(ev_o, sc);
         if (e == cudaSuccess) e = cudaStreamWaitEvent(res.sout, ev_o, 0);
@@ -226,8 +228,9 @@ GNN_API gnn_status_t gnn_run_host_multi(const gnn_graph_t *gh, int32_t upload_gr
         if (done > rows_done) rows_done = done;
       }
       if (Eh && en > b) {
-        st = launch_sddmm(plan, &gd, X, K, X, K, out, sc, GNN_F32, "gnn_run_host sddmm",
-                          whole ? -1 : c0, c1);
+        // A1 = the shard's own rows of X (destination rows), A2T = all of X
+        st = launch_sddmm(plan, &gd, X + r0 * K, K, X, K, out, sc, GNN_F32,
+                          "gnn_run_host sddmm", whole ? -1 : c0, c1);
         if (st != GNN_OK) break;
         e = cudaEventRecord(ev_e, sc);
         if (e == cudaSuccess) e = cudaStreamWaitEvent(res.sout, ev_e, 0);

@@ -133,7 +133,8 @@ __global__ void __launch_bounds__(kMaxThreads, (SddmmShape<VW, L, SMAX>::minb))
                    cs_ = cc * a.chunk;
                    n_ = (int)(min(cs_ + (int64_t)a.chunk, a.nnz) - cs_);
                  }
-               });
+               },
+               cs, n);
   }
   tiles.issue(0, 0, lane);
 

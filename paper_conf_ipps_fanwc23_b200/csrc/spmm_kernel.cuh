@@ -193,7 +193,8 @@ __global__ void __launch_bounds__(kMaxThreads, GNN_SPMM_MINB)
                    cs_ = (it / a.slices) * a.chunk;
                    n_ = (int)(min(cs_ + (int64_t)a.chunk, a.nnz) - cs_);
                  }
-               });
+               },
+               cs, n);
   }
   tiles.issue(0, 0, lane);
 

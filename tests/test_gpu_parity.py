@@ -654,3 +654,35 @@ def test_locality_cap_plan_and_parity(no_locality):
         assert info["chunk"] == info["chunk_dtp"]
     else:
         assert info["chunk"] < info["chunk_dtp"]
+
+
+def test_run_host_multi_row_shards():
+    """gnn_run_host_multi on nnz-balanced row shards (bench.py's e2e at N ranks): each
+    shard's O rows and S_O entries (A1 = the shard's rows of X) against the oracle."""
+    import os
+    g = configs.make_graph("C2")
+    Ks = (32, 128)
+    Xs = [torch.from_numpy(_x(990 + K, g.N, K)).pin_memory() for K in Ks]
+    os.environ["GNN_HOST_PIECES"] = "4"
+    try:
+        for P in (2, 3):
+            b = gs.shard_rows(g.row_ptr, P)
+            for p in range(P):
+                r0, r1 = int(b[p]), int(b[p + 1])
+                e0, e1 = int(g.row_ptr[r0]), int(g.row_ptr[r1])
+                runner = gs.HostRunner(r1 - r0, g.N, g.row_ind[e0:e1], g.col_ind[e0:e1],
+                                       g.val[e0:e1], max(Ks), device=DEV, Ks=Ks,
+                                       row_base=r0).pin()
+                Os = [torch.full((r1 - r0, K), float("nan")).pin_memory() for K in Ks]
+                Es = [torch.full((e1 - e0,), float("nan")).pin_memory() for _ in Ks]
+                runner.run_multi(Xs, Ks, Os, Es)
+                torch.cuda.synchronize()
+                for j, K in enumerate(Ks):
+                    X = Xs[j].numpy()
+                    ref, T = oracle.spmm(g.row_ind, g.col_ind, g.val, X, i0=e0, i1=e1, r0=r0,
+                                         nrows=r1 - r0)
+                    assert_within(Os[j].numpy(), ref, T, what=f"shard {p}/{P} spmm K={K}")
+                    r2, T2 = oracle.sddmm(g.row_ind, g.col_ind, g.val, X, X, i0=e0, i1=e1)
+                    assert_within(Es[j].numpy(), r2, T2, what=f"shard {p}/{P} sddmm K={K}")
+    finally:
+        os.environ.pop("GNN_HOST_PIECES", None)
