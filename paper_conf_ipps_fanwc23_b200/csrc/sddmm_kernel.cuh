@@ -70,6 +70,20 @@ __device__ __forceinline__ void reduce_scale_store(float (&part)[U], const float
     const int u = l / R;
     if (l % R == 0 && u < valid) out[u] = part[0] * (sval ? sval[u] : 1.f);
   } else {
+    // this lane holds P consecutive results: one vector store for a full, aligned batch
+    // (the scalar stores of narrow rows -- 64-byte rows: 16 groups x 4 stores per batch
+    // -- were a visible share of the L1 store wavefronts)
+    if constexpr (P == 2 || P == 4) {
+      float *o = out + l * P;
+      if (valid >= U && (reinterpret_cast<uintptr_t>(o) & (4 * P - 1)) == 0) {
+        float v[P];
+#pragma unroll
+        for (int i = 0; i < P; ++i) v[i] = part[i] * (sval ? sval[l * P + i] : 1.f);
+        if constexpr (P == 4) *reinterpret_cast<float4 *>(o) = make_float4(v[0], v[1], v[2], v[3]);
+        else *reinterpret_cast<float2 *>(o) = make_float2(v[0], v[1]);
+        return;
+      }
+    }
 #pragma unroll
     for (int i = 0; i < P; ++i) {
       const int u = l * P + i;
