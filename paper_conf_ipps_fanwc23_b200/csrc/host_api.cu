@@ -1,11 +1,14 @@
 // host_api.cu -- the end-to-end entry point on HOST buffers (bench.py's e2e path): the
 // caller hands host arrays and one device workspace; the library copies the graph and X
 // in, plans (GPU plan kernel), runs SpMM and SDDMM, and copies O and S_O out.
-// Pipelined over pieces of the plan's chunks on three streams: ColInd/Value of piece p+1
-// upload (copy-in stream) while piece p computes (caller's stream) while the finished
-// rows / edge values of piece p-1 download (copy-out stream); PCIe is full duplex, so
-// the call costs about max(upload, compute, download) instead of their sum.
+// Pipelined over pieces of the nonzeros: X of every width uploads first, then the graph
+// piece by piece (copy-in stream); each piece is planned (plan kernel over its chunks +
+// pre-zero, prep stream) and computed for every width (two alternating compute streams)
+// while the next piece uploads and the finished rows / edge values of the previous one
+// download (copy-out stream).  PCIe is full duplex, so the call costs about
+// max(upload, compute, download) plus the X upload instead of their sum.
 #include <cuda_runtime.h>
+#include <stdio.h>
 #include <stdlib.h>
 
 #include "internal.cuh"
@@ -43,12 +46,13 @@ bool layout(int64_t M, int64_t N, int64_t nnz, int32_t nk, const int32_t *K,
 // Internal streams + events of one gnn_run_host call, released on every return path
 // (cudaStreamDestroy / cudaEventDestroy defer the release until pending work is done).
 struct CallResources {
-  cudaStream_t sin = nullptr, sout = nullptr, s2 = nullptr;
+  cudaStream_t sin = nullptr, sout = nullptr, s2 = nullptr, sp = nullptr;
   cudaEvent_t ev[8] = {};
   int nev = 0;
   ~CallResources() {
     for (int i = 0; i < nev; ++i) cudaEventDestroy(ev[i]);
     if (s2) cudaStreamDestroy(s2);
+    if (sp) cudaStreamDestroy(sp);
     if (sin) cudaStreamDestroy(sin);
     if (sout) cudaStreamDestroy(sout);
   }
@@ -69,6 +73,53 @@ int host_pieces(int64_t nnz) {
   const int64_t p = nnz / (int64_t(4) << 20);
   return p < 1 ? 1 : (p > kMaxPieces ? kMaxPieces : (int)p);
 }
+// GNN_HOST_TRACE=1: timing events at the pipeline's milestones (X uploaded; per piece:
+// uploaded, planned, computed, downloaded), printed to stderr as ms since the call's entry
+// once the call has finished (synchronises: a measurement aid, not for timed runs).
+struct Trace {
+  bool on = false;
+  cudaEvent_t t0 = nullptr, tx = nullptr;
+  cudaEvent_t ev[kMaxPieces][4] = {};
+  int n = 0;
+  Trace() {
+    const char *e = getenv("GNN_HOST_TRACE");
+    on = e && atoi(e) > 0;
+  }
+  cudaEvent_t mk() {
+    cudaEvent_t x = nullptr;
+    cudaEventCreate(&x);
+    return x;
+  }
+  void entry(cudaStream_t s) {
+    if (on) cudaEventRecord(t0 = mk(), s);
+  }
+  void xdone(cudaStream_t s) {
+    if (on) cudaEventRecord(tx = mk(), s);
+  }
+  void mark(int p, int i, cudaStream_t s) {
+    if (!on || p >= kMaxPieces) return;
+    cudaEventRecord(ev[p][i] = mk(), s);
+    if (p + 1 > n) n = p + 1;
+  }
+  ~Trace() {
+    if (!on) return;
+    cudaDeviceSynchronize();
+    auto ms = [&](cudaEvent_t e) {
+      float t = -1.f;
+      if (e) cudaEventElapsedTime(&t, t0, e);
+      return t;
+    };
+    fprintf(stderr, "gnn_run_host trace: X uploaded %.3f ms\n", ms(tx));
+    for (int p = 0; p < n; ++p)
+      fprintf(stderr, "  piece %2d: in %.3f  planned %.3f  computed %.3f  out %.3f\n", p,
+              ms(ev[p][0]), ms(ev[p][1]), ms(ev[p][2]), ms(ev[p][3]));
+    for (int p = 0; p < n; ++p)
+      for (int i = 0; i < 4; ++i)
+        if (ev[p][i]) cudaEventDestroy(ev[p][i]);
+    if (tx) cudaEventDestroy(tx);
+    if (t0) cudaEventDestroy(t0);
+  }
+};
 }  // namespace
 }  // namespace gnn
 
@@ -120,29 +171,25 @@ GNN_API gnn_status_t gnn_run_host_multi(const gnn_graph_t *gh, int32_t upload_gr
   const int64_t nnz = gh->nnz, M = gh->M, N = gh->N, r0 = gh->row_base;
   const bool up = upload_graph && nnz > 0;
   // Events are re-recorded for every piece: a stream wait captures the event's most recent
-  // record at the time it is enqueued, so a fixed set of 8 serves the whole call.
+  // record at the time it is enqueued, so a fixed set serves the whole call.
   CallResources res;
-  cudaEvent_t ev_entry, ev_ri, ev_x, ev_done, ev_pz, ev_in, ev_o, ev_e;
+  Trace trace;  // declared after res: reported before the streams are released
+  cudaEvent_t ev_entry, ev_done, ev_prep, ev_in, ev_o, ev_e;
   cudaError_t e = cudaStreamCreateWithFlags(&res.sin, cudaStreamNonBlocking);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&res.sout, cudaStreamNonBlocking);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&res.s2, cudaStreamNonBlocking);
-  cudaEvent_t *evs[8] = {&ev_entry, &ev_ri, &ev_x, &ev_done, &ev_pz, &ev_in, &ev_o, &ev_e};
-  for (int i = 0; i < 8 && e == cudaSuccess; ++i) e = res.event(evs[i]);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&res.sp, cudaStreamNonBlocking);
+  cudaEvent_t *evs[6] = {&ev_entry, &ev_done, &ev_prep, &ev_in, &ev_o, &ev_e};
+  for (int i = 0; i < 6 && e == cudaSuccess; ++i) e = res.event(evs[i]);
   // everything earlier on the caller's stream (e.g. the previous call still reading this
   // workspace) happens before this call's copies
   if (e == cudaSuccess) e = cudaEventRecord(ev_entry, s);
   if (e == cudaSuccess) e = cudaStreamWaitEvent(res.sin, ev_entry, 0);
   if (e == cudaSuccess) e = cudaStreamWaitEvent(res.sout, ev_entry, 0);
   if (e == cudaSuccess) e = cudaStreamWaitEvent(res.s2, ev_entry, 0);
+  if (e == cudaSuccess) e = cudaStreamWaitEvent(res.sp, ev_entry, 0);
   if (e != cudaSuccess) return cuda_fail(e, "gnn_run_host streams/events");
-  // copy-in stream: RowInd (the plan kernels read all of it), X_0, ColInd/Value piece by
-  // piece (piece p computes while piece p+1 is in flight), then X_1, X_2, ...
-  if (up) {
-    e = cudaMemcpyAsync(w + l.row_ind, gh->row_ind, 4 * nnz, cudaMemcpyHostToDevice, res.sin);
-    if (e == cudaSuccess) e = cudaEventRecord(ev_ri, res.sin);
-    if (e == cudaSuccess) e = cudaStreamWaitEvent(s, ev_ri, 0);
-    if (e != cudaSuccess) return cuda_fail(e, "gnn_run_host graph upload");
-  }
+  trace.entry(s);
   gnn_graph_t gd = *gh;
   gd.row_ptr = nullptr;
   gd.row_ind = (const int32_t *)(w + l.row_ind);
@@ -155,97 +202,123 @@ GNN_API gnn_status_t gnn_run_host_multi(const gnn_graph_t *gh, int32_t upload_gr
         if (q) gnn_plan_destroy(q);
     }
   } plans;
-  // every plan (GPU plan kernel) and every pre-zero pass up front on the caller's stream:
-  // afterwards the pieces are independent and alternate between the two compute streams
-  // (one piece's tail wave overlaps the next piece)
-  const bool det = opts && opts->deterministic;
-  for (int k = 0; k < nk; ++k) {
-    if (gnn_status_t st = gnn_plan_create(&gd, Ks[k], opts, w + l.plan[k],
-                                          gnn_plan_workspace_bytes(M, nnz, Ks[k], opts), stream,
-                                          &plans.p[k]))
+  // the host half of every plan (C*, chunk count: scalar arithmetic, no device reads); the
+  // plan kernel runs piece by piece below, as the row array arrives
+  for (int k = 0; k < nk; ++k)
+    if (gnn_status_t st = plan_create(&gd, Ks[k], opts, w + l.plan[k],
+                                      gnn_plan_workspace_bytes(M, nnz, Ks[k], opts), stream,
+                                      &plans.p[k], false))
       return st;
-    if (O_host && O_host[k] && !det && nnz > 0)
-      if (gnn_status_t st = launch_spmm_prezero(reinterpret_cast<const Plan *>(plans.p[k]), &gd,
-                                                (float *)(w + l.O[k]), Ks[k], stream))
-        return st;
+  // Pieces are ranges of nonzeros common to every width (width k takes the chunks that
+  // end inside the piece).  Deterministic plans combine split rows after the whole SpMM
+  // (fix-up pass): one piece.
+  const bool det = opts && opts->deterministic;
+  const int P = (nnz == 0 || det) ? 1 : host_pieces(nnz);
+  const bool whole = P == 1;  // whole-plan launches (pre-zero / fix-up inside)
+  // copy-in stream: every X_k first (each piece of each width gathers from all of X), then
+  // the graph piece by piece: RowInd (+ the next piece's first entry, which the plan
+  // kernel's tail flag reads), ColInd, Value
+  for (int k = 0; k < nk && N > 0; ++k) {
+    e = cudaMemcpyAsync(w + l.X[k], X_host[k], 4 * (size_t)N * Ks[k], cudaMemcpyHostToDevice,
+                        res.sin);
+    if (e != cudaSuccess) return cuda_fail(e, "gnn_run_host X upload");
   }
-  if ((e = cudaEventRecord(ev_pz, s)) == cudaSuccess) e = cudaStreamWaitEvent(res.s2, ev_pz, 0);
-  if (e != cudaSuccess) return cuda_fail(e, "gnn_run_host compute stream");
+  trace.xdone(res.sin);
+  int64_t c_prev[kMaxK] = {}, rows_done[kMaxK] = {};
   gnn_status_t st = GNN_OK;
-  int64_t piece_no = 0;
-  for (int k = 0; k < nk && st == GNN_OK; ++k) {
-    const int32_t K = Ks[k];
-    const Plan *plan = reinterpret_cast<const Plan *>(plans.p[k]);
-    const float *X = (const float *)(w + l.X[k]);
-    float *O = (float *)(w + l.O[k]), *out = (float *)(w + l.out[k]);
-    float *Oh = O_host ? O_host[k] : nullptr, *Eh = out_host ? out_host[k] : nullptr;
-    if (N > 0) {
-      e = cudaMemcpyAsync(w + l.X[k], X_host[k], 4 * (size_t)N * K, cudaMemcpyHostToDevice,
-                          res.sin);
-      if (e != cudaSuccess) { st = cuda_fail(e, "gnn_run_host X upload"); break; }
-    }
-    if ((e = cudaEventRecord(ev_x, res.sin)) == cudaSuccess) e = cudaStreamWaitEvent(s, ev_x, 0);
-    if (e == cudaSuccess) e = cudaStreamWaitEvent(res.s2, ev_x, 0);
-    if (e != cudaSuccess) { st = cuda_fail(e, "gnn_run_host event"); break; }
-    const int64_t nch = plan->info.num_chunks, C = plan->info.chunk;
-    // deterministic plans combine split rows after the whole SpMM: one piece
-    const int P = (nnz == 0 || det) ? 1 : (int)(host_pieces(nnz) < nch ? host_pieces(nnz) : nch);
-    const bool whole = P == 1;  // whole-plan launches (pre-zero / fix-up inside) when unpipelined
-    int64_t rows_done = 0;
-    for (int p = 0; p < P && st == GNN_OK; ++p, ++piece_no) {
-      const int64_t c0 = nch * p / P, c1 = nch * (p + 1) / P;
-      const int64_t b = c0 * C, en = c1 * C < nnz ? c1 * C : nnz;  // this piece's nonzeros
-      cudaStream_t sc = (piece_no & 1) ? res.s2 : s;
-      if (k == 0 && up && en > b) {  // the graph arrives with the first feature width
+  int64_t b = 0;
+  for (int p = 0; p < P && st == GNN_OK; ++p) {
+    const int64_t en = p + 1 == P ? nnz : nnz * (p + 1) / P;  // this piece: nonzeros [b, en)
+    if (up && en > b) {
+      const int64_t er = en < nnz ? en + 1 : nnz;
+      e = cudaMemcpyAsync(w + l.row_ind + 4 * b, gh->row_ind + b, 4 * (er - b),
+                          cudaMemcpyHostToDevice, res.sin);
+      if (e == cudaSuccess)
         e = cudaMemcpyAsync(w + l.col_ind + 4 * b, gh->col_ind + b, 4 * (en - b),
                             cudaMemcpyHostToDevice, res.sin);
-        if (e == cudaSuccess && gh->val)
-          e = cudaMemcpyAsync(w + l.val + 4 * b, gh->val + b, 4 * (en - b),
-                              cudaMemcpyHostToDevice, res.sin);
-        if (e == cudaSuccess) e = cudaEventRecord(ev_in, res.sin);
-        if (e == cudaSuccess) e = cudaStreamWaitEvent(sc, ev_in, 0);  // (after X_0: in order)
-        if (e != cudaSuccess) { st = cuda_fail(e, "gnn_run_host piece upload"); break; }
-      }
+      if (e == cudaSuccess && gh->val)
+        e = cudaMemcpyAsync(w + l.val + 4 * b, gh->val + b, 4 * (en - b),
+                            cudaMemcpyHostToDevice, res.sin);
+      if (e != cudaSuccess) { st = cuda_fail(e, "gnn_run_host piece upload"); break; }
+    }
+    // plan + pre-zero of this piece's chunks on the prep stream, in piece order: a row
+    // split across pieces is zeroed (by the chunk it starts in) before any later piece
+    // adds into it, and a chunk's plan entry exists before the next chunk reads it
+    trace.mark(p, 0, res.sin);
+    if ((e = cudaEventRecord(ev_in, res.sin)) == cudaSuccess)
+      e = cudaStreamWaitEvent(res.sp, ev_in, 0);
+    if (e != cudaSuccess) { st = cuda_fail(e, "gnn_run_host event"); break; }
+    int64_t c1[kMaxK];
+    for (int k = 0; k < nk && st == GNN_OK; ++k) {
+      const Plan *plan = reinterpret_cast<const Plan *>(plans.p[k]);
+      const int64_t nch = plan->info.num_chunks;
+      c1[k] = p + 1 == P ? nch : en / plan->info.chunk;
+      st = launch_plan_range(plan, res.sp, c_prev[k], c1[k]);
+      if (st == GNN_OK && O_host && O_host[k] && !whole)
+        st = launch_spmm_prezero(plan, &gd, (float *)(w + l.O[k]), Ks[k], res.sp, c_prev[k],
+                                 c1[k]);
+    }
+    if (st != GNN_OK) break;
+    cudaStream_t sc = (p & 1) ? res.s2 : s;  // pieces alternate between two compute streams
+    trace.mark(p, 1, res.sp);
+    if ((e = cudaEventRecord(ev_prep, res.sp)) == cudaSuccess)
+      e = cudaStreamWaitEvent(sc, ev_prep, 0);
+    if (e != cudaSuccess) { st = cuda_fail(e, "gnn_run_host event"); break; }
+    for (int k = 0; k < nk && st == GNN_OK; ++k) {
+      const int32_t K = Ks[k];
+      const Plan *plan = reinterpret_cast<const Plan *>(plans.p[k]);
+      const int64_t C = plan->info.chunk, c0 = c_prev[k];
+      c_prev[k] = c1[k];
+      if (!whole && c1[k] == c0) continue;
+      const float *X = (const float *)(w + l.X[k]);
+      float *O = (float *)(w + l.O[k]), *out = (float *)(w + l.out[k]);
+      float *Oh = O_host ? O_host[k] : nullptr, *Eh = out_host ? out_host[k] : nullptr;
+      const int64_t eb = c0 * C, ee = c1[k] * C < nnz ? c1[k] * C : nnz;  // its nonzeros
       if (Oh) {
         st = launch_spmm(plan, &gd, X, K, O, K, sc, GNN_F32, GNN_AGG_SUM, 0, "gnn_run_host spmm",
-                         whole ? -1 : c0, c1);
+                         whole ? -1 : c0, c1[k]);
         if (st != GNN_OK) break;
-        // rows final once pieces 0..p are done: up to this piece's last row, minus that
-        // row if it continues into the next piece (whose first chunk also zeroes the empty
-        // rows before it).  The copy-out stream waits for every piece in order.
+        // rows final once chunks [0, c1) are done: up to the last chunk's last row, minus
+        // that row if it continues into the next chunk (which also zeroes the empty rows
+        // before its first row).  The copy-out stream waits for every piece in order.
         int64_t done = M;  // (local rows: global row id - row_base)
-        if (p + 1 < P) {
-          const int32_t rl = gh->row_ind[en - 1];
-          done = (gh->row_ind[en] == rl ? rl : (int64_t)rl + 1) - r0;
+        if (ee < nnz) {
+          const int32_t rl = gh->row_ind[ee - 1];
+          done = (gh->row_ind[ee] == rl ? rl : (int64_t)rl + 1) - r0;
         }
         e = cudaEventRecord(ev_o, sc);
         if (e == cudaSuccess) e = cudaStreamWaitEvent(res.sout, ev_o, 0);
-        if (e == cudaSuccess && done > rows_done)
-          e = cudaMemcpyAsync(Oh + rows_done * K, O + rows_done * K,
-                              4 * (size_t)(done - rows_done) * K, cudaMemcpyDeviceToHost,
+        if (e == cudaSuccess && done > rows_done[k])
+          e = cudaMemcpyAsync(Oh + rows_done[k] * K, O + rows_done[k] * K,
+                              4 * (size_t)(done - rows_done[k]) * K, cudaMemcpyDeviceToHost,
                               res.sout);
         if (e != cudaSuccess) { st = cuda_fail(e, "gnn_run_host O download"); break; }
-        if (done > rows_done) rows_done = done;
+        if (done > rows_done[k]) rows_done[k] = done;
       }
-      if (Eh && en > b) {
+      if (Eh && ee > eb) {
         // A1 = the shard's own rows of X (destination rows), A2T = all of X
         st = launch_sddmm(plan, &gd, X + r0 * K, K, X, K, out, sc, GNN_F32,
-                          "gnn_run_host sddmm", whole ? -1 : c0, c1);
+                          "gnn_run_host sddmm", whole ? -1 : c0, c1[k]);
         if (st != GNN_OK) break;
         e = cudaEventRecord(ev_e, sc);
         if (e == cudaSuccess) e = cudaStreamWaitEvent(res.sout, ev_e, 0);
         if (e == cudaSuccess)
-          e = cudaMemcpyAsync(Eh + b, out + b, 4 * (size_t)(en - b), cudaMemcpyDeviceToHost,
+          e = cudaMemcpyAsync(Eh + eb, out + eb, 4 * (size_t)(ee - eb), cudaMemcpyDeviceToHost,
                               res.sout);
         if (e != cudaSuccess) { st = cuda_fail(e, "gnn_run_host S_O download"); break; }
       }
     }
+    trace.mark(p, 2, sc);
+    trace.mark(p, 3, res.sout);
+    b = en;
   }
   // the caller's stream covers every copy and kernel of this call (the copy-out stream
-  // waited for every piece; s2 is joined explicitly for calls without outputs)
+  // waited for every piece; s2, the prep and the copy-in stream are joined explicitly)
   cudaError_t e2 = cudaEventRecord(ev_done, res.sout);
   if (e2 == cudaSuccess) e2 = cudaStreamWaitEvent(s, ev_done, 0);
   if (e2 == cudaSuccess) e2 = cudaEventRecord(ev_done, res.s2);
+  if (e2 == cudaSuccess) e2 = cudaStreamWaitEvent(s, ev_done, 0);
+  if (e2 == cudaSuccess) e2 = cudaEventRecord(ev_done, res.sp);
   if (e2 == cudaSuccess) e2 = cudaStreamWaitEvent(s, ev_done, 0);
   if (e2 == cudaSuccess) e2 = cudaEventRecord(ev_done, res.sin);
   if (e2 == cudaSuccess) e2 = cudaStreamWaitEvent(s, ev_done, 0);

@@ -69,8 +69,15 @@ SparseArgs make_args(const Plan *p, const gnn_graph_t *g);
 gnn_status_t launch_spmm(const Plan *p, const gnn_graph_t *g, const void *A, int64_t lda,
                          float *O, int64_t ldo, gnn_stream_t stream, int dtype, int agg_api,
                          int accumulate, const char *who, int64_t c0, int64_t c1);
+// Pre-zero of the rows split across chunks, for the chunks [c0, c1) (c0 < 0: all).
 gnn_status_t launch_spmm_prezero(const Plan *p, const gnn_graph_t *g, float *O, int64_t ldo,
-                                 gnn_stream_t stream);
+                                 gnn_stream_t stream, int64_t c0 = -1, int64_t c1 = 0);
+// gnn_plan_create with launch = false: the host half only (C*, info, workspace views);
+// the caller fills the plan arrays with launch_plan_range as the row array arrives.
+gnn_status_t plan_create(const gnn_graph_t *g, int32_t K, const gnn_plan_opts_t *opts,
+                         void *workspace, size_t ws_bytes, gnn_stream_t stream, gnn_plan_t *out,
+                         bool launch);
+gnn_status_t launch_plan_range(const Plan *p, gnn_stream_t stream, int64_t c0, int64_t c1);
 gnn_status_t launch_sddmm(const Plan *p, const gnn_graph_t *g, const void *A1, int64_t lda1,
                           const void *A2T, int64_t lda2, float *out, gnn_stream_t stream,
                           int dtype, const char *who, int64_t c0, int64_t c1);

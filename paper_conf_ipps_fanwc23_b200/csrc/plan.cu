@@ -132,11 +132,12 @@ size_t ws_bytes_for(int64_t nch, int32_t K, int32_t deterministic) {
 
 // One thread per chunk: Algo 3 lines 2-3 (warp_start = id * NnzPerWarp, end
 // clamped to NNZ) and the node-boundary flags of the hybrid strategy.
+// Chunks [c0, c1) (the pipelined host path plans piece by piece as the row array lands).
 __global__ void plan_kernel(const int32_t *__restrict__ row_ind, int64_t nnz, int32_t C,
-                            int64_t nch, int32_t *__restrict__ row_first,
+                            int64_t c0, int64_t c1, int32_t *__restrict__ row_first,
                             int32_t *__restrict__ row_last, uint8_t *__restrict__ flags) {
-  const int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (c >= nch) return;
+  const int64_t c = c0 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= c1) return;
   const int64_t s = c * C;
   const int64_t e = s + C < nnz ? s + C : nnz;
   const int32_t rf = row_ind[s], rl = row_ind[e - 1];
@@ -153,18 +154,11 @@ __global__ void plan_kernel(const int32_t *__restrict__ row_ind, int64_t nnz, in
 
 using namespace gnn;
 
-extern "C" {
-
-GNN_API size_t gnn_plan_workspace_bytes(int64_t M, int64_t nnz, int32_t K,
-                                        const gnn_plan_opts_t *opts) {
-  gnn_plan_info_t info;
-  if (make_info(M, nnz, K, opts, &info) != GNN_OK) return (size_t)-1;
-  return ws_bytes_for(info.num_chunks, K, opts ? opts->deterministic : 0);
-}
-
-GNN_API gnn_status_t gnn_plan_create(const gnn_graph_t *g, int32_t K,
-                                     const gnn_plan_opts_t *opts, void *workspace,
-                                     size_t ws_bytes, gnn_stream_t stream, gnn_plan_t *out) {
+namespace gnn {
+// gnn_plan_create; launch = false leaves the plan arrays to launch_plan_range calls.
+gnn_status_t plan_create(const gnn_graph_t *g, int32_t K, const gnn_plan_opts_t *opts,
+                         void *workspace, size_t ws_bytes, gnn_stream_t stream, gnn_plan_t *out,
+                         bool launch) {
   if (!out) return fail(GNN_ERR_INVALID_ARG, "gnn_plan_create: out is NULL");
   *out = nullptr;
   if (!g || g->M < 0 || g->N < 0 || g->nnz < 0 || g->row_base < 0 ||
@@ -193,18 +187,44 @@ GNN_API gnn_status_t gnn_plan_create(const gnn_graph_t *g, int32_t K,
   DeviceInfo d;
   device_info(&d);
   p->device = d.device;
-  if (nch > 0) {
-    const int threads = 256;
-    plan_kernel<<<(unsigned)cdiv(nch, threads), threads, 0, (cudaStream_t)stream>>>(
-        g->row_ind, g->nnz, info.chunk, nch, p->row_first, p->row_last, p->flags);
-    cudaError_t e = cudaGetLastError();
-    if (e != cudaSuccess) {
+  if (launch && nch > 0) {
+    if (gnn_status_t st = launch_plan_range(p, stream, 0, nch)) {
       delete p;
-      return cuda_fail(e, "plan kernel launch");
+      return st;
     }
   }
   *out = reinterpret_cast<gnn_plan_t>(p);
   return GNN_OK;
+}
+
+// Plan kernel over chunks [c0, c1): reads RowInd[c0*C* - 1 .. min(c1*C*, nnz)] only.
+gnn_status_t launch_plan_range(const Plan *p, gnn_stream_t stream, int64_t c0, int64_t c1) {
+  if (c0 < 0 || c1 > p->info.num_chunks || c1 < c0)
+    return fail(GNN_ERR_INVALID_ARG, "plan: bad chunk range [%lld, %lld)", (long long)c0,
+                (long long)c1);
+  if (c1 == c0) return GNN_OK;
+  const int threads = 256;
+  plan_kernel<<<(unsigned)cdiv(c1 - c0, threads), threads, 0, (cudaStream_t)stream>>>(
+      p->row_ind, p->info.nnz, p->info.chunk, c0, c1, p->row_first, p->row_last, p->flags);
+  cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? GNN_OK : cuda_fail(e, "plan kernel launch");
+}
+
+}  // namespace gnn
+
+extern "C" {
+
+GNN_API size_t gnn_plan_workspace_bytes(int64_t M, int64_t nnz, int32_t K,
+                                        const gnn_plan_opts_t *opts) {
+  gnn_plan_info_t info;
+  if (make_info(M, nnz, K, opts, &info) != GNN_OK) return (size_t)-1;
+  return ws_bytes_for(info.num_chunks, K, opts ? opts->deterministic : 0);
+}
+
+GNN_API gnn_status_t gnn_plan_create(const gnn_graph_t *g, int32_t K,
+                                     const gnn_plan_opts_t *opts, void *workspace,
+                                     size_t ws_bytes, gnn_stream_t stream, gnn_plan_t *out) {
+  return plan_create(g, K, opts, workspace, ws_bytes, stream, out, true);
 }
 
 GNN_API gnn_status_t gnn_plan_info(gnn_plan_t plan, gnn_plan_info_t *info) {

@@ -280,12 +280,20 @@ gnn_status_t launch_spmm(const Plan *p, const gnn_graph_t *g, const void *A, int
 
 namespace gnn {
 gnn_status_t launch_spmm_prezero(const Plan *p, const gnn_graph_t *g, float *O, int64_t ldo,
-                                 gnn_stream_t stream) {
+                                 gnn_stream_t stream, int64_t c0, int64_t c1) {
   if (gnn_status_t st = check_common(p, g, "spmm prezero")) return st;
   if (p->info.num_chunks == 0) return GNN_OK;
   SparseArgs a = make_args(p, g);
+  if (c0 >= 0) {
+    if (c1 < c0 || c1 > a.num_chunks)
+      return fail(GNN_ERR_INVALID_ARG, "spmm prezero: bad chunk range [%lld, %lld)",
+                  (long long)c0, (long long)c1);
+    if (c1 == c0) return GNN_OK;
+    a.c_begin = c0;
+    a.c_end = c1;
+  }
   const int VW = p->info.vw_feat, VO = VW < 8 ? VW : 8;
-  const int64_t blocks = (a.num_chunks * 32 + 255) / 256;
+  const int64_t blocks = ((a.c_end - a.c_begin) * 32 + 255) / 256;
   cudaStream_t s = (cudaStream_t)stream;
   switch (VO) {
     case 1: spmm_prezero_kernel<1><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, 0.f); break;

@@ -548,6 +548,15 @@ def test_run_host_pipelined_pieces(pieces):
     _run_host_check(g2, (8, 32, 128), pieces)
 
 
+@pytest.mark.parametrize("chunk", [1000, 4096])
+def test_run_host_pieces_smaller_than_chunks(chunk):
+    """Pieces are ranges of nonzeros common to every width and a width takes the chunks
+    that end inside a piece: with chunks longer than a piece, some pieces run no chunk of
+    that width, and a chunk's plan entry (tail flag) reads the first row of the next piece."""
+    g = configs.make_graph("C2")
+    _run_host_check(g, (32, 64), 32, opts={"force_chunk": chunk})
+
+
 def test_run_host_pipelined_deterministic_and_no_values():
     """Deterministic plans run unpipelined; a NULL value array means all ones."""
     g = configs.make_graph("C2")

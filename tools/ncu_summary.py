@@ -1,6 +1,8 @@
 """Summarise `ncu --set full` reports into profiles/ (run here, without a GPU).
 
-    python tools/ncu_summary.py TAG WORKLOAD rep1.ncu-rep [rep2.ncu-rep ...]
+    python tools/ncu_summary.py TAG WORKLOAD rep1.ncu-rep|rep1.csv [...]
+
+(a .csv is the `ncu -i rep --page raw --csv` export, for reports too large to bring back)
 
 Writes profiles/<TAG>_ncu_full.json (key counters per launch) and merges the DRAM
 traffic per launch into profiles/ncu_traffic.json (read by bench.py's roofline
@@ -25,13 +27,19 @@ KEYS = ['Kernel Name', 'gpu__time_duration.sum', 'dram__bytes_read.sum', 'dram__
         'smsp__average_warps_issue_stalled_long_scoreboard_per_issue_active.ratio',
         'smsp__average_warps_issue_stalled_wait_per_issue_active.ratio',
         'smsp__inst_executed.sum', 'sm__cycles_elapsed.avg.per_second', 'launch__grid_size',
-        'launch__occupancy_limit_registers']
+        'launch__occupancy_limit_registers', 'lts__throughput.avg.pct_of_peak_sustained_elapsed',
+        'lts__t_sectors_srcunit_tex.sum.pct_of_peak_sustained_elapsed',
+        'l1tex__throughput.avg.pct_of_peak_sustained_elapsed',
+        'l1tex__data_pipe_lsu_wavefronts.avg.pct_of_peak_sustained_elapsed']
 SCALE = {'byte': 1, 'Kbyte': 1e3, 'Mbyte': 1e6, 'Gbyte': 1e9, 'Tbyte': 1e12}
 
 
 def rows_of(rep):
-    out = subprocess.run(['ncu', '-i', rep, '--page', 'raw', '--csv'], capture_output=True,
-                         text=True).stdout
+    if rep.endswith('.csv'):  # `ncu -i rep --page raw --csv` exported on the GPU box
+        out = open(rep).read()
+    else:
+        out = subprocess.run(['ncu', '-i', rep, '--page', 'raw', '--csv'], capture_output=True,
+                             text=True).stdout
     rows = list(csv.reader(io.StringIO(out)))
     h, u = rows[0], rows[1]
     for r in rows[2:]:
@@ -43,7 +51,13 @@ def rows_of(rep):
 
 
 def main():
-    tag, workload, reps = sys.argv[1], sys.argv[2], sys.argv[3:]
+    args = sys.argv[1:]
+    ks = None  # --ks 32,32,64,...: K of each spmm/sddmm launch in report order
+    if '--ks' in args:
+        i = args.index('--ks')
+        ks = [int(x) for x in args[i + 1].split(',')]
+        del args[i:i + 2]
+    tag, workload, reps = args[0], args[1], args[2:]
     summ = []
     traffic_path = os.path.join(ROOT, 'profiles', 'ncu_traffic.json')
     traffic = json.load(open(traffic_path)) if os.path.exists(traffic_path) else {}
@@ -62,8 +76,14 @@ def main():
                 rec['report'] = os.path.basename(rep)
                 # K is recorded by tools/profile_one.py order; store by kernel name too
                 rec['kind'] = kind
+                if ks is not None:
+                    K = ks[sum(1 for r in summ if 'kind' in r)]
+                    rec['K'] = K
+                    traffic[f"{workload}:{kind}:K{K}"] = int(b)
             summ.append(rec)
     json.dump(summ, open(os.path.join(ROOT, 'profiles', f'{tag}_ncu_full.json'), 'w'), indent=1)
+    if ks is not None:
+        json.dump(traffic, open(traffic_path, 'w'), indent=1)
     print(json.dumps(summ, indent=1)[:3000])
 
 
