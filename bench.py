@@ -208,7 +208,7 @@ def parse_ks(s, name):
 
 
 # ------------------------------------------------------------ our impl ------
-def time_path(args, g, perm, name, Ks, dev, world, rank, dtype="f32"):
+def time_path(args, g, perm, name, Ks, dev, world, rank, dtype="f32", xmode=None):
     """Resident graph + features for this rank's shard; W warm-up steps, then K timed
     steps (CUDA events per kernel on the launching stream, L2 flushed between steps
     outside the events).  Returns per-kernel times, this rank's bytes/flops, launches."""
@@ -220,16 +220,17 @@ def time_path(args, g, perm, name, Ks, dev, world, rank, dtype="f32"):
     from paper_conf_ipps_fanwc23_b200 import dist as gdist
 
     P = world
+    xm = xmode or xm
     spec = gdist.shard_spec(g.row_ptr, g.N, rank, world)
     full = gs.DeviceGraph.from_arrays(g.M, g.N, g.row_ind, g.col_ind, g.val, g.row_ptr, device=dev)
     spg, sdg = gdist.local_graphs(full, spec)
     perm_d = None if perm is None else torch.from_numpy(perm).to(dev)
     X, Xown, ov = {}, {}, {}
-    overlap = args.xmode == "overlap" and P > 1
+    overlap = xm == "overlap" and P > 1
     for K in Ks:
         if overlap:  # f1: per-block broadcasts overlapped with column-block SpMM
             ov[K] = gdist.OverlappedSpMM(g.row_ind, g.col_ind, g.val, spec, K, dev)
-        if args.xmode in ("allgather", "overlap") and P > 1:
+        if xm in ("allgather", "overlap") and P > 1:
             own = configs.make_features(name, spec.x1 - spec.x0, K, row0=spec.x0)
             Xown[K] = torch.zeros((spec.xblk, K), dtype=torch.float32, device=dev)
             Xown[K][:own.shape[0]] = torch.from_numpy(own).to(dev)
@@ -256,7 +257,7 @@ def time_path(args, g, perm, name, Ks, dev, world, rank, dtype="f32"):
         for K in Ks:
             if ev is not None:
                 ev[K][4].record(stream)  # step start: the X exchange is inside the step
-            if args.xmode == "allgather" and P > 1:
+            if xm == "allgather" and P > 1:
                 gdist.gather_features(Xown[K], spec, g.N, out=X[K])
             if ev is not None:
                 ev[K][0].record(stream)
@@ -340,6 +341,11 @@ def time_path(args, g, perm, name, Ks, dev, world, rank, dtype="f32"):
            "detail": detail, "clocks": clocks, "launches": counts["n"], "spg": spg, "sdg": sdg,
            "full": full}
     return out
+
+
+def gdist_spec(g, rank, world):
+    from paper_conf_ipps_fanwc23_b200 import dist as gdist
+    return gdist.shard_spec(g.row_ptr, g.N, rank, world)
 
 
 def init_dist(world, local):
@@ -455,6 +461,32 @@ def run_ours(args):
                "ms_per_step": round(ms2 / args.steps, 4), "kernels": r2["detail"]}
         del r2
         torch.cuda.empty_cache()
+    exchange = None
+    if world > 1 and args.xmode == "replicate" and args.exchange:
+        # SURVEY §8(e)/(f1) at N ranks: X all-gathered (NCCL) inside the step, and the
+        # per-owner-block broadcasts overlapped with column-block SpMM, on the graph as
+        # generated (the exchange modes keep X in its original row order)
+        exchange = {}
+        for xm in ("allgather", "overlap"):
+            torch.cuda.empty_cache()
+            try:
+                rx = time_path(args, g0, None, name, Ks, dev, world, rank, xmode=xm)
+                msx, bx, _ = aggregate(rx, args, world, dev)
+                spec = gdist_spec(g0, rank, world)
+                comm = {f"K{K}": rx["detail"][f"K{K}"]["comm_ms"] for K in Ks}
+                exchange[xm] = {"value": round(bx / (msx * 1e-3) / 1e9, 2), "unit": "GB/s",
+                                "ms_per_step": round(msx / args.steps, 4),
+                                "kernels": rx["detail"]}
+                if xm == "allgather":  # nccl-tests style bus bandwidth of the X all-gather
+                    exchange[xm]["allgather_busbw_GBps"] = {
+                        f"K{K}": round(4 * K * spec.xblk * world * (world - 1) / world
+                                       / (comm[f"K{K}"] * 1e-3) / 1e9, 1)
+                        for K in Ks if comm[f"K{K}"] > 0}
+                del rx
+            except Exception as ex:  # report, never lose the main line
+                exchange[xm] = {"error": f"{type(ex).__name__}: {ex}"[:300]}
+        exchange["note"] = ("graph as generated (no reorder); compare with no_reorder "
+                            "(X replicated, same graph)")
     e2e = None
     if not args.no_e2e:
         e2e = run_e2e(args, g, Ks, dev, perm, world, rank)
@@ -479,7 +511,7 @@ def run_ours(args):
             "gflops": round(tot_flops / (tot_ms * 1e-3) / 1e9, 1),
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": launches * args.steps, "clocks": clocks, "kernels": detail,
-            "no_reorder": alt, "bf16": bf16,
+            "no_reorder": alt, "bf16": bf16, "exchange": exchange,
         }
         print(json.dumps(line), flush=True)
     if world > 1:
@@ -562,14 +594,18 @@ def run_c3(args, dev, world, rank):
     clk.start()
     time.sleep(0.3)
     nbytes, pl, sp, sd, chunks = 0, [], [], [], []
+    # eager, as a training loop runs it: no host sync between steps (the host enqueues
+    # ahead of the device, so launch overhead overlaps the previous step); the L2 flush
+    # between steps is on the stream but outside the events
+    torch.cuda.synchronize()
     for s in range(nsteps):
         flush.fill_(float(s))
-        torch.cuda.synchronize()
         p = one(s, evs[s])
-        torch.cuda.synchronize()
         g = subs[s % len(subs)][0]
         nbytes += spmm_bytes(g.nnz, g.M, K) + sddmm_bytes(g.nnz, g.M, K)
         chunks.append(p.info()["chunk"])
+    torch.cuda.synchronize()
+    for s in range(nsteps):
         e = evs[s]
         pl.append(e[0].elapsed_time(e[1]))
         sp.append(e[1].elapsed_time(e[2]))
@@ -780,6 +816,9 @@ def main():
                          "the paper's full-graph setup)")
     ap.add_argument("--no-bf16", dest="bf16", action="store_false",
                     help="skip the extra timing with bf16 feature storage")
+    ap.add_argument("--no-exchange", dest="exchange", action="store_false",
+                    help="at N > 1, skip the extra timings with X all-gathered / broadcast "
+                         "per block inside the step")
     ap.add_argument("--no-compare", dest="compare", action="store_false",
                     help="skip the extra timing of the un-reordered graph")
     args = ap.parse_args()

@@ -1,12 +1,13 @@
 // host_api.cu -- the end-to-end entry point on HOST buffers (bench.py's e2e path): the
 // caller hands host arrays and one device workspace; the library copies the graph and X
 // in, plans (GPU plan kernel), runs SpMM and SDDMM, and copies O and S_O out.
-// Pipelined over pieces of the nonzeros: X of every width uploads first, then the graph
-// piece by piece (copy-in stream); each piece is planned (plan kernel over its chunks +
-// pre-zero, prep stream) and computed for every width (two alternating compute streams)
-// while the next piece uploads and the finished rows / edge values of the previous one
-// download (copy-out stream).  PCIe is full duplex, so the call costs about
-// max(upload, compute, download) plus the X upload instead of their sum.
+// Pipelined over pieces of the nonzeros.  Copy-in stream: X_0, piece 0, X_1, piece 1, ...
+// (a piece = RowInd/ColInd/Value of a range of nonzeros common to every width); prep
+// stream: each piece is planned (plan kernel over the chunks that end inside it) and its
+// split rows pre-zeroed, in piece order; two alternating compute streams: SpMM + SDDMM of
+// every width whose X has landed (a width catches up on earlier pieces when its X lands);
+// copy-out stream: each unit's S_O entries and the O rows that became final.  PCIe is
+// full duplex, so the call costs about max(upload, compute, download) instead of their sum.
 #include <cuda_runtime.h>
 #include <stdio.h>
 #include <stdlib.h>
@@ -109,7 +110,7 @@ struct Trace {
       if (e) cudaEventElapsedTime(&t, t0, e);
       return t;
     };
-    fprintf(stderr, "gnn_run_host trace: X uploaded %.3f ms\n", ms(tx));
+    fprintf(stderr, "gnn_run_host trace: copy-in done %.3f ms\n", ms(tx));
     for (int p = 0; p < n; ++p)
       fprintf(stderr, "  piece %2d: in %.3f  planned %.3f  computed %.3f  out %.3f\n", p,
               ms(ev[p][0]), ms(ev[p][1]), ms(ev[p][2]), ms(ev[p][3]));
@@ -174,13 +175,13 @@ GNN_API gnn_status_t gnn_run_host_multi(const gnn_graph_t *gh, int32_t upload_gr
   // record at the time it is enqueued, so a fixed set serves the whole call.
   CallResources res;
   Trace trace;  // declared after res: reported before the streams are released
-  cudaEvent_t ev_entry, ev_done, ev_prep, ev_in, ev_o, ev_e;
+  cudaEvent_t ev_entry, ev_done, ev_prep, ev_in, ev_o, ev_e, ev_x;
   cudaError_t e = cudaStreamCreateWithFlags(&res.sin, cudaStreamNonBlocking);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&res.sout, cudaStreamNonBlocking);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&res.s2, cudaStreamNonBlocking);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&res.sp, cudaStreamNonBlocking);
-  cudaEvent_t *evs[6] = {&ev_entry, &ev_done, &ev_prep, &ev_in, &ev_o, &ev_e};
-  for (int i = 0; i < 6 && e == cudaSuccess; ++i) e = res.event(evs[i]);
+  cudaEvent_t *evs[7] = {&ev_entry, &ev_done, &ev_prep, &ev_in, &ev_o, &ev_e, &ev_x};
+  for (int i = 0; i < 7 && e == cudaSuccess; ++i) e = res.event(evs[i]);
   // everything earlier on the caller's stream (e.g. the previous call still reading this
   // workspace) happens before this call's copies
   if (e == cudaSuccess) e = cudaEventRecord(ev_entry, s);
@@ -215,19 +216,89 @@ GNN_API gnn_status_t gnn_run_host_multi(const gnn_graph_t *gh, int32_t upload_gr
   const bool det = opts && opts->deterministic;
   const int P = (nnz == 0 || det) ? 1 : host_pieces(nnz);
   const bool whole = P == 1;  // whole-plan launches (pre-zero / fix-up inside)
-  // copy-in stream: every X_k first (each piece of each width gathers from all of X), then
-  // the graph piece by piece: RowInd (+ the next piece's first entry, which the plan
-  // kernel's tail flag reads), ColInd, Value
-  for (int k = 0; k < nk && N > 0; ++k) {
-    e = cudaMemcpyAsync(w + l.X[k], X_host[k], 4 * (size_t)N * Ks[k], cudaMemcpyHostToDevice,
-                        res.sin);
-    if (e != cudaSuccess) return cuda_fail(e, "gnn_run_host X upload");
+  // Chunk range of width k in piece p: the chunks that end inside the piece's nonzeros.
+  int64_t cb[kMaxK][kMaxPieces + 1];
+  for (int k = 0; k < nk; ++k) {
+    const Plan *plan = reinterpret_cast<const Plan *>(plans.p[k]);
+    cb[k][0] = 0;
+    for (int p = 0; p < P; ++p)
+      cb[k][p + 1] = p + 1 == P ? plan->info.num_chunks : (nnz * (p + 1) / P) / plan->info.chunk;
   }
-  trace.xdone(res.sin);
-  int64_t c_prev[kMaxK] = {}, rows_done[kMaxK] = {};
+  int64_t rows_done[kMaxK] = {};
+  int units = 0;  // (width, piece) work units so far: they alternate between two streams
+  // SpMM + SDDMM of width k on piece p, then the downloads of what became final.  The
+  // stream first waits for the latest prep record (covers pieces 0..p, enqueued in piece
+  // order) and, for a width whose X landed after the piece, the latest X record.
+  auto compute = [&](int k, int p, bool wait_x, cudaEvent_t ev_x) -> gnn_status_t {
+    const int32_t K = Ks[k];
+    const Plan *plan = reinterpret_cast<const Plan *>(plans.p[k]);
+    const int64_t C = plan->info.chunk, c0 = cb[k][p], c1 = cb[k][p + 1];
+    if (!whole && c1 == c0) return GNN_OK;
+    cudaStream_t sc = (units++ & 1) ? res.s2 : s;
+    cudaError_t e = cudaStreamWaitEvent(sc, ev_prep, 0);
+    if (e == cudaSuccess && wait_x) e = cudaStreamWaitEvent(sc, ev_x, 0);
+    if (e != cudaSuccess) return cuda_fail(e, "gnn_run_host event");
+    const float *X = (const float *)(w + l.X[k]);
+    float *O = (float *)(w + l.O[k]), *out = (float *)(w + l.out[k]);
+    float *Oh = O_host ? O_host[k] : nullptr, *Eh = out_host ? out_host[k] : nullptr;
+    const int64_t eb = c0 * C, ee = c1 * C < nnz ? c1 * C : nnz;  // its nonzeros
+    if (Oh) {
+      if (gnn_status_t st = launch_spmm(plan, &gd, X, K, O, K, sc, GNN_F32, GNN_AGG_SUM, 0,
+                                        "gnn_run_host spmm", whole ? -1 : c0, c1))
+        return st;
+      // rows final once chunks [0, c1) are done: up to the last chunk's last row, minus
+      // that row if it continues into the next chunk (which also zeroes the empty rows
+      // before its first row).  The copy-out stream waits for every unit of a width in
+      // piece order, so the earlier pieces (on the other stream) are done too.
+      int64_t done = M;  // (local rows: global row id - row_base)
+      if (ee < nnz) {
+        const int32_t rl = gh->row_ind[ee - 1];
+        done = (gh->row_ind[ee] == rl ? rl : (int64_t)rl + 1) - r0;
+      }
+      e = cudaEventRecord(ev_o, sc);
+      if (e == cudaSuccess) e = cudaStreamWaitEvent(res.sout, ev_o, 0);
+      if (e == cudaSuccess && done > rows_done[k])
+        e = cudaMemcpyAsync(Oh + rows_done[k] * K, O + rows_done[k] * K,
+                            4 * (size_t)(done - rows_done[k]) * K, cudaMemcpyDeviceToHost,
+                            res.sout);
+      if (e != cudaSuccess) return cuda_fail(e, "gnn_run_host O download");
+      if (done > rows_done[k]) rows_done[k] = done;
+    }
+    if (Eh && ee > eb) {
+      // A1 = the shard's own rows of X (destination rows), A2T = all of X
+      if (gnn_status_t st = launch_sddmm(plan, &gd, X + r0 * K, K, X, K, out, sc, GNN_F32,
+                                         "gnn_run_host sddmm", whole ? -1 : c0, c1))
+        return st;
+      e = cudaEventRecord(ev_e, sc);
+      if (e == cudaSuccess) e = cudaStreamWaitEvent(res.sout, ev_e, 0);
+      if (e == cudaSuccess)
+        e = cudaMemcpyAsync(Eh + eb, out + eb, 4 * (size_t)(ee - eb), cudaMemcpyDeviceToHost,
+                            res.sout);
+      if (e != cudaSuccess) return cuda_fail(e, "gnn_run_host S_O download");
+    }
+    return GNN_OK;
+  };
+  // X_k (width k, all N rows) uploads on the copy-in stream; width k then catches up on
+  // the pieces that landed before it
+  auto upload_x = [&](int k, int pieces_in) -> gnn_status_t {
+    if (N > 0) {
+      cudaError_t e = cudaMemcpyAsync(w + l.X[k], X_host[k], 4 * (size_t)N * Ks[k],
+                                      cudaMemcpyHostToDevice, res.sin);
+      if (e == cudaSuccess) e = cudaEventRecord(ev_x, res.sin);
+      if (e != cudaSuccess) return cuda_fail(e, "gnn_run_host X upload");
+    }
+    for (int q = 0; q < pieces_in; ++q)
+      if (gnn_status_t st = compute(k, q, N > 0, ev_x)) return st;
+    return GNN_OK;
+  };
+  // Copy-in order X_0, piece 0, X_1, piece 1, ...: the copy-out stream gets width 0's
+  // first results after X_0 + one piece instead of after every X (PCIe is duplex, and the
+  // downloads are the longer direction).  Pieces: RowInd (+ the next piece's first
+  // entry, which the plan kernel's tail flag reads), ColInd, Value.
   gnn_status_t st = GNN_OK;
   int64_t b = 0;
   for (int p = 0; p < P && st == GNN_OK; ++p) {
+    if (p < nk && (st = upload_x(p, p)) != GNN_OK) break;
     const int64_t en = p + 1 == P ? nnz : nnz * (p + 1) / P;  // this piece: nonzeros [b, en)
     if (up && en > b) {
       const int64_t er = en < nnz ? en + 1 : nnz;
@@ -248,70 +319,27 @@ GNN_API gnn_status_t gnn_run_host_multi(const gnn_graph_t *gh, int32_t upload_gr
     if ((e = cudaEventRecord(ev_in, res.sin)) == cudaSuccess)
       e = cudaStreamWaitEvent(res.sp, ev_in, 0);
     if (e != cudaSuccess) { st = cuda_fail(e, "gnn_run_host event"); break; }
-    int64_t c1[kMaxK];
     for (int k = 0; k < nk && st == GNN_OK; ++k) {
       const Plan *plan = reinterpret_cast<const Plan *>(plans.p[k]);
-      const int64_t nch = plan->info.num_chunks;
-      c1[k] = p + 1 == P ? nch : en / plan->info.chunk;
-      st = launch_plan_range(plan, res.sp, c_prev[k], c1[k]);
+      st = launch_plan_range(plan, res.sp, cb[k][p], cb[k][p + 1]);
       if (st == GNN_OK && O_host && O_host[k] && !whole)
-        st = launch_spmm_prezero(plan, &gd, (float *)(w + l.O[k]), Ks[k], res.sp, c_prev[k],
-                                 c1[k]);
+        st = launch_spmm_prezero(plan, &gd, (float *)(w + l.O[k]), Ks[k], res.sp, cb[k][p],
+                                 cb[k][p + 1]);
     }
     if (st != GNN_OK) break;
-    cudaStream_t sc = (p & 1) ? res.s2 : s;  // pieces alternate between two compute streams
     trace.mark(p, 1, res.sp);
-    if ((e = cudaEventRecord(ev_prep, res.sp)) == cudaSuccess)
-      e = cudaStreamWaitEvent(sc, ev_prep, 0);
-    if (e != cudaSuccess) { st = cuda_fail(e, "gnn_run_host event"); break; }
-    for (int k = 0; k < nk && st == GNN_OK; ++k) {
-      const int32_t K = Ks[k];
-      const Plan *plan = reinterpret_cast<const Plan *>(plans.p[k]);
-      const int64_t C = plan->info.chunk, c0 = c_prev[k];
-      c_prev[k] = c1[k];
-      if (!whole && c1[k] == c0) continue;
-      const float *X = (const float *)(w + l.X[k]);
-      float *O = (float *)(w + l.O[k]), *out = (float *)(w + l.out[k]);
-      float *Oh = O_host ? O_host[k] : nullptr, *Eh = out_host ? out_host[k] : nullptr;
-      const int64_t eb = c0 * C, ee = c1[k] * C < nnz ? c1[k] * C : nnz;  // its nonzeros
-      if (Oh) {
-        st = launch_spmm(plan, &gd, X, K, O, K, sc, GNN_F32, GNN_AGG_SUM, 0, "gnn_run_host spmm",
-                         whole ? -1 : c0, c1[k]);
-        if (st != GNN_OK) break;
-        // rows final once chunks [0, c1) are done: up to the last chunk's last row, minus
-        // that row if it continues into the next chunk (which also zeroes the empty rows
-        // before its first row).  The copy-out stream waits for every piece in order.
-        int64_t done = M;  // (local rows: global row id - row_base)
-        if (ee < nnz) {
-          const int32_t rl = gh->row_ind[ee - 1];
-          done = (gh->row_ind[ee] == rl ? rl : (int64_t)rl + 1) - r0;
-        }
-        e = cudaEventRecord(ev_o, sc);
-        if (e == cudaSuccess) e = cudaStreamWaitEvent(res.sout, ev_o, 0);
-        if (e == cudaSuccess && done > rows_done[k])
-          e = cudaMemcpyAsync(Oh + rows_done[k] * K, O + rows_done[k] * K,
-                              4 * (size_t)(done - rows_done[k]) * K, cudaMemcpyDeviceToHost,
-                              res.sout);
-        if (e != cudaSuccess) { st = cuda_fail(e, "gnn_run_host O download"); break; }
-        if (done > rows_done[k]) rows_done[k] = done;
-      }
-      if (Eh && ee > eb) {
-        // A1 = the shard's own rows of X (destination rows), A2T = all of X
-        st = launch_sddmm(plan, &gd, X + r0 * K, K, X, K, out, sc, GNN_F32,
-                          "gnn_run_host sddmm", whole ? -1 : c0, c1[k]);
-        if (st != GNN_OK) break;
-        e = cudaEventRecord(ev_e, sc);
-        if (e == cudaSuccess) e = cudaStreamWaitEvent(res.sout, ev_e, 0);
-        if (e == cudaSuccess)
-          e = cudaMemcpyAsync(Eh + eb, out + eb, 4 * (size_t)(ee - eb), cudaMemcpyDeviceToHost,
-                              res.sout);
-        if (e != cudaSuccess) { st = cuda_fail(e, "gnn_run_host S_O download"); break; }
-      }
+    if ((e = cudaEventRecord(ev_prep, res.sp)) != cudaSuccess) {
+      st = cuda_fail(e, "gnn_run_host event");
+      break;
     }
-    trace.mark(p, 2, sc);
+    // every width whose X has landed (X_k precedes piece k on the copy-in stream)
+    for (int k = 0; k < nk && k <= p && st == GNN_OK; ++k) st = compute(k, p, false, ev_x);
+    trace.mark(p, 2, (units & 1) ? s : res.s2);
     trace.mark(p, 3, res.sout);
     b = en;
   }
+  for (int k = P; k < nk && st == GNN_OK; ++k) st = upload_x(k, P);  // fewer pieces than widths
+  trace.xdone(res.sin);
   // the caller's stream covers every copy and kernel of this call (the copy-out stream
   // waited for every piece; s2, the prep and the copy-in stream are joined explicitly)
   cudaError_t e2 = cudaEventRecord(ev_done, res.sout);
