@@ -145,6 +145,12 @@ class ClockSampler:
                 stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
         except Exception:
             self.proc = None
+            return
+        # nvidia-smi takes a moment to start: wait (up to 3 s) for its first sample so the
+        # timed region that follows is covered
+        t0 = time.time()
+        while time.time() - t0 < 3.0 and os.path.getsize(self.path) == 0:
+            time.sleep(0.05)
 
     def stop(self):
         if self.proc is None:
@@ -220,7 +226,7 @@ def time_path(args, g, perm, name, Ks, dev, world, rank, dtype="f32", xmode=None
     from paper_conf_ipps_fanwc23_b200 import dist as gdist
 
     P = world
-    xm = xmode or xm
+    xm = xmode or args.xmode
     spec = gdist.shard_spec(g.row_ptr, g.N, rank, world)
     full = gs.DeviceGraph.from_arrays(g.M, g.N, g.row_ind, g.col_ind, g.val, g.row_ptr, device=dev)
     spg, sdg = gdist.local_graphs(full, spec)
@@ -565,7 +571,9 @@ def run_c3(args, dev, world, rank):
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
-    nsteps = args.steps
+    # a C3 step is ~0.1 ms: time enough of them (>= 4000, cycling over the resident
+    # subgraphs) for the clock sampler to see the timed region
+    nsteps = max(args.steps, 4000)
 
     # CUDA-graph variant: each subgraph's plan + SpMM + SDDMM captured once, replayed per
     # step (the plan kernel re-runs on every replay; only host launch overhead disappears)
