@@ -38,6 +38,9 @@ __device__ __forceinline__ uint64_t l2_evict_last() {
 #ifndef GNN_USE_FFMA2
 #define GNN_USE_FFMA2 1
 #endif
+#ifndef GNN_BF16_FHFMA
+#define GNN_BF16_FHFMA 1  // bf16 dot products (SDDMM) on the mixed-precision FMA
+#endif
 
 // ------------------------------------------------------------ features ----
 template <int VW>
@@ -248,6 +251,25 @@ __device__ __forceinline__ void axpy_f(float (&acc)[VW], float s, const FeatVec<
 template <typename TF, int VW>
 __device__ __forceinline__ float dot_f(float d, const FeatVec<TF, VW> &a,
                                        const FeatVec<TF, VW> &x) {
+#if GNN_BF16_FHFMA
+  if constexpr (std::is_same<TF, BF16>::value && VW >= 4) {
+    // bf16 x bf16 products accumulated in fp32 by the mixed-precision FMA (FHFMA.BF16,
+    // half selectors straight from the packed words): no widening instructions.  The
+    // product of two bf16 values is exact in fp32, so e0 / e1 (even / odd elements) round
+    // exactly like the FFMA2 pair chains on widened operands below: identical results.
+    float e0 = 0.f, e1 = 0.f;
+#pragma unroll
+    for (int w = 0; w < VW / 2; ++w)
+      asm("{.reg .b16 al, ah, xl, xh;\n\t"
+          "mov.b32 {al, ah}, %2;\n\t"
+          "mov.b32 {xl, xh}, %3;\n\t"
+          "fma.rn.f32.bf16 %0, al, xl, %0;\n\t"
+          "fma.rn.f32.bf16 %1, ah, xh, %1;}"
+          : "+f"(e0), "+f"(e1)
+          : "r"(a.r[w]), "r"(x.r[w]));
+    return d + (e0 + e1);
+  }
+#endif
 #if GNN_USE_FFMA2
   if constexpr (VW >= 4) {
     float e0 = 0.f, e1 = 0.f;

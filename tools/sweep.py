@@ -44,7 +44,8 @@ if REORDER:
     res["modularity"] = q
 dg = gs.DeviceGraph.from_arrays(g.M, g.N, g.row_ind, g.col_ind, g.val, g.row_ptr)
 flush = torch.empty(64 * 1024 * 1024, device="cuda")
-for K, fvw in [(k, 0) for k in KS] + [(k, 8) for k in KS if VW8 and k % 8 == 0 and k < 256]:
+for K, fvw in ([(k, 0) for k in KS] + [(k, 8) for k in KS if VW8 and k % 8 == 0 and k < 256]
+                + [(k, ALTVW) for k in KS if ALTVW and k % ALTVW == 0]):
     X = torch.from_numpy(configs.make_features(WL, g.N, K)).cuda()
     if perm is not None:
         X = gs.permute_rows(X, torch.from_numpy(perm))
@@ -60,7 +61,7 @@ for K, fvw in [(k, 0) for k in KS] + [(k, 8) for k in KS if VW8 and k % 8 == 0 a
         torch.cuda.synchronize()
         if it >= 2:
             ts.append(a.elapsed_time(b)); td.append(b.elapsed_time(c))
-    res[f"K{K}" + ("_vw8" if fvw else "")] = {"spmm_ms": round(min(ts), 4), "sddmm_ms": round(min(td), 4),
+    res[f"K{K}" + (f"_vw{fvw}" if fvw else "")] = {"spmm_ms": round(min(ts), 4), "sddmm_ms": round(min(td), 4),
                     "spmm_med": round(sorted(ts)[len(ts)//2], 4), "info": {k: p.info()[k] for k in ("chunk", "active_blocks_per_sm")}}
 print("RESULT " + json.dumps(res), flush=True)
 '''
@@ -72,13 +73,15 @@ def main():
     ap.add_argument("--K", default="32,64,128,256")
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--vw8", action="store_true")
+    ap.add_argument("--alt-vw", type=int, default=0,
+                    help="also time every K with force_vw = this (elements per feature load)")
     ap.add_argument("--reorder", action="store_true")
     ap.add_argument("--dtype", default="f32", choices=["f32", "bf16"])
     ap.add_argument("--force-chunk", type=int, default=0)
     ap.add_argument("libs", nargs="+")
     a = ap.parse_args()
     code = CHILD.replace("ROOT", repr(ROOT)).replace("WL", repr(a.workload)).replace(
-        "KS", repr([int(k) for k in a.K.split(",")])).replace("REPS", str(a.reps)).replace("VW8", str(a.vw8)).replace("REORDER", str(a.reorder)).replace("DTYPE", repr(a.dtype)).replace("FCHUNK", str(a.force_chunk))
+        "KS", repr([int(k) for k in a.K.split(",")])).replace("REPS", str(a.reps)).replace("VW8", str(a.vw8)).replace("REORDER", str(a.reorder)).replace("DTYPE", repr(a.dtype)).replace("FCHUNK", str(a.force_chunk)).replace("ALTVW", str(a.alt_vw))
     for lib in a.libs:
         env = dict(os.environ, GNN_LIB_PATH=os.path.abspath(lib))
         r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
