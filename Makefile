@@ -37,7 +37,13 @@ variant: $(OBJS)
 	$(NVCC) $(ARCH) -shared -cudart static -o build/libgnnsparse_$(TAG).so $(OBJS)
 	cat $(OBJDIR)/*.ptxas.log > build/ptxas_$(TAG).log
 
+# measurement probes (tools/microbench.py), not part of the product
+micro: build/libgnnmicro.so
+build/libgnnmicro.so: tools/microbench.cu
+	@mkdir -p build
+	$(NVCC) $(ARCH) -O3 -shared -Xcompiler -fPIC -o $@ $<
+
 clean:
 	rm -rf gen/libgnngen.so oracle/liboracle.so $(PKG)/libgnnsparse.so build/obj*
 
-.PHONY: all clean variant
+.PHONY: all clean variant micro

@@ -18,7 +18,7 @@ namespace gnn {
 constexpr unsigned kFull = 0xffffffffu;
 
 #ifndef GNN_SPARSE_EVICT_FIRST
-#define GNN_SPARSE_EVICT_FIRST 0  // L2 evict_first hint on the streamed sparse arrays
+#define GNN_SPARSE_EVICT_FIRST 1  // L2 evict_first hint on the streamed sparse arrays
 #endif
 #ifndef GNN_FEAT_EVICT_LAST
 #define GNN_FEAT_EVICT_LAST 0     // L2 evict_last hint on gathered feature rows
@@ -353,9 +353,16 @@ template <int BYTES>
 __device__ __forceinline__ void cp_async(void *smem_dst, const void *gsrc, int src_bytes) {
   const uint32_t d = (uint32_t)__cvta_generic_to_shared(smem_dst);
   if constexpr (BYTES == 16) {
+#if GNN_SPARSE_EVICT_FIRST
+    // streamed once: ask L2 to evict these lines first (keeps the gathered rows of X)
+    asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2, %3;" ::"r"(d),
+                 "l"(gsrc), "r"(src_bytes), "l"(l2_evict_first())
+                 : "memory");
+#else
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(d), "l"(gsrc),
                  "r"(src_bytes)
                  : "memory");
+#endif
   } else {
     asm volatile("cp.async.ca.shared.global [%0], [%1], %2, %3;" ::"r"(d), "l"(gsrc),
                  "n"(BYTES), "r"(src_bytes)

@@ -3,6 +3,8 @@
 //              operation SpMM/SDDMM are built from, with no sparse values, rows or
 //              stores: a lane group of L = K/VW lanes per row, U rows in flight/lane.
 //   mb_copy  : streaming copy (HBM read+write).
+//   mb_shfl  : warp-shuffle issue rate (8 independent xor-shuffle chains per thread):
+//              the cost of a shuffle-based segmented reduction in SpMM.
 // Not part of the product ABI (built into build/libgnnmicro.so).
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -52,7 +54,25 @@ __global__ void copy_kernel(const float4 *__restrict__ a, float4 *__restrict__ b
     b[i] = a[i];
 }
 
+__global__ void shfl_kernel(int iters, float *__restrict__ out) {
+  float v[8];
+#pragma unroll
+  for (int j = 0; j < 8; ++j) v[j] = threadIdx.x + j;
+  for (int it = 0; it < iters; ++it) {
+#pragma unroll
+    for (int j = 0; j < 8; ++j) v[j] = __shfl_xor_sync(0xffffffffu, v[j], 1 + (j & 3));
+  }
+  float s = 0.f;
+#pragma unroll
+  for (int j = 0; j < 8; ++j) s += v[j];
+  if (s == 1234.5f) out[0] = s;
+}
+
 extern "C" {
+__attribute__((visibility("default"))) int mb_shfl(int blocks, int iters, float *out, void *stream) {
+  shfl_kernel<<<blocks, 256, 0, (cudaStream_t)stream>>>(iters, out);
+  return cudaGetLastError() == cudaSuccess ? 0 : 2;
+}
 __attribute__((visibility("default"))) int mb_gather(const float *X, int64_t ld, const int32_t *idx,
                                                      int64_t n, int K, float *out, void *stream,
                                                      int blocks) {

@@ -15,6 +15,7 @@ lib = ctypes.CDLL(os.path.join(ROOT, "build", "libgnnmicro.so"))
 vp, i64, i32 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32
 lib.mb_gather.argtypes = [vp, i64, vp, i64, i32, vp, vp, i32]
 lib.mb_copy.argtypes = [vp, vp, i64, vp, i32]
+lib.mb_shfl.argtypes = [i32, i32, vp, vp]
 
 
 def timed(fn, reps=10):
@@ -58,6 +59,12 @@ def main():
                 key = f"K{K}_{tier}"
                 res["gather"][key] = max(res["gather"].get(key, 0), round(gbps, 1))
             del X, idx
+    # warp-shuffle issue rate: warp-wide SHFL instructions per SM per clock
+    blocks, iters = nsm * 8, 4096
+    ms = timed(lambda: lib.mb_shfl(blocks, iters, vp(out.data_ptr()), st))
+    warps = blocks * 8
+    res["shfl_warp_instr_per_s"] = round(warps * iters * 8 / (ms * 1e-3), 1)
+    res["shfl_per_sm_per_clk_at_1965MHz"] = round(warps * iters * 8 / (ms * 1e-3) / nsm / 1.965e9, 3)
     print(json.dumps(res), flush=True)
 
 
