@@ -251,13 +251,17 @@ GNN_API gnn_status_t gnn_permute_rows(const float *X, int64_t ldx, int64_t n, in
  * and S_O (nnz) back.  Everything is enqueued asynchronously and the call returns without
  * waiting; `stream` is ordered after every copy of the call, so synchronise it before
  * reading O_host / out_host or reusing X_host (pinned host memory gives asynchronous DMA;
- * pageable memory works but copies synchronously).  Internally the plan's chunks are cut
- * into pieces (about one per 4 Mi nonzeros, at most 32; env GNN_HOST_PIECES overrides):
- * ColInd/Value of later pieces upload on a copy-in stream while earlier pieces compute
- * (alternating between `stream` and a second compute stream) and finished O rows / S_O
- * values download on a copy-out stream, so the call costs about max(upload, compute,
- * download) instead of their sum.  Deterministic plans run as one piece.  Reads the host
- * row_ind to find the rows each piece completes.
+ * pageable memory works but copies synchronously).  Internally the nonzeros are cut into
+ * pieces (about one per 4 Mi nonzeros, at most 32; env GNN_HOST_PIECES overrides): the
+ * graph uploads piece by piece on a copy-in stream (RowInd/ColInd/Value of the piece plus
+ * the next piece's first RowInd entry), each piece is planned as it lands (the plan
+ * kernel over the chunks that end inside it, then the pre-zero of its split rows, on a
+ * prep stream in piece order), earlier pieces compute (alternating between `stream` and a
+ * second compute stream) and finished O rows / S_O values download on a copy-out stream,
+ * so the call costs about max(upload, compute, download) instead of their sum.
+ * Deterministic plans run as one piece.  Reads the host row_ind to find the rows each
+ * piece completes.  GNN_HOST_TRACE=1 prints a per-piece timeline to stderr (synchronises;
+ * a measurement aid).
  * graph_host: host pointers (row_ptr unused), a square N-node graph or a row shard of one
  * (rows [row_base, row_base + M) with row_base + M <= N; SDDMM then uses A1 = those rows
  * of X, O holds the shard's M rows).  fp32 only.
@@ -273,9 +277,10 @@ GNN_API gnn_status_t gnn_run_host(const gnn_graph_t *graph_host, int32_t upload_
 
 /* gnn_run_host for nk feature widths K[0..nk) on one graph in ONE pipelined call
  * (1 <= nk <= 16): X_host[k] (N x K[k]), O_host[k] (M x K[k], or O_host / O_host[k] NULL
- * to skip that SpMM), out_host[k] (nnz, or NULL to skip that SDDMM).  The graph uploads
- * with the first width; X_host[k+1] uploads and every download overlap the kernels of
- * earlier widths, so the call costs about max(total upload, total compute, total
+ * to skip that SpMM), out_host[k] (nnz, or NULL to skip that SDDMM).  Copy-in order
+ * X_host[0], piece 0, X_host[1], piece 1, ...: width k computes every piece that has
+ * landed once its X has (catching up on earlier pieces), so downloads start after the
+ * first X and piece, and the call costs about max(total upload, total compute, total
  * download).  Each width has its own plan and workspace region, so no width waits for
  * an earlier width's download.  Same ordering, ownership and error rules as gnn_run_host
  * (gnn_run_host is this call with nk = 1).  workspace:

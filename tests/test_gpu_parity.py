@@ -695,3 +695,40 @@ def test_run_host_multi_row_shards():
                     assert_within(Es[j].numpy(), r2, T2, what=f"shard {p}/{P} sddmm K={K}")
     finally:
         os.environ.pop("GNN_HOST_PIECES", None)
+
+
+@pytest.mark.parametrize("dtype", ["f32", "bf16"])
+def test_feature_matrix_beyond_4GB(dtype):
+    """Byte offsets of gathered rows beyond 2^32 (X of 4.6 GB: row c starts at c * 1 KB
+    (fp32) / 512 B (bf16) with K = 256): the 64-bit address arithmetic of both kernels.
+    300 destination rows gather from the last rows of X and from random ones; the oracle
+    sees only the referenced rows (counter-based features: the same values by row id)."""
+    K = 256
+    N = 4_500_000 if dtype == "f32" else 9_000_000
+    M, deg, seed = 300, 160, 4242
+    rng = np.random.default_rng(77)
+    rows = np.repeat(np.arange(M), deg)
+    cols = np.where(rng.random(rows.size) < 0.5, rng.integers(N - 200_000, N, rows.size),
+                    rng.integers(0, N, rows.size))
+    g = gen.from_coo(M, N, rows, cols, gen.uniform_values(78, rows.size))
+    dg = upload(g)
+    X = torch.empty((N, K), dtype=torch.float32 if dtype == "f32" else torch.bfloat16, device=DEV)
+    step = 1_000_000
+    for r0 in range(0, N, step):
+        n = min(step, N - r0)
+        X[r0:r0 + n] = torch.from_numpy(gen.features(seed, n, K, row0=r0)).to(DEV)
+    assert X.numel() * X.element_size() > (1 << 32)
+    p = gs.plan(dg, K, feature_dtype=dtype)
+    O = gs.spmm(p, dg, X).cpu().numpy()
+    E = gs.sddmm(p, dg, X, X).cpu().numpy()
+    # the oracle on the referenced rows only (column ids remapped); bf16: the rounded values
+    uniq, inv = np.unique(np.concatenate([g.col_ind, np.arange(M)]), return_inverse=True)
+    Xs = np.concatenate([gen.features(seed, 1, K, row0=int(c)) for c in uniq])
+    if dtype == "bf16":
+        Xs = torch.from_numpy(Xs).to(torch.bfloat16).float().numpy()
+    col_s = inv[:g.nnz].astype(np.int32)
+    A1s = Xs[inv[g.nnz:]]
+    r, T = oracle.spmm(g.row_ind, col_s, g.val, Xs, M=M)
+    assert_within(O, r, T, what=f"spmm {dtype} X > 4 GB")
+    r2, T2 = oracle.sddmm(g.row_ind, col_s, g.val, A1s, Xs)
+    assert_within(E, r2, T2, what=f"sddmm {dtype} X > 4 GB")
