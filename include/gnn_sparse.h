@@ -171,6 +171,23 @@ GNN_API gnn_status_t gnn_spmm_ex(gnn_plan_t plan, const gnn_graph_t *graph, cons
                                  int64_t lda, float *O, int64_t ldo, int32_t agg,
                                  int32_t accumulate, gnn_stream_t stream);
 
+/* Backward of gnn_spmm_ex with agg = GNN_AGG_MAX / GNN_AGG_MIN (fp32).  The forward keeps,
+ * for every (r, k), exactly one fp32 product fl(val[i] * A[col_ind[i]][k]); the gradient
+ * of O[r][k] flows to the FIRST nonzero i of row r (storage order) whose product equals
+ * O[r][k] (recomputed in the same fp32 arithmetic, so it is the term the forward kept;
+ * ties, e.g. zeros of a ReLU'd input, go to the first):
+ *   dA[col_ind[i]][k] += val[i] * dO[r][k]      dval[i] += A[col_ind[i]][k] * dO[r][k]
+ * ACCUMULATES into dA (N x K, pitch ldda) and, if dval is non-NULL, into dval (nnz, in
+ * col_ind order): zero them first for a plain gradient.  Needs graph->row_ptr (read
+ * relative to row_ptr[0]); O is the forward's output (M x K, pitch ldo), dO the incoming
+ * gradient (M x K, pitch lddo).  val NULL means all ones.  Float atomics make dA / dval
+ * order-dependent within fp32 rounding.  Device pointers; asynchronous on `stream`. */
+GNN_API gnn_status_t gnn_spmm_extremum_backward(const gnn_graph_t *graph, int32_t agg, int32_t K,
+                                                const float *A, int64_t lda, const float *O,
+                                                int64_t ldo, const float *dO, int64_t lddo,
+                                                float *dA, int64_t ldda, float *dval,
+                                                gnn_stream_t stream);
+
 /* SDDMM, S_O = (A1 A2) (.) S (Algorithm 2), hybrid-parallel
  * (Algorithm 4): out[i] = val[i] * sum_k A1[row_ind[i] - row_base][k] *
  * A2T[col_ind[i]][k] for i in [0, nnz).  A1: M x K (destination rows, lda1 >= K);
@@ -277,11 +294,11 @@ GNN_API gnn_status_t gnn_run_host(const gnn_graph_t *graph_host, int32_t upload_
 
 /* gnn_run_host for nk feature widths K[0..nk) on one graph in ONE pipelined call
  * (1 <= nk <= 16): X_host[k] (N x K[k]), O_host[k] (M x K[k], or O_host / O_host[k] NULL
- * to skip that SpMM), out_host[k] (nnz, or NULL to skip that SDDMM).  Copy-in order
- * X_host[0], piece 0, X_host[1], piece 1, ...: width k computes every piece that has
- * landed once its X has (catching up on earlier pieces), so downloads start after the
- * first X and piece, and the call costs about max(total upload, total compute, total
- * download).  Each width has its own plan and workspace region, so no width waits for
+ * to skip that SpMM), out_host[k] (nnz, or NULL to skip that SDDMM).  Copy-in order:
+ * the narrower widths' X interleaved with the first pieces (narrowest first), the widest
+ * width's X near the end; a width computes every piece that has landed once its X has
+ * (catching up on earlier pieces), so downloads start after the first X and piece, and
+ * the call costs about max(total upload, total compute, total download).  Each width has its own plan and workspace region, so no width waits for
  * an earlier width's download.  Same ordering, ownership and error rules as gnn_run_host
  * (gnn_run_host is this call with nk = 1).  workspace:
  * gnn_run_host_multi_workspace_bytes(M, N, nnz, nk, K, opts) bytes ((size_t)-1 on

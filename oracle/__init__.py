@@ -44,6 +44,8 @@ def _load():
     lib.oracle_spmm.argtypes = [i64, i64, vp, vp, vp, i64, vp, i64, i64, i64, vp, vp]
     lib.oracle_sddmm.argtypes = [i64, i64, vp, vp, vp, i64, vp, i64, vp, i64, vp, vp]
     lib.oracle_spmm_agg.argtypes = [i64, i64, vp, vp, vp, i64, vp, i64, i64, i64, i32, vp, vp]
+    lib.oracle_spmm_extremum_backward.argtypes = [i64, i64, vp, vp, vp, i64, vp, i64, i64, i64,
+                                                  i64, i32, vp, vp, vp]
     lib.oracle_plan.argtypes = [i64, vp, i32, i32, i32, i32, i32, i32, i32, i32, i64, i64,
                                 ctypes.POINTER(_PlanInfo), vp, vp, vp]
     lib.oracle_shard_rows.argtypes = [vp, i64, i32, vp]
@@ -113,6 +115,28 @@ def spmm_agg(row_ind, col_ind, val, A, agg, M=None, i0=0, i1=None, r0=0, nrows=N
     if rc != 0:
         raise ValueError("oracle_spmm_agg: invalid arguments")
     return O, T
+
+
+def spmm_extremum_backward(row_ind, col_ind, val, A, dO, agg, M=None):
+    """Gradients (dA N x K, dval nnz) of sum(dO * O) for O = spmm_agg(..., agg) with
+    agg in {max, min}: the first nonzero of each row attaining the fp32 extremum takes
+    the gradient of each (row, column) (oracle.c, reading 26)."""
+    lib = _load()
+    row_ind, col_ind = _i32(row_ind), _i32(col_ind)
+    val = None if val is None else np.ascontiguousarray(val, np.float32)
+    A = _f32_2d(A)
+    dO = np.ascontiguousarray(dO, np.float32)
+    nrows = M if M is not None else (int(row_ind.max()) + 1 if row_ind.size else 0)
+    N, K = A.shape
+    assert dO.shape == (nrows, K)
+    dA = np.empty((N, K), np.float64)
+    dval = np.empty(row_ind.shape[0], np.float64)
+    rc = lib.oracle_spmm_extremum_backward(0, row_ind.shape[0], _ptr(row_ind), _ptr(col_ind),
+                                           _ptr(val), K, _ptr(A), A.strides[0] // 4, N, 0,
+                                           nrows, AGG[agg], _ptr(dO), _ptr(dA), _ptr(dval))
+    if rc != 0:
+        raise ValueError("oracle_spmm_extremum_backward: invalid arguments")
+    return dA, dval
 
 
 def spmm_rows(g, A, rows):

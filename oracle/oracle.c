@@ -76,6 +76,54 @@ int oracle_spmm_agg(int64_t i0, int64_t i1, const int32_t *row_ind, const int32_
   return 0;
 }
 
+/* Backward of the max / min node-wise op (Eq. 1; the subgradient rule is
+ * DESIGN.md reading 26).  The forward keeps one fp32 product fl(v_i * A[c_i][k]) per
+ * (r, k) -- the decision is taken in the kernel's precision (fp32 products, exact
+ * comparisons), the gradients are accumulated in fp64:
+ *   1. E[r][k] = max (min) over the row's nonzeros of the fp32 product;
+ *   2. the first nonzero i of row r (storage order) whose product equals E[r][k] gets
+ *      dA[c_i][k] += v_i * dO[r][k] and dval[i - i0] += A[c_i][k] * dO[r][k].
+ * dA (N x K, zeroed here) and dval (i1 - i0, zeroed here; may be NULL). */
+int oracle_spmm_extremum_backward(int64_t i0, int64_t i1, const int32_t *row_ind,
+                                  const int32_t *col_ind, const float *val, int64_t K,
+                                  const float *A, int64_t lda, int64_t N, int64_t r0,
+                                  int64_t nrows, int32_t agg, const float *dO, double *dA,
+                                  double *dval) {
+  if (i0 < 0 || i1 < i0 || K < 1 || lda < K || nrows < 0 || N < 0 || (agg != 2 && agg != 3))
+    return -1;
+  memset(dA, 0, sizeof(double) * (size_t)(N * K));
+  if (dval) memset(dval, 0, sizeof(double) * (size_t)(i1 - i0));
+  float *E = (float *)malloc(sizeof(float) * (size_t)(nrows * K + 1));
+  char *seen = (char *)calloc((size_t)nrows + 1, 1);
+  char *taken = (char *)calloc((size_t)(nrows * K + 1), 1);
+  if (!E || !seen || !taken) { free(E); free(seen); free(taken); return -1; }
+  for (int64_t i = i0; i < i1; ++i) {                       /* step 1 */
+    int64_t r = row_ind[i] - r0, c = col_ind[i];
+    if (r < 0 || r >= nrows || c < 0 || c >= N) { free(E); free(seen); free(taken); return -1; }
+    float v = val ? val[i] : 1.0f;
+    for (int64_t k = 0; k < K; ++k) {
+      float p = v * A[c * lda + k];
+      float *e = E + r * K + k;
+      if (!seen[r] || (agg == 2 ? p > *e : p < *e)) *e = p;
+    }
+    seen[r] = 1;
+  }
+  for (int64_t i = i0; i < i1; ++i) {                       /* step 2, storage order */
+    int64_t r = row_ind[i] - r0, c = col_ind[i];
+    float v = val ? val[i] : 1.0f;
+    for (int64_t k = 0; k < K; ++k) {
+      float p = v * A[c * lda + k];
+      if (taken[r * K + k] || p != E[r * K + k]) continue;
+      taken[r * K + k] = 1;
+      double g = (double)dO[r * K + k];
+      dA[c * K + k] += (double)v * g;
+      if (dval) dval[i - i0] += (double)A[c * lda + k] * g;
+    }
+  }
+  free(E); free(seen); free(taken);
+  return 0;
+}
+
 /* ----------------------------------------------------------- SDDMM ------ */
 /* Algorithm 2. */
 int oracle_sddmm(int64_t i0, int64_t i1, const int32_t *row_ind, const int32_t *col_ind,

@@ -68,7 +68,8 @@ class ReorderOpts(ctypes.Structure):
 
 EXPORTS = ["gnn_plan_workspace_bytes", "gnn_plan_create", "gnn_plan_info", "gnn_plan_arrays",
            "gnn_plan_destroy", "gnn_spmm", "gnn_sddmm", "gnn_spmm_bf16", "gnn_sddmm_bf16",
-           "gnn_spmm_ex", "gnn_transpose_workspace_bytes", "gnn_transpose",
+           "gnn_spmm_ex", "gnn_spmm_extremum_backward", "gnn_transpose_workspace_bytes",
+           "gnn_transpose",
            "gnn_shard_rows", "gnn_shard_edges", "gnn_split_col_blocks",
            "gnn_reorder_gcr", "gnn_permute_graph", "gnn_permute_rows",
            "gnn_probe_gather", "gnn_run_host_workspace_bytes", "gnn_run_host",
@@ -102,6 +103,8 @@ def lib():
         L.gnn_sddmm_bf16.argtypes = [vp, P(_Graph), vp, i64, vp, i64, vp, vp]
     if hasattr(L, "gnn_spmm_ex"):
         L.gnn_spmm_ex.argtypes = [vp, P(_Graph), vp, i64, vp, i64, i32, i32, vp]
+        L.gnn_spmm_extremum_backward.argtypes = [P(_Graph), i32, i32, vp, i64, vp, i64, vp,
+                                                 i64, vp, i64, vp, vp]
         L.gnn_transpose_workspace_bytes.argtypes = [i64]
         L.gnn_transpose_workspace_bytes.restype = ctypes.c_size_t
         L.gnn_transpose.argtypes = [P(_Graph), vp, ctypes.c_size_t, vp, vp, vp, vp, vp, vp]
@@ -319,6 +322,27 @@ def spmm(p: Plan, graph: DeviceGraph, A: torch.Tensor, out: torch.Tensor | None 
     _check(fn(p.handle, ctypes.byref(g), _ptr(A), A.stride(0), _ptr(out), out.stride(0),
               _stream(stream)))
     return out
+
+
+def spmm_extremum_backward(graph: DeviceGraph, agg: str, A: torch.Tensor, O: torch.Tensor,
+                           dO: torch.Tensor, dA: torch.Tensor | None = None,
+                           dval: torch.Tensor | None = None, stream=None):
+    """gnn_spmm_extremum_backward: gradients of sum(dO * O) for O = spmm(..., agg=max|min)
+    (the first nonzero of each row attaining the extremum takes each column's gradient).
+    Accumulates into dA (N x K) / dval (nnz) when given, else returns fresh zeroed ones."""
+    if agg not in ("max", "min"):
+        raise ValueError("agg must be 'max' or 'min'")
+    for t, n in ((A, "A"), (O, "O"), (dO, "dO")):
+        _dense(t, n)
+    K = A.shape[1]
+    if dA is None:
+        dA = torch.zeros((graph.N, K), dtype=torch.float32, device=A.device)
+    _dense(dA, "dA")
+    g = graph.desc()
+    _check(lib().gnn_spmm_extremum_backward(ctypes.byref(g), AGG[agg], K, _ptr(A), A.stride(0),
+                                            _ptr(O), O.stride(0), _ptr(dO), dO.stride(0),
+                                            _ptr(dA), dA.stride(0), _ptr(dval), _stream(stream)))
+    return dA, dval
 
 
 def transpose(graph: DeviceGraph, stream=None):

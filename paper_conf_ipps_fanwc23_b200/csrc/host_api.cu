@@ -1,8 +1,9 @@
 // host_api.cu -- the end-to-end entry point on HOST buffers (bench.py's e2e path): the
 // caller hands host arrays and one device workspace; the library copies the graph and X
 // in, plans (GPU plan kernel), runs SpMM and SDDMM, and copies O and S_O out.
-// Pipelined over pieces of the nonzeros.  Copy-in stream: X_0, piece 0, X_1, piece 1, ...
-// (a piece = RowInd/ColInd/Value of a range of nonzeros common to every width); prep
+// Pipelined over pieces of the nonzeros.  Copy-in stream: the narrow widths' X
+// interleaved with the first pieces, the widest X near the end (a piece =
+// RowInd/ColInd/Value of a range of nonzeros common to every width); prep
 // stream: each piece is planned (plan kernel over the chunks that end inside it) and its
 // split rows pre-zeroed, in piece order; two alternating compute streams: SpMM + SDDMM of
 // every width whose X has landed (a width catches up on earlier pieces when its X lands);
@@ -291,14 +292,36 @@ GNN_API gnn_status_t gnn_run_host_multi(const gnn_graph_t *gh, int32_t upload_gr
       if (gnn_status_t st = compute(k, q, N > 0, ev_x)) return st;
     return GNN_OK;
   };
-  // Copy-in order X_0, piece 0, X_1, piece 1, ...: the copy-out stream gets width 0's
-  // first results after X_0 + one piece instead of after every X (PCIe is duplex, and the
-  // downloads are the longer direction).  Pieces: RowInd (+ the next piece's first
-  // entry, which the plan kernel's tail flag reads), ColInd, Value.
+  // Copy-in schedule.  Every width downloads the same S_O volume (4 B per nonzero) but
+  // costs 4*N*K bytes of X to start, and the downloads are the longer PCIe direction: so
+  // the narrow widths' X go first, one per piece (X_(0), piece 0, X_(1), piece 1, ...),
+  // keeping the copy-out stream fed from the first piece on, and the widest width's X goes
+  // near the end (before piece P - 1 - P/8), where its catch-up over every landed piece
+  // fills the copy-out queue for the tail (profiles/r01_v24_e2e_schedule.txt).  Pieces:
+  // RowInd (+ the next piece's first entry, which the plan kernel's tail flag reads),
+  // ColInd, Value.
+  int xpos[kMaxK];
+  {
+    int order[kMaxK];
+    for (int k = 0; k < nk; ++k) order[k] = k;
+    for (int i = 1; i < nk; ++i)  // stable insertion sort by K
+      for (int j = i; j > 0 && Ks[order[j]] < Ks[order[j - 1]]; --j) {
+        const int t = order[j];
+        order[j] = order[j - 1];
+        order[j - 1] = t;
+      }
+    for (int j = 0; j < nk; ++j) xpos[order[j]] = j;
+    if (nk >= 2) {
+      const int late = P - 1 - P / 8;
+      if (late > nk - 1) xpos[order[nk - 1]] = late;
+    }
+  }
   gnn_status_t st = GNN_OK;
   int64_t b = 0;
   for (int p = 0; p < P && st == GNN_OK; ++p) {
-    if (p < nk && (st = upload_x(p, p)) != GNN_OK) break;
+    for (int k = 0; k < nk && st == GNN_OK; ++k)
+      if (xpos[k] == p) st = upload_x(k, p);
+    if (st != GNN_OK) break;
     const int64_t en = p + 1 == P ? nnz : nnz * (p + 1) / P;  // this piece: nonzeros [b, en)
     if (up && en > b) {
       const int64_t er = en < nnz ? en + 1 : nnz;
@@ -332,13 +355,15 @@ GNN_API gnn_status_t gnn_run_host_multi(const gnn_graph_t *gh, int32_t upload_gr
       st = cuda_fail(e, "gnn_run_host event");
       break;
     }
-    // every width whose X has landed (X_k precedes piece k on the copy-in stream)
-    for (int k = 0; k < nk && k <= p && st == GNN_OK; ++k) st = compute(k, p, false, ev_x);
+    // every width whose X has landed (X_k precedes piece xpos[k] on the copy-in stream)
+    for (int k = 0; k < nk && st == GNN_OK; ++k)
+      if (xpos[k] <= p) st = compute(k, p, false, ev_x);
     trace.mark(p, 2, (units & 1) ? s : res.s2);
     trace.mark(p, 3, res.sout);
     b = en;
   }
-  for (int k = P; k < nk && st == GNN_OK; ++k) st = upload_x(k, P);  // fewer pieces than widths
+  for (int k = 0; k < nk && st == GNN_OK; ++k)  // fewer pieces than widths
+    if (xpos[k] >= P) st = upload_x(k, P);
   trace.xdone(res.sin);
   // the caller's stream covers every copy and kernel of this call (the copy-out stream
   // waited for every piece; s2, the prep and the copy-in stream are joined explicitly)

@@ -9,7 +9,8 @@ SpMM / SDDMM into torch.autograd:
     dv_i = <dO[row_i], X[col_i]>                  backward  (gnn_sddmm: SDDMM is the
                                                              gradient of SpMM w.r.t. v)
 
-Max / min aggregation has no backward here (it needs the arg-extremum per output).
+    max / min: the first nonzero of each row attaining the extremum takes the gradient
+    of each (row, column)                               (gnn_spmm_extremum_backward)
 All arithmetic runs in the library's kernels; torch supplies memory and the dense GEMM of
 the fully-connected part (cuBLAS, a plain library GEMM).
 """
@@ -19,7 +20,7 @@ import math
 
 import torch
 
-from . import DeviceGraph, plan, sddmm, spmm, transpose
+from . import DeviceGraph, plan, sddmm, spmm, spmm_extremum_backward, transpose
 
 
 class SparseOp:
@@ -64,16 +65,22 @@ class _SpMMFunction(torch.autograd.Function):
         g = op.g if val is None else op.with_val(val.detach().contiguous())
         O = spmm(op.plan_for("f", K, X.dtype), g, X, agg=agg)
         ctx.op, ctx.agg = op, agg
-        ctx.save_for_backward(X, val)
+        ctx.save_for_backward(X, val, O if agg in ("max", "min") else None)
         return O
 
     @staticmethod
     def backward(ctx, dO):
-        X, val = ctx.saved_tensors
+        X, val, O = ctx.saved_tensors
         op, agg = ctx.op, ctx.agg
-        if agg not in ("sum", "mean"):
-            raise NotImplementedError(f"no backward for the {agg} aggregator")
         dO = dO.contiguous().float()
+        if agg in ("max", "min"):
+            if X.dtype != torch.float32:
+                raise NotImplementedError("max / min backward: fp32 features only")
+            g = op.g if val is None else op.with_val(val.detach().contiguous())
+            need_v = val is not None and ctx.needs_input_grad[1]
+            dval = torch.zeros(op.g.nnz, dtype=torch.float32, device=X.device) if need_v else None
+            dX, dval = spmm_extremum_backward(g, agg, X, O, dO, dval=dval)
+            return (dX if ctx.needs_input_grad[0] else None), dval, None, None
         if agg == "mean":
             cnt = op.counts()
             dO = dO / torch.clamp(cnt, min=1.0)[:, None]

@@ -183,3 +183,75 @@ def test_deterministic_spmm_bitwise_reproducible(agg, C):
         if agg == "sum":  # beta = 1 through the fix-up pass as well
             gs.spmm(p, dg, X, out=O, accumulate=True)
             assert_within(O.cpu().numpy(), 2 * ref, 2 * T, what="det accumulate")
+
+
+# ------------------------------------------------ max / min backward (f3) ---
+def _extremum_bounds(g, A, dO):
+    """Upper bounds of sum|terms| for dA (N x K) and dval (nnz), independent of which
+    term each (row, column) selects: the tolerance scale of the float-atomic sums."""
+    v = np.abs(g.val.astype(np.float64)) if g.val is not None else np.ones(g.nnz)
+    TdA = np.zeros((g.N, A.shape[1]))
+    np.add.at(TdA, g.col_ind, v[:, None] * np.abs(dO[g.row_ind].astype(np.float64)))
+    Tdv = (np.abs(A[g.col_ind].astype(np.float64)) * np.abs(dO[g.row_ind])).sum(1)
+    return TdA, Tdv
+
+
+@pytest.mark.parametrize("agg", ["max", "min"])
+@pytest.mark.parametrize("K", [1, 7, 32, 100])
+@pytest.mark.parametrize("relu", [False, True])
+def test_extremum_backward_matches_oracle(agg, K, relu):
+    """gnn_spmm_extremum_backward against the oracle's first-occurrence subgradient on
+    graphs with empty rows, duplicates and a hub, values of both signs; relu=True zeroes
+    half the features so most (row, column) maxima are ties between zeros."""
+    for g in graphs():
+        dg = upload(g)
+        X = gen.features(41 + K, g.N, K)
+        if relu:
+            X = np.maximum(X, 0)
+        dO = gen.features(43 + K, g.M, K)
+        Xd = torch.from_numpy(X).to(DEV)
+        p = gs.plan(dg, K)
+        O = gs.spmm(p, dg, Xd, agg=agg)
+        dval = torch.zeros(g.nnz, device=DEV)
+        dA, _ = gs.spmm_extremum_backward(dg, agg, Xd, O, torch.from_numpy(dO).to(DEV),
+                                          dval=dval)
+        torch.cuda.synchronize()
+        rA, rv = oracle.spmm_extremum_backward(g.row_ind, g.col_ind, g.val, X, dO, agg, M=g.M)
+        TdA, Tdv = _extremum_bounds(g, X, dO)
+        assert_within(dA.cpu().numpy(), rA, TdA, what=f"{agg} dA K={K} relu={relu}")
+        assert_within(dval.cpu().numpy(), rv, Tdv, what=f"{agg} dval K={K} relu={relu}")
+
+
+def test_extremum_backward_matches_torch_scatter_reduce():
+    """An independent library reference on tie-free data: torch's scatter_reduce(amax /
+    amin) autograd (ties split evenly there; none occur here) gives the same dX and dv."""
+    rng = np.random.default_rng(11)
+    M, N, K = 300, 400, 16
+    rows = np.sort(rng.integers(0, M, 5000))
+    cols = rng.integers(0, N, rows.size)
+    keep = np.sort(np.unique(rows * N + cols, return_index=True)[1])
+    rows, cols = rows[keep], cols[keep]
+    g = gen.from_coo(M, N, rows, cols, rng.uniform(0.5, 1.5, rows.size).astype(np.float32))
+    dg = upload(g)
+    X = torch.randn(N, K, device=DEV, dtype=torch.float64).float().requires_grad_()
+    v = torch.from_numpy(g.val).to(DEV).requires_grad_()
+    dO = torch.randn(M, K, device=DEV)
+    op = gnn.SparseOp(dg)
+    ri = torch.from_numpy(g.row_ind.astype(np.int64)).to(DEV)
+    ci = torch.from_numpy(g.col_ind.astype(np.int64)).to(DEV)
+    present = torch.zeros(M, dtype=torch.bool, device=DEV)
+    present[ri] = True
+    for agg, red in (("max", "amax"), ("min", "amin")):
+        O = gnn.spmm_autograd(op, X, v, agg=agg)
+        (O * dO).sum().backward()
+        gX, gv = X.grad.clone(), v.grad.clone()
+        X.grad = v.grad = None
+        terms = v[:, None] * X[ci]
+        Oref = torch.zeros(M, K, device=DEV).scatter_reduce(
+            0, ri[:, None].expand(-1, K), terms, reduce=red, include_self=False)
+        Oref = torch.where(present[:, None], Oref, torch.zeros_like(Oref))
+        assert torch.equal(O.detach(), Oref.detach())
+        (Oref * dO).sum().backward()
+        torch.testing.assert_close(gX, X.grad, rtol=1e-5, atol=1e-5)
+        torch.testing.assert_close(gv, v.grad, rtol=1e-5, atol=1e-5)
+        X.grad = v.grad = None

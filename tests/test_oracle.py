@@ -470,3 +470,68 @@ def test_spmm_agg_sum_is_algorithm_1():
     a = oracle.spmm_agg(g.row_ind, g.col_ind, g.val, A, "sum", M=30)
     b = oracle.spmm(g.row_ind, g.col_ind, g.val, A, M=30)
     assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1])
+
+
+# ---------------------------------------------- max / min backward (f3) ----
+@pytest.mark.parametrize("agg", ["max", "min"])
+@pytest.mark.parametrize("seed", range(3))
+def test_extremum_backward_matches_finite_differences(agg, seed):
+    """d/dA and d/dval of L = sum(dO * O), O = the max / min aggregation, by central
+    differences of the oracle's FORWARD (oracle.spmm_agg, fp64) on tie-free inputs: the
+    selected term moves with its inputs, the others do not move O at all."""
+    rng = np.random.default_rng(900 + seed)
+    M, N, K, nnz = 6, 9, 3, 30
+    rows = np.sort(rng.integers(0, M, nnz))
+    cols = rng.integers(0, N, nnz)
+    keep = np.unique(rows * N + cols, return_index=True)[1]  # no duplicate (r, c): no ties
+    rows, cols = rows[np.sort(keep)], cols[np.sort(keep)]
+    val = rng.uniform(0.5, 1.5, rows.size).astype(np.float32)
+    A = rng.uniform(-1, 1, (N, K)).astype(np.float32)
+    dO = rng.uniform(-1, 1, (M, K)).astype(np.float32)
+    dA, dval = oracle.spmm_extremum_backward(rows, cols, val, A, dO, agg, M=M)
+
+    def loss(A_, v_):
+        O, _ = oracle.spmm_agg(rows, cols, v_, A_, agg, M=M)
+        return float((O * dO.astype(np.float64)).sum())
+
+    eps = 2.0 ** -12  # far below the gaps between competing terms (checked below)
+    fd_A = np.zeros_like(dA)
+    for c in range(N):
+        for k in range(K):
+            Ap, Am = A.copy(), A.copy()
+            Ap[c, k] += eps
+            Am[c, k] -= eps
+            fd_A[c, k] = (loss(Ap, val) - loss(Am, val)) / (2 * eps)
+    fd_v = np.zeros_like(dval)
+    for i in range(rows.size):
+        vp, vm = val.copy(), val.copy()
+        vp[i] += eps
+        vm[i] -= eps
+        fd_v[i] = (loss(A, vp) - loss(A, vm)) / (2 * eps)
+    terms = val[:, None].astype(np.float64) * A[cols]
+    for r in range(M):  # tie-free by a margin larger than the perturbation
+        t = np.sort(terms[rows == r], axis=0)
+        if t.shape[0] > 1:
+            assert (np.diff(t, axis=0) > 4 * eps).all()
+    np.testing.assert_allclose(dA, fd_A, rtol=0, atol=1e-6)
+    np.testing.assert_allclose(dval, fd_v, rtol=0, atol=1e-6)
+
+
+def test_extremum_backward_ties_go_to_the_first_term():
+    """Hand-worked: row 0 has three terms, two of them tied for the max (A[1] = A[2] = 2
+    with v = 1) and one tied zero pair in column 1; row 1 is a single term; row 2 empty.
+    The first tied nonzero in storage order takes the whole gradient."""
+    rows = np.array([0, 0, 0, 1])
+    cols = np.array([0, 1, 2, 0])
+    val = np.ones(4, np.float32)
+    A = np.array([[1.0, 0.0], [2.0, 0.0], [2.0, -1.0]], np.float32)
+    dO = np.array([[10.0, 20.0], [30.0, 40.0], [50.0, 60.0]], np.float32)
+    dA, dval = oracle.spmm_extremum_backward(rows, cols, val, A, dO, "max", M=3)
+    # row 0, col 0: max 2 at nonzeros 1 and 2 -> nonzero 1 (source 1); col 1: max 0 at
+    # nonzeros 0 and 1 -> nonzero 0 (source 0).  row 1: nonzero 3 (source 0) everywhere.
+    np.testing.assert_array_equal(dA, [[30.0, 20.0 + 40.0], [10.0, 0.0], [0.0, 0.0]])
+    np.testing.assert_array_equal(dval, [0.0 * 20.0, 2.0 * 10.0, 0.0, 1.0 * 30.0 + 0.0 * 40.0])
+    dA, dval = oracle.spmm_extremum_backward(rows, cols, val, A, dO, "min", M=3)
+    # min: col 0 -> nonzero 0 (value 1); col 1 -> nonzero 2 (value -1)
+    np.testing.assert_array_equal(dA, [[10.0 + 30.0, 40.0], [0.0, 0.0], [0.0, 20.0]])
+    np.testing.assert_array_equal(dval, [10.0, 0.0, -20.0, 30.0])

@@ -4,6 +4,12 @@ synthetic graph with random features / labels, our SpMM/SDDMM kernels vs torch.s
 (cuSPARSE CSR SpMM) in the same model.  One step = forward + backward + Adam.
 
     python tools/train_gcn.py --workload C4 --hidden 32,128,256 --steps 20
+    python tools/train_gcn.py --workload C3 --hidden 128 --steps 100   # GraphSAINT-style
+
+C3 (BASELINE.json configs[2]): a new sampled subgraph every step (pre-generated and
+resident, as a sampler running ahead would leave them), so every step also builds the
+graph's transpose (gnn_transpose) and plans (GPU plan kernel) -- or, for torch.sparse, its
+CSR tensors -- inside the timed region.
 """
 import argparse
 import json
@@ -63,8 +69,11 @@ def main():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--reorder", action="store_true")
+    ap.add_argument("--subgraphs", type=int, default=20, help="C3: resident subgraphs cycled")
     a = ap.parse_args()
     dev = torch.device("cuda")
+    if a.workload == "C3":
+        return run_sampled(a, dev)
     g = configs.make_graph(a.workload)
     if a.reorder:
         perm, _, _ = gs.reorder_gcr(g.row_ptr, g.col_ind)
@@ -92,6 +101,60 @@ def main():
             o1.step()
 
         def step_base():
+            o2.zero_grad(set_to_none=True)
+            torch.nn.functional.cross_entropy(base(A, X), y).backward()
+            o2.step()
+
+        t_ours = time_steps(step_ours, a.steps, a.warmup)
+        try:
+            t_base = time_steps(step_base, a.steps, a.warmup)
+        except Exception as e:  # noqa: BLE001
+            t_base = None
+            res["baseline_error"] = str(e)[:200]
+        res["runs"].append({"hidden": h, "ours_ms": round(t_ours, 3),
+                            "torch_sparse_ms": None if t_base is None else round(t_base, 3),
+                            "speedup": None if t_base is None else round(t_base / t_ours, 3)})
+        print(json.dumps(res["runs"][-1]), flush=True)
+    print(json.dumps(res), flush=True)
+
+
+def run_sampled(a, dev):
+    """GraphSAINT-style training: step t trains on subgraph t mod T (its own features and
+    labels); the per-subgraph sparse structures are built inside the step."""
+    torch.manual_seed(0)
+    subs = []
+    for t in range(a.subgraphs):
+        g = configs.make_c3(t)
+        tens = {k: torch.from_numpy(np.ascontiguousarray(v)).to(dev) for k, v in
+                (("row_ptr", g.row_ptr), ("row_ind", g.row_ind), ("col_ind", g.col_ind),
+                 ("val", g.val))}
+        X = torch.randn(g.N, a.features, device=dev)
+        y = torch.randint(0, a.classes, (g.M,), device=dev)
+        subs.append((g, tens, X, y))
+    nnz = [s[0].nnz for s in subs]
+    res = {"workload": "C3", "subgraphs": a.subgraphs, "nnz_mean": int(np.mean(nnz)),
+           "features": a.features, "classes": a.classes, "layers": a.layers, "runs": []}
+    for h in [int(x) for x in a.hidden.split(",")]:
+        ours = gnn.GCN(a.features, h, a.classes, a.layers).to(dev)
+        base = TorchSparseGCN(a.features, h, a.classes, a.layers).to(dev)
+        o1 = torch.optim.Adam(ours.parameters(), lr=0.01)
+        o2 = torch.optim.Adam(base.parameters(), lr=0.01)
+        it = {"i": 0}
+
+        def step_ours():
+            g, t, X, y = subs[it["i"] % len(subs)]
+            it["i"] += 1
+            dg = gs.DeviceGraph(g.M, g.N, t["row_ind"], t["col_ind"], t["val"], t["row_ptr"])
+            op = gnn.SparseOp(dg)  # transpose + (lazily) plans: re-built every step
+            o1.zero_grad(set_to_none=True)
+            torch.nn.functional.cross_entropy(ours(op, X), y).backward()
+            o1.step()
+
+        def step_base():
+            g, t, X, y = subs[it["i"] % len(subs)]
+            it["i"] += 1
+            A = torch.sparse_csr_tensor(t["row_ptr"].long(), t["col_ind"].long(), t["val"],
+                                        size=(g.M, g.N))
             o2.zero_grad(set_to_none=True)
             torch.nn.functional.cross_entropy(base(A, X), y).backward()
             o2.step()
