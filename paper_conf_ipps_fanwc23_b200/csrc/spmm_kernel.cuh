@@ -43,13 +43,16 @@ __device__ __forceinline__ float agg_init() {
 }
 
 // float atomic max / min through the ordered-integer trick (there is no red.max.f32):
-// non-negative floats order like signed ints, negative ones reversed like unsigned.
+// floats with the sign bit clear order like signed ints, those with it set (negatives and
+// -0.0) reversed like unsigned.  The branch tests the sign BIT, not v >= 0: -0.0 >= 0 is
+// true, but as a signed int -0.0 is INT_MIN and would beat every negative value in a
+// signed atomicMin (and lose to them in atomicMax).
 __device__ __forceinline__ void atomic_max_f32(float *p, float v) {
-  if (v >= 0.f) atomicMax(reinterpret_cast<int *>(p), __float_as_int(v));
+  if (!(__float_as_uint(v) >> 31)) atomicMax(reinterpret_cast<int *>(p), __float_as_int(v));
   else atomicMin(reinterpret_cast<unsigned *>(p), __float_as_uint(v));
 }
 __device__ __forceinline__ void atomic_min_f32(float *p, float v) {
-  if (v >= 0.f) atomicMin(reinterpret_cast<int *>(p), __float_as_int(v));
+  if (!(__float_as_uint(v) >> 31)) atomicMin(reinterpret_cast<int *>(p), __float_as_int(v));
   else atomicMax(reinterpret_cast<unsigned *>(p), __float_as_uint(v));
 }
 

@@ -210,6 +210,10 @@ def test_extremum_backward_matches_oracle(agg, K, relu):
             X = np.maximum(X, 0)
         dO = gen.features(43 + K, g.M, K)
         Xd = torch.from_numpy(X).to(DEV)
+        for C in (0, 8):  # rows split across chunks meet in the float atomics (+-0 included)
+            Oc = gs.spmm(gs.plan(dg, K, force_chunk=C), dg, Xd, agg=agg).cpu().numpy()
+            rO, TO = oracle.spmm_agg(g.row_ind, g.col_ind, g.val, X, agg, M=g.M)
+            assert_within(Oc, rO, TO, what=f"{agg} forward K={K} relu={relu} C={C}")
         p = gs.plan(dg, K)
         O = gs.spmm(p, dg, Xd, agg=agg)
         dval = torch.zeros(g.nnz, device=DEV)
