@@ -296,7 +296,7 @@ GNN_API gnn_status_t gnn_run_host(const gnn_graph_t *graph_host, int32_t upload_
  * (1 <= nk <= 16): X_host[k] (N x K[k]), O_host[k] (M x K[k], or O_host / O_host[k] NULL
  * to skip that SpMM), out_host[k] (nnz, or NULL to skip that SDDMM).  Copy-in order:
  * the narrower widths' X interleaved with the first pieces (narrowest first), the widest
- * width's X near the end; a width computes every piece that has landed once its X has
+ * width's X half-way (env GNN_HOST_WIDE_X_AT = piece index overrides); a width computes every piece that has landed once its X has
  * (catching up on earlier pieces), so downloads start after the first X and piece, and
  * the call costs about max(total upload, total compute, total download).  Each width has its own plan and workspace region, so no width waits for
  * an earlier width's download.  Same ordering, ownership and error rules as gnn_run_host

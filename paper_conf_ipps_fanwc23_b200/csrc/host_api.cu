@@ -296,8 +296,10 @@ GNN_API gnn_status_t gnn_run_host_multi(const gnn_graph_t *gh, int32_t upload_gr
   // costs 4*N*K bytes of X to start, and the downloads are the longer PCIe direction: so
   // the narrow widths' X go first, one per piece (X_(0), piece 0, X_(1), piece 1, ...),
   // keeping the copy-out stream fed from the first piece on, and the widest width's X goes
-  // near the end (before piece P - 1 - P/8), where its catch-up over every landed piece
-  // fills the copy-out queue for the tail (profiles/r01_v24_e2e_schedule.txt).  Pieces:
+  // half-way (before piece P/2), where its catch-up over every landed piece fills the
+  // copy-out queue while the rest of the graph streams in (profiles/r01_v24_e2e_schedule.txt,
+  // r01_v27_e2e_wide_x_at.txt: before piece 14 of 28 measured best, 24 / 18 / 10 within
+  // 0.5-1.2 ms of it).  Pieces:
   // RowInd (+ the next piece's first entry, which the plan kernel's tail flag reads),
   // ColInd, Value.
   int xpos[kMaxK];
@@ -312,7 +314,7 @@ GNN_API gnn_status_t gnn_run_host_multi(const gnn_graph_t *gh, int32_t upload_gr
       }
     for (int j = 0; j < nk; ++j) xpos[order[j]] = j;
     if (nk >= 2) {
-      int late = P - 1 - P / 8;
+      int late = P / 2;
       if (const char *e = getenv("GNN_HOST_WIDE_X_AT")) late = atoi(e);  // tuning knob
       if (late > nk - 1) xpos[order[nk - 1]] = late < P ? late : P;
     }
