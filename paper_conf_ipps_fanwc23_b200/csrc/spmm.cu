@@ -224,7 +224,16 @@ gnn_status_t launch_spmm(const Plan *p, const gnn_graph_t *g, const void *A, int
     cudaError_t e = cudaMemset2DAsync(O, ldo * sizeof(float), 0, K * sizeof(float), g->M, s);
     return e == cudaSuccess ? GNN_OK : cuda_fail(e, "gnn_spmm memset");
   }
-  const int vws = effective_vws(in.vw_sparse, g, nullptr);
+  int vws = effective_vws(in.vw_sparse, g, nullptr);
+#ifndef GNN_SPMM_BF16_R2_VWS2
+#define GNN_SPMM_BF16_R2_VWS2 1  // measured: bf16 K=256 SpMM 4.43 -> 4.30 ms (r01_sweep39)
+#endif
+#if GNN_SPMM_BF16_R2_VWS2
+  // bf16 rows of two 32-byte vectors per lane (R = 2): with 4-wide sparse vectors the
+  // batch holds 4 nonzeros x 2 vectors of 16 bf16 in flight, which spills at the 128-register
+  // budget (ptxas: 308 B); 2-wide sparse copies halve the batch and remove the spill
+  if (dtype == GNN_BF16 && in.vecs == 2 && vws > 2) vws = 2;
+#endif
   SpmmFn f = pick_spmm(dtype, VW, in.lanes, in.vecs, vws, agg);
   if (!f)
     return fail(GNN_ERR_UNSUPPORTED, "%s: no kernel for vw=%d L=%d agg=%d dtype=%d", who, VW,
