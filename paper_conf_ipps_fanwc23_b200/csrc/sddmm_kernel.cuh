@@ -24,6 +24,9 @@ namespace gnn {
 #ifndef GNN_SDDMM_PIPE
 #define GNN_SDDMM_PIPE 1     // next batch's loads issued before this batch's reduction
 #endif
+#ifndef GNN_SDDMM_PIPE_GENERAL
+#define GNN_SDDMM_PIPE_GENERAL 1  // ... also on tiles with row switches (r01_sweep40)
+#endif
 template <int VW, int V, int SMAX>
 struct SddmmShape {
   static constexpr int R = (V >= GNN_SDDMM_R2_FROM && V >= 2) ? 2 : 1;
@@ -277,11 +280,55 @@ __global__ void __launch_bounds__(kMaxThreads, (SddmmShape<VW, L, SMAX>::minb))
     // measured (profiles/r01_sweep39): a gain where the butterfly is long (Lg >= 8 lanes per
     // dot product: fp32 K=256 6.47 -> 6.16 ms, K=128 3.21 -> 3.11 ms, bf16 K=256 3.48 ->
     // 3.41 ms), a small loss at Lg = 4 (fp32 K=64 +0.7%, bf16 K=64 +2.6%)
+#if GNN_SDDMM_PIPE_GENERAL
+    // the same pipelining for tiles with row switches / a partial last tile: the next
+    // batch's A2T rows do not depend on the row switches of this one
+    auto run_general_pipelined = [&]() {
+      const char *A2l = A2b + (int64_t)(l * VW) * ES;
+      bool lane_ok[R];
+#pragma unroll
+      for (int r = 0; r < R; ++r) lane_ok[r] = item_ok && (r * Lg + l) * VW < a.K;
+      FeatVec<TF, VW> x[U][R];
+      auto load_batch = [&](int jj) {
+        const int valid = n - (tb + jj);
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          const char *rowp = A2l + (uint64_t)(uint32_t)s_col[jj + u] * ld2B;
+#pragma unroll
+          for (int r = 0; r < R; ++r) {
+            if (lane_ok[r] && u < valid) x[u][r].load(rowp + r * Lg * VW * ES);
+            else x[u][r].zero();
+          }
+        }
+      };
+      load_batch(0);
+#pragma unroll 1
+      for (int jj = 0; jj < T; jj += U) {
+        const int valid = n - (tb + jj);
+        float part[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          part[u] = 0.f;
+          const int32_t rj = s_row[jj + u];
+          if (item_ok && u < valid && rj != cur[0]) load_a1_slice(0, rj);  // Algo 4 l. 8-11
+#pragma unroll
+          for (int r = 0; r < R; ++r) part[u] = dot_f<TF, VW>(part[u], a1[0][r], x[u][r]);
+        }
+        if (jj + U < T) load_batch(jj + U);
+        reduce_scale_store<U, Lg>(part, vi ? s_val + jj : nullptr, l, oc + tb + jj,
+                                  item_ok ? valid : 0);
+      }
+    };
+#endif
     if constexpr (SMAX == 1 && Lg >= 8) {
       if (fast) {
         run_fast_pipelined();
         continue;
       }
+#if GNN_SDDMM_PIPE_GENERAL
+      run_general_pipelined();
+      continue;
+#endif
     }
 #endif
     if (fast) run_tile(std::true_type{});
