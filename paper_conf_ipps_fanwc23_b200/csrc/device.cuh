@@ -82,8 +82,28 @@ __device__ __forceinline__ void ld_feat<8>(const float *p, float (&x)[8]) {
 }
 
 // ------------------------------------------------------------- outputs ----
+#ifndef GNN_OUT_STREAMING
+#define GNN_OUT_STREAMING 0  // outputs stored with the streaming (.cs, evict-first) policy
+#endif
 template <int VW>
 __device__ __forceinline__ void st_vec(float *p, const float (&x)[VW]) {
+#if GNN_OUT_STREAMING
+  // written once, never re-read by the kernel: keep them from displacing gathered rows
+  if constexpr (VW == 1) {
+    __stcs(p, x[0]);
+  } else if constexpr (VW == 2) {
+    __stcs(reinterpret_cast<float2 *>(p), make_float2(x[0], x[1]));
+  } else if constexpr (VW == 4) {
+    __stcs(reinterpret_cast<float4 *>(p), make_float4(x[0], x[1], x[2], x[3]));
+  } else {
+#pragma unroll
+    for (int h = 0; h < VW; h += 8)
+      asm volatile("st.global.cs.v8.f32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p + h),
+                   "f"(x[h]), "f"(x[h + 1]), "f"(x[h + 2]), "f"(x[h + 3]), "f"(x[h + 4]),
+                   "f"(x[h + 5]), "f"(x[h + 6]), "f"(x[h + 7])
+                   : "memory");
+  }
+#else
   if constexpr (VW == 1) {
     p[0] = x[0];
   } else if constexpr (VW == 2) {
@@ -98,6 +118,7 @@ __device__ __forceinline__ void st_vec(float *p, const float (&x)[VW]) {
                    "f"(x[h + 5]), "f"(x[h + 6]), "f"(x[h + 7])
                    : "memory");
   }
+#endif
 }
 
 template <int VW>

@@ -74,7 +74,13 @@ __device__ __forceinline__ void reduce_scale_store(float (&part)[U], const float
   if constexpr (U <= L) {
     constexpr int R = L / U;
     const int u = l / R;
-    if (l % R == 0 && u < valid) out[u] = part[0] * (sval ? sval[u] : 1.f);
+    if (l % R == 0 && u < valid) {
+#if GNN_OUT_STREAMING
+      __stcs(out + u, part[0] * (sval ? sval[u] : 1.f));
+#else
+      out[u] = part[0] * (sval ? sval[u] : 1.f);
+#endif
+    }
   } else {
     // this lane holds P consecutive results: one vector store for a full, aligned batch
     // (the scalar stores of narrow rows -- 64-byte rows: 16 groups x 4 stores per batch
@@ -85,15 +91,26 @@ __device__ __forceinline__ void reduce_scale_store(float (&part)[U], const float
         float v[P];
 #pragma unroll
         for (int i = 0; i < P; ++i) v[i] = part[i] * (sval ? sval[l * P + i] : 1.f);
+#if GNN_OUT_STREAMING
+        if constexpr (P == 4) __stcs(reinterpret_cast<float4 *>(o), make_float4(v[0], v[1], v[2], v[3]));
+        else __stcs(reinterpret_cast<float2 *>(o), make_float2(v[0], v[1]));
+#else
         if constexpr (P == 4) *reinterpret_cast<float4 *>(o) = make_float4(v[0], v[1], v[2], v[3]);
         else *reinterpret_cast<float2 *>(o) = make_float2(v[0], v[1]);
+#endif
         return;
       }
     }
 #pragma unroll
     for (int i = 0; i < P; ++i) {
       const int u = l * P + i;
-      if (u < valid) out[u] = part[i] * (sval ? sval[u] : 1.f);
+      if (u < valid) {
+#if GNN_OUT_STREAMING
+        __stcs(out + u, part[i] * (sval ? sval[u] : 1.f));
+#else
+        out[u] = part[i] * (sval ? sval[u] : 1.f);
+#endif
+      }
     }
   }
 }
