@@ -608,6 +608,26 @@ def run_c3(args, dev, world, rank):
         b.record()
         torch.cuda.synchronize()
         graph_ms = a.elapsed_time(b) / nsteps
+    # the native one-call step (gnn_plan_spmm_sddmm: plan + SpMM + SDDMM in one C-ABI call,
+    # SDDMM on a forked side stream), eager, events around each step, flush between
+    native_ms = None
+    try:
+        run1 = gs.StepRunner(dev)
+        for i in range(min(len(subs), args.warmup + 1)):
+            g_, dg_, X_, O_, E_ = subs[i]
+            run1(dg_, X_, O_, E_)
+        torch.cuda.synchronize()
+        nev = [[torch.cuda.Event(enable_timing=True) for _ in range(2)] for _ in range(nsteps)]
+        for s in range(nsteps):
+            flush.fill_(float(s))
+            g_, dg_, X_, O_, E_ = subs[s % len(subs)]
+            nev[s][0].record(stream)
+            run1(dg_, X_, O_, E_)
+            nev[s][1].record(stream)
+        torch.cuda.synchronize()
+        native_ms = statistics.mean(e[0].elapsed_time(e[1]) for e in nev)
+    except Exception as ex:  # report, never lose the main line
+        native_ms = f"error: {type(ex).__name__}: {ex}"[:200]
     evs = [[torch.cuda.Event(enable_timing=True) for _ in range(5)] for _ in range(nsteps)]
     clk = ClockSampler(dev.index)
     clk.start()
@@ -651,6 +671,8 @@ def run_c3(args, dev, world, rank):
                            "K": [K], "subgraphs_per_rank": len(subs),
                            "l2": "flushed between timed steps (256 MiB write, outside events)"},
                 "c3": {"cuda_graph_ms_per_step": None if graph_ms is None else round(graph_ms, 4),
+                       "native_one_call_ms_per_step": round(native_ms, 4)
+                       if isinstance(native_ms, float) else native_ms,
                        "plan_ms_mean": round(statistics.mean(pl), 4),
                        "spmm_ms_mean": round(statistics.mean(sp), 4),
                        "sddmm_ms_mean": round(statistics.mean(sd), 4),

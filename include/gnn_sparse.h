@@ -311,6 +311,21 @@ GNN_API gnn_status_t gnn_run_host_multi(const gnn_graph_t *graph_host, int32_t u
                                         float *const *out_host, const gnn_plan_opts_t *opts,
                                         void *workspace, size_t ws_bytes, gnn_stream_t stream);
 
+/* One message-passing step on DEVICE data in one call (BJ configs[2]: a new sampled
+ * subgraph every step, re-planned every step): gnn_plan_create into `workspace`
+ * (gnn_plan_workspace_bytes bytes; host DTP + plan kernel, no sync), then O = S X
+ * (gnn_spmm, if O) and out[i] = val[i] <X[row_i], X[col_i]> (gnn_sddmm with A1 = the
+ * graph's rows of X, i.e. X + row_base * ldx, A2T = X, if out).  The SDDMM runs on a
+ * per-thread side stream forked from `stream` after the plan and joined back, so the two
+ * kernels overlap; `stream` is ordered after both.  The plan handle is internal and
+ * released before return (its arrays stay in `workspace`).  fp32; same alignment and
+ * error rules as gnn_spmm / gnn_sddmm.  Device pointers. */
+GNN_API gnn_status_t gnn_plan_spmm_sddmm(const gnn_graph_t *graph, int32_t K,
+                                         const gnn_plan_opts_t *opts, const float *X,
+                                         int64_t ldx, float *O, int64_t ldo, float *out,
+                                         void *workspace, size_t ws_bytes,
+                                         gnn_stream_t stream);
+
 /* ----------------------------------------------------------- measurement --- */
 /* Roofline probe (not part of the method): gathers rows X[idx[i]][0:K] for i in [0, n)
  * with the same 256-bit row loads the kernels use and no other work (sums are folded

@@ -68,7 +68,8 @@ class ReorderOpts(ctypes.Structure):
 
 EXPORTS = ["gnn_plan_workspace_bytes", "gnn_plan_create", "gnn_plan_info", "gnn_plan_arrays",
            "gnn_plan_destroy", "gnn_spmm", "gnn_sddmm", "gnn_spmm_bf16", "gnn_sddmm_bf16",
-           "gnn_spmm_ex", "gnn_spmm_extremum_backward", "gnn_transpose_workspace_bytes",
+           "gnn_spmm_ex", "gnn_spmm_extremum_backward", "gnn_plan_spmm_sddmm",
+           "gnn_transpose_workspace_bytes",
            "gnn_transpose",
            "gnn_shard_rows", "gnn_shard_edges", "gnn_split_col_blocks",
            "gnn_reorder_gcr", "gnn_permute_graph", "gnn_permute_rows",
@@ -105,6 +106,8 @@ def lib():
         L.gnn_spmm_ex.argtypes = [vp, P(_Graph), vp, i64, vp, i64, i32, i32, vp]
         L.gnn_spmm_extremum_backward.argtypes = [P(_Graph), i32, i32, vp, i64, vp, i64, vp,
                                                  i64, vp, i64, vp, vp]
+        L.gnn_plan_spmm_sddmm.argtypes = [P(_Graph), i32, P(PlanOpts), vp, i64, vp, i64, vp, vp,
+                                          ctypes.c_size_t, vp]
         L.gnn_transpose_workspace_bytes.argtypes = [i64]
         L.gnn_transpose_workspace_bytes.restype = ctypes.c_size_t
         L.gnn_transpose.argtypes = [P(_Graph), vp, ctypes.c_size_t, vp, vp, vp, vp, vp, vp]
@@ -343,6 +346,31 @@ def spmm_extremum_backward(graph: DeviceGraph, agg: str, A: torch.Tensor, O: tor
                                             _ptr(O), O.stride(0), _ptr(dO), dO.stride(0),
                                             _ptr(dA), dA.stride(0), _ptr(dval), _stream(stream)))
     return dA, dval
+
+
+class StepRunner:
+    """gnn_plan_spmm_sddmm: plan + SpMM + SDDMM (A1 = A2T = X) of one device graph in a
+    single native call, with a reusable plan workspace (sized for the largest graph seen)
+    -- the per-step path for sampled subgraphs (BJ configs[2])."""
+
+    def __init__(self, device="cuda"):
+        self.device = device
+        self.ws = torch.empty(256, dtype=torch.uint8, device=device)
+        self.opts = PlanOpts()
+
+    def __call__(self, graph: DeviceGraph, X: torch.Tensor, O: torch.Tensor | None,
+                 out: torch.Tensor | None, stream=None):
+        K = X.shape[1]
+        L = lib()
+        nbytes = L.gnn_plan_workspace_bytes(graph.M, graph.nnz, K, ctypes.byref(self.opts))
+        if nbytes == ctypes.c_size_t(-1).value:
+            _check(GNN_ERR_INVALID_ARG)
+        if nbytes > self.ws.numel():
+            self.ws = torch.empty(int(nbytes) * 2, dtype=torch.uint8, device=self.device)
+        _check(L.gnn_plan_spmm_sddmm(ctypes.byref(graph.desc()), K, ctypes.byref(self.opts),
+                                     _ptr(X), X.stride(0), _ptr(O),
+                                     0 if O is None else O.stride(0), _ptr(out), _ptr(self.ws),
+                                     self.ws.numel(), _stream(stream)))
 
 
 def transpose(graph: DeviceGraph, stream=None):

@@ -391,3 +391,86 @@ GNN_API gnn_status_t gnn_run_host(const gnn_graph_t *gh, int32_t upload_graph, c
 }
 
 }  // extern "C"
+
+// ----------------------------------------------------------------------------------
+// One message-passing step on device-resident data in ONE call (BJ configs[2]: a new
+// sampled subgraph every step, re-planned every step): plan (host DTP + plan kernel) ->
+// SpMM and SDDMM.  The SDDMM runs on a per-thread, per-device side stream forked from
+// `stream` after the plan and joined back before return, so the two kernels' tails
+// overlap on graphs that fill only a few waves; no allocation, no host sync.
+namespace gnn {
+namespace {
+struct SideStream {
+  int device = -1;
+  cudaStream_t s = nullptr;
+  cudaEvent_t fork = nullptr, join = nullptr;
+};
+thread_local SideStream tl_side[8];
+gnn_status_t side_stream(SideStream **out) {
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return cuda_fail(e, "gnn_plan_spmm_sddmm device");
+  SideStream &t = tl_side[dev & 7];
+  if (t.device != dev) {
+    if (t.s) {  // another device used this slot: rebuild
+      cudaStreamDestroy(t.s);
+      cudaEventDestroy(t.fork);
+      cudaEventDestroy(t.join);
+      t.s = nullptr;
+    }
+    e = cudaStreamCreateWithFlags(&t.s, cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&t.fork, cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&t.join, cudaEventDisableTiming);
+    if (e != cudaSuccess) return cuda_fail(e, "gnn_plan_spmm_sddmm side stream");
+    t.device = dev;
+  }
+  *out = &t;
+  return GNN_OK;
+}
+}  // namespace
+}  // namespace gnn
+
+extern "C" {
+
+GNN_API gnn_status_t gnn_plan_spmm_sddmm(const gnn_graph_t *g, int32_t K,
+                                         const gnn_plan_opts_t *opts, const float *X,
+                                         int64_t ldx, float *O, int64_t ldo, float *out,
+                                         void *workspace, size_t ws_bytes,
+                                         gnn_stream_t stream) {
+  if (!g || (!O && !out))
+    return fail(GNN_ERR_INVALID_ARG, "gnn_plan_spmm_sddmm: NULL graph / no output");
+  if (opts && opts->feature_dtype != GNN_F32)
+    return fail(GNN_ERR_UNSUPPORTED, "gnn_plan_spmm_sddmm: fp32 features only");
+  gnn_plan_t plan = nullptr;
+  if (gnn_status_t st = gnn_plan_create(g, K, opts, workspace, ws_bytes, stream, &plan))
+    return st;
+  struct Guard {
+    gnn_plan_t p;
+    ~Guard() { gnn_plan_destroy(p); }
+  } guard{plan};
+  const Plan *p = reinterpret_cast<const Plan *>(plan);
+  cudaStream_t s = (cudaStream_t)stream;
+  SideStream *side = nullptr;
+  const bool fork = O && out && g->nnz > 0;
+  if (fork) {
+    if (gnn_status_t st = side_stream(&side)) return st;
+    cudaError_t e = cudaEventRecord(side->fork, s);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(side->s, side->fork, 0);
+    if (e != cudaSuccess) return cuda_fail(e, "gnn_plan_spmm_sddmm fork");
+  }
+  gnn_status_t st = GNN_OK;
+  if (out)  // A1 = the graph's own rows of X (row_base), A2T = all of X
+    st = launch_sddmm(p, g, X ? X + g->row_base * ldx : nullptr, ldx, X, ldx, out,
+                      fork ? side->s : s, GNN_F32, "gnn_plan_spmm_sddmm sddmm", -1, 0);
+  if (st == GNN_OK && O)
+    st = launch_spmm(p, g, X, ldx, O, ldo, s, GNN_F32, GNN_AGG_SUM, 0,
+                     "gnn_plan_spmm_sddmm spmm", -1, 0);
+  if (fork) {  // join even after an error, so `stream` covers everything enqueued
+    cudaError_t e = cudaEventRecord(side->join, side->s);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(s, side->join, 0);
+    if (e != cudaSuccess && st == GNN_OK) st = cuda_fail(e, "gnn_plan_spmm_sddmm join");
+  }
+  return st;
+}
+
+}  // extern "C"

@@ -732,3 +732,48 @@ def test_feature_matrix_beyond_4GB(dtype):
     assert_within(O, r, T, what=f"spmm {dtype} X > 4 GB")
     r2, T2 = oracle.sddmm(g.row_ind, col_s, g.val, A1s, Xs)
     assert_within(E, r2, T2, what=f"sddmm {dtype} X > 4 GB")
+
+
+def test_plan_spmm_sddmm_one_call():
+    """gnn_plan_spmm_sddmm (plan + SpMM + SDDMM with A1 = A2T = X in one native call, the
+    SDDMM on a forked side stream; the plan workspace reused across graphs): every output
+    against the oracle on sampled subgraphs of different sizes, a row shard (row_base > 0,
+    A1 = the shard's rows of X) and the single-output forms."""
+    run = gs.StepRunner()
+    for t in (0, 1, 2, 0):
+        g = configs.make_c3(t)
+        dg = upload(g)
+        X = _x(960 + t, g.N, 128)
+        Xd = torch.from_numpy(X).to(DEV)
+        O = torch.full((g.M, 128), float("nan"), device=DEV)
+        E = torch.full((g.nnz,), float("nan"), device=DEV)
+        run(dg, Xd, O, E)
+        torch.cuda.synchronize()
+        r, T = oracle.spmm(g.row_ind, g.col_ind, g.val, X, M=g.M)
+        assert_within(O.cpu().numpy(), r, T, what=f"one-call spmm t={t}")
+        r2, T2 = oracle.sddmm(g.row_ind, g.col_ind, g.val, X, X)
+        assert_within(E.cpu().numpy(), r2, T2, what=f"one-call sddmm t={t}")
+    # row shard [r0, r1) of a square graph
+    g = configs.make_graph("C2")
+    r0, r1 = 5000, 12000
+    e0, e1 = int(g.row_ptr[r0]), int(g.row_ptr[r1])
+    full = upload(g)
+    sh = full.shard(r0, r1, e0, e1)
+    X = _x(970, g.N, 64)
+    Xd = torch.from_numpy(X).to(DEV)
+    O = torch.full((r1 - r0, 64), float("nan"), device=DEV)
+    E = torch.full((e1 - e0,), float("nan"), device=DEV)
+    run(sh, Xd, O, E)
+    torch.cuda.synchronize()
+    r, T = oracle.spmm(g.row_ind, g.col_ind, g.val, X, i0=e0, i1=e1, r0=r0, nrows=r1 - r0)
+    assert_within(O.cpu().numpy(), r, T, what="one-call spmm shard")
+    r2, T2 = oracle.sddmm(g.row_ind, g.col_ind, g.val, X, X, i0=e0, i1=e1)
+    assert_within(E.cpu().numpy(), r2, T2, what="one-call sddmm shard")
+    # one output only
+    E2 = torch.full((e1 - e0,), float("nan"), device=DEV)
+    run(sh, Xd, None, E2)
+    O2 = torch.full((r1 - r0, 64), float("nan"), device=DEV)
+    run(sh, Xd, O2, None)
+    torch.cuda.synchronize()
+    assert torch.equal(E2, E)  # SDDMM writes each output once: bit-reproducible
+    assert_within(O2.cpu().numpy(), r, T, what="one-call spmm only")  # (atomics: not bitwise)
