@@ -659,7 +659,8 @@ def run_c3(args, dev, world, rank):
     three_ms = sum(st)
     my_ms = sum(native_st) if native_st else three_ms
     if world > 1:
-        t = torch.tensor([my_ms, float(nbytes)], dtype=torch.float64)
+        t = torch.tensor([my_ms, float(nbytes)], dtype=torch.float64,
+                         device=dev if dist.get_backend() == "nccl" else "cpu")
         mx, sm = t.clone(), t.clone()
         dist.all_reduce(mx, op=dist.ReduceOp.MAX)
         dist.all_reduce(sm, op=dist.ReduceOp.SUM)
