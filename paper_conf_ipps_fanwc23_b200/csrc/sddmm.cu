@@ -35,9 +35,21 @@ gnn_status_t launch_sddmm(const Plan *p, const gnn_graph_t *g, const void *A1, i
                 "%s: A1/A2T must be %d-byte aligned with pitches multiple of %d", who, ES * VW,
                 VW);
   const int vws = effective_vws(in.vw_sparse, g, out);
-  const int V = in.lanes * in.vecs;  // vectors per K-slice
-  SddmmFn f = dtype == GNN_BF16 ? pick_sddmm_bf16(VW, V, vws, in.slices)
-                                : pick_sddmm_f32(VW, V, vws, in.slices);
+  int V = in.lanes * in.vecs;  // vectors per K-slice
+  int VWk = VW;
+#if GNN_SDDMM_BF16_NARROW
+  // bf16 single-slice rows held as two 16-element vectors (K = 32): a 2-lane dot product
+  // leaves the butterfly nothing to batch; as four 8-element vectors (4-lane dot
+  // products) the kernel measured 0.82 -> 0.69 ms on C4 (profiles/r01_sweep36).  SpMM
+  // keeps the plan's 16-wide vectors (faster there).  The plan's alignment check for 16
+  // elements covers 8.
+  if (dtype == GNN_BF16 && in.slices == 1 && VW == 16 && V == 2) {
+    VWk = 8;
+    V = 4;
+  }
+#endif
+  SddmmFn f = dtype == GNN_BF16 ? pick_sddmm_bf16(VWk, V, vws, in.slices)
+                                : pick_sddmm_f32(VWk, V, vws, in.slices);
   if (!f)
     return fail(GNN_ERR_UNSUPPORTED, "%s: K=%d needs %d slices (max 4 at vw=%d)", who, K,
                 in.slices, VW);

@@ -21,6 +21,9 @@ namespace gnn {
 #ifndef GNN_SDDMM_UR
 #define GNN_SDDMM_UR 8       // U * Rsd: feature vectors in flight per lane
 #endif
+#ifndef GNN_SDDMM_BF16_NARROW
+#define GNN_SDDMM_BF16_NARROW 1  // bf16 K = 32: 4 lanes x 8 instead of 2 lanes x 16
+#endif
 #ifndef GNN_SDDMM_PIPE
 #define GNN_SDDMM_PIPE 1     // next batch's loads issued before this batch's reduction
 #endif
