@@ -234,10 +234,29 @@ gnn_status_t launch_spmm(const Plan *p, const gnn_graph_t *g, const void *A, int
   // budget (ptxas: 308 B); 2-wide sparse copies halve the batch and remove the spill
   if (dtype == GNN_BF16 && in.vecs == 2 && vws > 2) vws = 2;
 #endif
-  SpmmFn f = pick_spmm(dtype, VW, in.lanes, in.vecs, vws, agg);
+  int lanes = in.lanes, vecs = in.vecs;
+#ifndef GNN_SPMM_BF16_R2_WIDEN
+#define GNN_SPMM_BF16_R2_WIDEN 1  // measured: bf16 K=256 SpMM 4.30 -> 3.96 ms (r01_sweep43)
+#endif
+#ifndef GNN_SPMM_F32_R2_WIDEN
+#define GNN_SPMM_F32_R2_WIDEN 0
+#endif
+  // Rows of two vectors per lane (R = 2) run as one vector per lane on twice the lanes:
+  // half the accumulators per lane (no spill with 2-wide sparse copies), half the
+  // nonzeros in flight per warp; each output element is summed in the same order, so the
+  // results are identical.
+  if (agg == kAggSum && vecs == 2 && lanes <= 16 &&
+      ((dtype == GNN_BF16 && GNN_SPMM_BF16_R2_WIDEN) ||
+       (dtype == GNN_F32 && GNN_SPMM_F32_R2_WIDEN))) {
+    lanes *= 2;
+    vecs = 1;
+    vws = effective_vws(in.vw_sparse, g, nullptr);
+    if (vws > 2) vws = 2;
+  }
+  SpmmFn f = pick_spmm(dtype, VW, lanes, vecs, vws, agg);
   if (!f)
     return fail(GNN_ERR_UNSUPPORTED, "%s: no kernel for vw=%d L=%d agg=%d dtype=%d", who, VW,
-                in.lanes, agg_api, dtype);
+                lanes, agg_api, dtype);
   SparseArgs a = make_args(p, g);
   a.accum = accumulate;
   a.carry = p->carry;
@@ -261,12 +280,12 @@ gnn_status_t launch_spmm(const Plan *p, const gnn_graph_t *g, const void *A, int
       default: spmm_prezero_kernel<8><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, init); break;
     }
   }
-  const size_t smem = (size_t)in.warps_per_block * spmm_tile_bytes_per_warp(in.lanes, vws);
+  const size_t smem = (size_t)in.warps_per_block * spmm_tile_bytes_per_warp(lanes, vws);
   if (smem > 48 * 1024) {
     cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return cuda_fail(e, "gnn_spmm smem attribute");
   }
-  const int64_t per_block = (int64_t)(32 / in.lanes) * in.warps_per_block;  // items / block
+  const int64_t per_block = (int64_t)(32 / lanes) * in.warps_per_block;  // items / block
   const int64_t grid = (nch * in.slices + per_block - 1) / per_block;
   f<<<(unsigned)grid, threads, smem, s>>>(a, A, lda, O, ldo);
   if (a.carry) {
