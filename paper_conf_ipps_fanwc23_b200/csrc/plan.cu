@@ -91,6 +91,12 @@ gnn_status_t make_info(int64_t M, int64_t nnz, int32_t K, const gnn_plan_opts_t 
       if (rows <= rows_fit) Cl = c;
     }
     C = Cl;
+    // step 5c (B200 addition, on with the cap): chunk floor 64.  On graphs that fill
+    // fewer than alpha waves (sampled subgraphs) Eq. 5 falls to 8 or 32, where the sparse
+    // loads are scalar and each chunk's fixed cost dominates; C* = 64 measured faster on
+    // every C3 subgraph mix (K=32 0.053 -> 0.044 ms, K=128 0.080 -> 0.073 ms;
+    // profiles/r01_sweep45).
+    if (C < 64) C = 64;
   }
   if (o.force_chunk > 0) C = o.force_chunk;
   // step 6: sparse vector width (HVMA)

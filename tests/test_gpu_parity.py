@@ -72,7 +72,8 @@ def run_full(g, K, seed=7, check_sddmm=True, with_val=True, ld_pad=0, **kw):
 def test_c1_tiny_powerlaw_k32():
     g = configs.make_graph("C1")
     info, _ = run_full(g, 32)
-    assert info["chunk"] == 8  # Eq. 5 infeasible on 148 SMs -> most parallel candidate
+    assert info["chunk_dtp"] == 8  # Eq. 5 infeasible on 148 SMs -> most parallel candidate
+    assert info["chunk"] == 64     # ... raised by the step-5c chunk floor
 
 
 def test_c2_cora_shaped_k64():
@@ -656,7 +657,9 @@ def test_locality_cap_plan_and_parity(no_locality):
     no_locality the plain DTP choice is kept."""
     rng = np.random.default_rng(31)
     M = 200_000
-    rows = np.sort(rng.integers(0, M, 800_000))
+    # 3.2 M nonzeros (degree 16): DTP picks 128-512 and the cap 64-128 (the step-5c floor
+    # of 64 leaves the cap visible; 0.8 M nonzeros had DTP itself at 64)
+    rows = np.sort(rng.integers(0, M, 3_200_000))
     g = gen.from_coo(M, M, rows, rng.integers(0, M, rows.size), gen.uniform_values(8, rows.size))
     info, _ = run_full(g, 256, no_locality=no_locality)
     if no_locality:

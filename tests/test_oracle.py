@@ -293,10 +293,11 @@ def test_plan_dtp_maximality_bruteforce(nnz, K, alpha, abs_):
 #   the rows fit, 32,768): C = 256 -> 48,496 rows > 32,768; C = 128 -> 24,248 -> 128.
 # Degree 100 (M = 100,000), fp32: C = 512 -> 24,248 > 16,384; C = 256 -> 12,124 -> 256.
 # Degree 500 (M = 20,000): C = 512 -> 4,849 rows -> 512.  L2 off -> 512.
-# L2 = 1 MiB: 256 rows fit; even C = 8 (37,888 nnz -> 757 rows) does not -> 8.
+# L2 = 1 MiB: 256 rows fit; even C = 8 (37,888 nnz -> 757 rows) does not -> 8, which the
+# step-5c chunk floor (on with the cap) raises to 64.
 @pytest.mark.parametrize("M,dtype,l2,expect", [
     (200_000, 0, 64 << 20, 128), (200_000, 1, 64 << 20, 128), (100_000, 0, 64 << 20, 256),
-    (200_000, 0, 0, 512), (20_000, 0, 64 << 20, 512), (200_000, 0, 1 << 20, 8)])
+    (200_000, 0, 0, 512), (20_000, 0, 64 << 20, 512), (200_000, 0, 1 << 20, 64)])
 def test_plan_locality_cap_worked_examples(M, dtype, l2, expect):
     p = oracle.plan(np.zeros(10_000_000, np.int32), 256, num_sms=148, active_blocks_per_sm=2,
                     feature_dtype=dtype, M=M, l2_bytes=l2)
@@ -307,7 +308,8 @@ def test_plan_locality_cap_worked_examples(M, dtype, l2, expect):
 
 def test_plan_locality_cap_monotone():
     """More L2 never shrinks C*, more rows per nonzero never grows it, the cap never
-    exceeds the DTP choice, and an unbounded L2 (or none) gives DTP exactly."""
+    exceeds the DTP choice except through the step-5c floor of 64, and an unbounded L2
+    gives DTP floored at 64 (no L2 model: DTP exactly)."""
     rng = np.random.default_rng(77)
     cands = [8, 32, 64, 128, 256, 512]
     for _ in range(60):
@@ -327,9 +329,9 @@ def test_plan_locality_cap_monotone():
         prev = 0
         for l2 in (1 << 16, 1 << 20, 16 << 20, 64 << 20, 126 << 20, 1 << 40):
             c = chunk(M, l2)["chunk"]
-            assert c in cands and c <= base["chunk"] and c >= prev
+            assert c in cands and c <= max(base["chunk"], 64) and c >= max(prev, 64)
             prev = c
-        assert prev == base["chunk"]
+        assert prev == max(base["chunk"], 64)
         c_small_m = chunk(max(1, M // 4), 64 << 20)["chunk"]
         assert c_small_m >= chunk(M, 64 << 20)["chunk"]
 
