@@ -11,7 +11,7 @@ NVFLAGS := -ccbin /usr/bin/g++ $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC
            -Xcompiler -fvisibility=hidden -Iinclude --expt-relaxed-constexpr -Xptxas -v
 CUSRC   := $(wildcard $(PKG)/csrc/*.cu) $(wildcard $(PKG)/csrc/*.cpp)
 CUHDR   := $(wildcard $(PKG)/csrc/*.cuh) include/gnn_sparse.h
-OBJDIR  := build/obj$(if $(TAG),_$(TAG),)
+OBJDIR  := $(if $(TAG),/tmp/gnn_obj_$(TAG),build/obj)
 OBJS    := $(patsubst $(PKG)/csrc/%,$(OBJDIR)/%.o,$(CUSRC))
 
 all: gen/libgnngen.so oracle/liboracle.so $(PKG)/libgnnsparse.so
@@ -31,10 +31,11 @@ $(PKG)/libgnnsparse.so: $(OBJS)
 	$(NVCC) $(ARCH) -shared -cudart static -o $@ $(OBJS)
 	cat $(OBJDIR)/*.ptxas.log > $(PKG)/ptxas.log
 
-# tuning variants: make -j variant TAG=x DEFS="-DGNN_SPMM_MINB=2 ..." -> build/libgnnsparse_x.so
+# tuning variants: make -j variant TAG=x DEFS="-DGNN_SPMM_REGS=80 ..." -> variants/libgnnsparse_x.so
+# (variants/ travels to the GPU box; build/ does not)
 variant: $(OBJS)
-	@mkdir -p build
-	$(NVCC) $(ARCH) -shared -cudart static -o build/libgnnsparse_$(TAG).so $(OBJS)
+	@mkdir -p variants build
+	$(NVCC) $(ARCH) -shared -cudart static -o variants/libgnnsparse_$(TAG).so $(OBJS)
 	cat $(OBJDIR)/*.ptxas.log > build/ptxas_$(TAG).log
 
 # measurement probes (tools/microbench.py), not part of the product

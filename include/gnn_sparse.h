@@ -80,8 +80,15 @@ typedef struct {
                               through per-chunk partials in the workspace (no atomics:
                               bit-reproducible; workspace grows by 8*K B per chunk)     */
   int32_t feature_dtype;   /* gnn_dtype_t of the feature matrices; default GNN_F32   */
-  int32_t no_locality;     /* 1: plain DTP, skip the L2 locality cap (DESIGN.md §3
-                              step 5b); 0 (default) applies it                       */
+  int32_t no_locality;     /* 1: plain DTP exactly as InEq. (5): skips
+                              the L2 locality cap (DESIGN.md §3 step 5b) AND the chunk
+                              floor (step 5c); 0 (default) applies both              */
+  /* Device-parameter overrides (0 = query the current device).  They change only the
+   * plan's arithmetic (DTP's NumSM, ActiveblocksPerSM and the cap's L2 size), never the
+   * launch: tests use them to feed identical inputs to the library and the oracle. */
+  int32_t num_sms;              /* NumSM of Eq. 4                                      */
+  int32_t active_blocks_per_sm; /* ActiveblocksPerSM of Eq. 3 (else the occupancy API) */
+  int64_t l2_bytes;             /* L2 bytes of step 5b (no_locality still disables it) */
 } gnn_plan_opts_t;
 
 /* What the plan decided (all integers; bit-exact with the oracle's plan). */
@@ -120,8 +127,9 @@ GNN_API size_t gnn_plan_workspace_bytes(int64_t M, int64_t nnz, int32_t K,
  * per-chunk boundary table of the hybrid-parallel strategy (Algo 3 lines
  * 2-3 P:175-176).  Host part: C* from InEq. (5) over the candidate set
  * {8,32,64,128,256,512}, capped so that the feature rows of the rows in flight fit a
- * quarter of L2 (DESIGN.md §3 step 5b, a B200 addition to DTP), scalar integer
- * arithmetic only -- no device read, no sync.
+ * quarter of L2 (DESIGN.md §3 step 5b, a B200 addition to DTP), then raised to 64 where
+ * InEq. (5) itself chose 8 or 32 (step 5c, B200 addition); no_locality skips 5b and 5c.
+ * Scalar integer arithmetic only -- no device read, no sync.
  * Device part: one launch writing, for every chunk c (nnz [c*C*, min((c+1)*C*, nnz))),
  *   row_first[c] = row_ind[start], row_last[c] = row_ind[end-1],
  *   flags[c] = (head row continues from chunk c-1) | (tail row continues into c+1) << 1.

@@ -152,6 +152,17 @@ def spmm_rows(g, A, rows):
     return O, T
 
 
+def sddmm_edges(g, A1, A2T, edges):
+    """Oracle outputs for a sample of edge ids (full-size parity): (out, T), each edge
+    Algorithm 2 over that one nonzero."""
+    out = np.empty(len(edges), np.float64)
+    T = np.empty(len(edges), np.float64)
+    for j, e in enumerate(edges):
+        a, b = sddmm(g.row_ind, g.col_ind, g.val, A1, A2T, i0=int(e), i1=int(e) + 1)
+        out[j], T[j] = a[0], b[0]
+    return out, T
+
+
 def sddmm(row_ind, col_ind, val, A1, A2T, i0=0, i1=None):
     """Algorithm 2 over nnz [i0, i1): returns (out, T) fp64 of length i1-i0."""
     lib = _load()

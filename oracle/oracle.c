@@ -226,8 +226,8 @@ int oracle_plan(int64_t nnz, const int32_t *row_ind, int32_t K, int32_t alpha,
     }
     C = capped;
     /* step 5c (a B200 reading -- not in the paper; on with the
-     * cap): C = max(C, 64). */
-    if (C < 64) C = 64;
+     * cap): where InEq. (5) itself chose fewer than 64 nonzeros per chunk, C = 64. */
+    if (C_dtp < 64) C = 64;
   }
   if (force_chunk > 0) C = force_chunk;
   /* step 6: sparse-load vector width (HVMA) */

@@ -49,7 +49,8 @@ class PlanOpts(ctypes.Structure):
     _fields_ = [("alpha", ctypes.c_int32), ("warps_per_block", ctypes.c_int32),
                 ("force_chunk", ctypes.c_int32), ("force_vw", ctypes.c_int32),
                 ("deterministic", ctypes.c_int32), ("feature_dtype", ctypes.c_int32),
-                ("no_locality", ctypes.c_int32)]
+                ("no_locality", ctypes.c_int32), ("num_sms", ctypes.c_int32),
+                ("active_blocks_per_sm", ctypes.c_int32), ("l2_bytes", ctypes.c_int64)]
 
 
 class _PlanInfo(ctypes.Structure):
@@ -266,21 +267,26 @@ def _dtype_code(d):
 
 
 def _opts(alpha=0, warps_per_block=0, force_chunk=0, force_vw=0, feature_dtype=0,
-          deterministic=False, no_locality=False):
+          deterministic=False, no_locality=False, num_sms=0, active_blocks_per_sm=0,
+          l2_bytes=0):
     return PlanOpts(alpha, warps_per_block, force_chunk, force_vw, int(bool(deterministic)),
-                    _dtype_code(feature_dtype), int(bool(no_locality)))
+                    _dtype_code(feature_dtype), int(bool(no_locality)), num_sms,
+                    active_blocks_per_sm, l2_bytes)
 
 
 def plan(graph: DeviceGraph, K: int, alpha: int = 0, warps_per_block: int = 0,
          force_chunk: int = 0, force_vw: int = 0, feature_dtype=GNN_F32,
-         deterministic: bool = False, no_locality: bool = False, stream=None) -> Plan:
+         deterministic: bool = False, no_locality: bool = False, num_sms: int = 0,
+         active_blocks_per_sm: int = 0, l2_bytes: int = 0, stream=None) -> Plan:
     """gnn_plan_create: DTP/HVMA chunking + the GPU plan kernel (no host sync).
     feature_dtype: fp32 (default) or bf16 feature matrices.
     deterministic: split rows summed in chunk order without atomics (bit-reproducible).
-    no_locality: plain DTP, without the L2 locality cap (DESIGN.md §3 step 5b)."""
+    no_locality: plain DTP (InEq. 5), without the L2 locality cap and the chunk floor
+    (DESIGN.md §3 steps 5b, 5c).  num_sms / active_blocks_per_sm / l2_bytes: device-
+    parameter overrides for the plan arithmetic only (0 = the device's)."""
     L = lib()
     o = _opts(alpha, warps_per_block, force_chunk, force_vw, feature_dtype, deterministic,
-              no_locality)
+              no_locality, num_sms, active_blocks_per_sm, l2_bytes)
     nbytes = L.gnn_plan_workspace_bytes(graph.M, graph.nnz, K, ctypes.byref(o))
     if nbytes == ctypes.c_size_t(-1).value:
         _check(GNN_ERR_INVALID_ARG)
@@ -293,9 +299,26 @@ def plan(graph: DeviceGraph, K: int, alpha: int = 0, warps_per_block: int = 0,
     return Plan(h, ws, graph, K)
 
 
-def _dense(t, name, dtypes=(torch.float32,)):
-    if t.dtype not in dtypes or t.dim() != 2 or t.stride(1) != 1 or not t.is_cuda:
+def _dense(t, name, dtypes=(torch.float32,), rows=None, cols=None, device=None):
+    """Check a dense operand before its pointer reaches a kernel: CUDA, row-major 2-D,
+    dtype, at least `rows` x `cols`, on `device` (the library reads / writes rows x cols
+    elements at pitch stride(0); a smaller tensor would be accessed out of bounds)."""
+    if (not torch.is_tensor(t) or t.dtype not in dtypes or t.dim() != 2 or t.stride(1) != 1
+            or not t.is_cuda):
         raise ValueError(f"{name} must be a CUDA row-major 2-D tensor of {dtypes}")
+    if (rows is not None and t.shape[0] < rows) or (cols is not None and t.shape[1] < cols):
+        raise ValueError(f"{name} is {tuple(t.shape)}, needs at least ({rows}, {cols})")
+    if device is not None and t.device != device:
+        raise ValueError(f"{name} is on {t.device}, the graph on {device}")
+    return t
+
+
+def _vec_out(t, name, n, device):
+    """A caller-supplied SDDMM output: contiguous fp32 CUDA vector of >= n elements."""
+    if (not torch.is_tensor(t) or t.dtype != torch.float32 or not t.is_cuda
+            or not t.is_contiguous() or t.numel() < n or t.device != device):
+        raise ValueError(f"{name} must be a contiguous fp32 tensor of >= {n} elements on "
+                         f"{device}")
     return t
 
 
@@ -310,12 +333,13 @@ def spmm(p: Plan, graph: DeviceGraph, A: torch.Tensor, out: torch.Tensor | None 
     """gnn_spmm: O = S A (overwrites out; returns it).  agg / accumulate select
     gnn_spmm_ex: (+) in {sum, mean, max, min}; accumulate=True computes O += S A."""
     K = p.K
-    _dense(A, "A", _FEAT)
+    dev = graph.row_ind.device
+    _dense(A, "A", _FEAT, rows=graph.N if graph.nnz else 0, cols=K, device=dev)
     if out is None:
         if accumulate:
             raise ValueError("accumulate=True needs an existing out")
         out = torch.empty((graph.M, K), dtype=torch.float32, device=A.device)
-    _dense(out, "out")
+    _dense(out, "out", rows=graph.M, cols=K, device=dev)
     g = graph.desc()
     if agg != "sum" or accumulate:
         _check(lib().gnn_spmm_ex(p.handle, ctypes.byref(g), _ptr(A), A.stride(0), _ptr(out),
@@ -360,7 +384,13 @@ class StepRunner:
 
     def __call__(self, graph: DeviceGraph, X: torch.Tensor, O: torch.Tensor | None,
                  out: torch.Tensor | None, stream=None):
+        dev = graph.row_ind.device
+        _dense(X, "X", rows=max(graph.N, graph.row_base + graph.M), device=dev)
         K = X.shape[1]
+        if O is not None:
+            _dense(O, "O", rows=graph.M, cols=K, device=dev)
+        if out is not None:
+            _vec_out(out, "out", graph.nnz, dev)
         L = lib()
         nbytes = L.gnn_plan_workspace_bytes(graph.M, graph.nnz, K, ctypes.byref(self.opts))
         if nbytes == ctypes.c_size_t(-1).value:
@@ -396,10 +426,13 @@ def transpose(graph: DeviceGraph, stream=None):
 def sddmm(p: Plan, graph: DeviceGraph, A1: torch.Tensor, A2T: torch.Tensor,
           out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
     """gnn_sddmm: out[i] = val[i] * <A1[row_i], A2T[col_i]> (returns out)."""
-    _dense(A1, "A1", _FEAT)
-    _dense(A2T, "A2T", (A1.dtype,))
+    dev = graph.row_ind.device
+    K = p.K
+    _dense(A1, "A1", _FEAT, rows=graph.M if graph.nnz else 0, cols=K, device=dev)
+    _dense(A2T, "A2T", (A1.dtype,), rows=graph.N if graph.nnz else 0, cols=K, device=dev)
     if out is None:
         out = torch.empty(graph.nnz, dtype=torch.float32, device=A1.device)
+    _vec_out(out, "out", graph.nnz, dev)
     g = graph.desc()
     fn = lib().gnn_sddmm_bf16 if A1.dtype == torch.bfloat16 else lib().gnn_sddmm
     _check(fn(p.handle, ctypes.byref(g), _ptr(A1), A1.stride(0), _ptr(A2T), A2T.stride(0),

@@ -64,12 +64,17 @@ gnn_status_t make_info(int64_t M, int64_t nnz, int32_t K, const gnn_plan_opts_t 
   while (L < cdiv(need, R) && L < 32) L *= 2;
   const int32_t S = (int32_t)cdiv(K, (int64_t)L * R * vw);
   const int32_t G = 32 / L;
-  // step 3: FullWaveSize (Eqs. 3-4) from the occupancy of the SpMM kernel
+  // step 3: FullWaveSize (Eqs. 3-4) from the occupancy of the SpMM kernel, unless the
+  // caller overrides the device parameters (tests feed the same values to the oracle)
+  if (o.num_sms < 0 || o.active_blocks_per_sm < 0 || o.l2_bytes < 0)
+    return fail(GNN_ERR_INVALID_ARG, "plan: negative device-parameter override");
   DeviceInfo d;
   if (gnn_status_t st = device_info(&d)) return st;
-  const int32_t abs = spmm_active_blocks_per_sm(dt, vw, L, R, wpb);
+  const int32_t nsm = o.num_sms ? o.num_sms : d.num_sms;
+  const int32_t abs = o.active_blocks_per_sm ? o.active_blocks_per_sm
+                                             : spmm_active_blocks_per_sm(dt, vw, L, R, wpb);
   if (abs < 1) return fail(GNN_ERR_CUDA, "plan: occupancy query failed (vw=%d L=%d)", vw, L);
-  const int64_t FW = (int64_t)d.num_sms * abs;
+  const int64_t FW = (int64_t)nsm * abs;
   // steps 4-5: the largest candidate satisfying InEq. (5); none -> 8
   int32_t C = 8;
   for (int32_t c : kCand)
@@ -79,7 +84,7 @@ gnn_status_t make_info(int64_t M, int64_t nnz, int32_t K, const gnn_plan_opts_t 
   // about that many * C / (nnz / M) rows in flight; after a clustering reorder their
   // feature rows are the L2 working set, so C* is the largest candidate <= C_dtp whose
   // rows in flight fit a quarter of L2 (else 8).
-  const int64_t l2 = o.no_locality ? 0 : d.l2_bytes;  // 0: cap off (reported in the info)
+  const int64_t l2 = o.no_locality ? 0 : (o.l2_bytes ? o.l2_bytes : d.l2_bytes);  // 0: cap off
   if (l2 > 0 && nnz > 0 && M > 0) {
     const int64_t eb = dt == GNN_BF16 ? 2 : 4;
     const int64_t rows_fit = (l2 / 4) / ((int64_t)K * eb);
@@ -91,12 +96,13 @@ gnn_status_t make_info(int64_t M, int64_t nnz, int32_t K, const gnn_plan_opts_t 
       if (rows <= rows_fit) Cl = c;
     }
     C = Cl;
-    // step 5c (B200 addition, on with the cap): chunk floor 64.  On graphs that fill
-    // fewer than alpha waves (sampled subgraphs) Eq. 5 falls to 8 or 32, where the sparse
-    // loads are scalar and each chunk's fixed cost dominates; C* = 64 measured faster on
-    // every C3 subgraph mix (K=32 0.053 -> 0.044 ms, K=128 0.080 -> 0.073 ms;
-    // profiles/r01_sweep45).
-    if (C < 64) C = 64;
+    // step 5c (B200 addition, on with the cap): chunk floor 64 where Eq. 5 itself fell
+    // below 64.  On graphs that fill fewer than alpha waves (sampled subgraphs) Eq. 5 gives
+    // 8 or 32, where the sparse loads are scalar and each chunk's fixed cost dominates;
+    // C* = 64 measured faster on every C3 subgraph mix (K=32 0.053 -> 0.044 ms, K=128
+    // 0.080 -> 0.073 ms; profiles/r01_sweep45).  A cap below 64 on a graph where Eq. 5
+    // was feasible at >= 64 stands (locality, not parallelism, decided it).
+    if (C_dtp < 64) C = 64;
   }
   if (o.force_chunk > 0) C = o.force_chunk;
   // step 6: sparse vector width (HVMA)
@@ -113,7 +119,7 @@ gnn_status_t make_info(int64_t M, int64_t nnz, int32_t K, const gnn_plan_opts_t 
   info->groups = G;
   info->warps_per_block = wpb;
   info->active_blocks_per_sm = abs;
-  info->num_sms = d.num_sms;
+  info->num_sms = nsm;
   info->alpha = alpha;
   info->K = K;
   info->feature_dtype = dt;

@@ -35,11 +35,17 @@ struct SddmmShape {
   static constexpr int R = (V >= GNN_SDDMM_R2_FROM && V >= 2) ? 2 : 1;
   static constexpr int Lg = V / R;
   static constexpr int depth = GNN_SDDMM_UR / R > 1 ? GNN_SDDMM_UR / R : 1;
-#if defined(GNN_SDDMM_MINB)
-  static constexpr int minb = GNN_SDDMM_MINB;
-#else
-  static constexpr int minb = 1;
+};
+// Register budget per thread: 128 = 2 resident blocks of 8 warps per SM, 80 = 3, 64 = 4.
+#ifndef GNN_SDDMM_REGS
+#define GNN_SDDMM_REGS 128
 #endif
+#ifndef GNN_SDDMM_REGS_BF16
+#define GNN_SDDMM_REGS_BF16 GNN_SDDMM_REGS
+#endif
+template <typename TF>
+struct SddmmRegs {
+  static constexpr int value = TF::bytes == 2 ? GNN_SDDMM_REGS_BF16 : GNN_SDDMM_REGS;
 };
 
 // WarpReduce (Algo 4 line 12) of U partial dot products at once over the group's L
@@ -120,7 +126,7 @@ __device__ __forceinline__ void reduce_scale_store(float (&part)[U], const float
 
 // L here is V, the number of VW-wide vectors in one K-slice (plan lanes x vecs).
 template <typename TF, int VW, int L, int VWS, int SMAX>
-__global__ void __launch_bounds__(kMaxThreads, (SddmmShape<VW, L, SMAX>::minb))
+__global__ void __maxnreg__(SddmmRegs<TF>::value)
     sddmm_kernel(const SparseArgs a, const void *__restrict__ A1, const int64_t lda1,
                  const void *__restrict__ A2T, const int64_t lda2, float *__restrict__ out) {
   constexpr int ES = TF::bytes;

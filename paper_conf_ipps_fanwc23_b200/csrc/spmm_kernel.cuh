@@ -11,9 +11,18 @@ namespace gnn {
 // Feature rows in flight per lane (U) and the register budget, per instantiation.
 // Measured on C4 (profiles/r01_sweep4.txt): with 256-bit loads U = 4 is best while
 // several chunks share a warp (L <= 8), U = 8 once a group spans >= 16 lanes.
-#ifndef GNN_SPMM_MINB
-#define GNN_SPMM_MINB 1  // min resident 512-thread blocks/SM the register budget must allow
+// Register budget per thread (the occupancy lever of PAPER.md P:392, "register pressure"
+// at large K): 128 = 2 resident blocks of 8 warps per SM, 80 = 3, 64 = 4.
+#ifndef GNN_SPMM_REGS
+#define GNN_SPMM_REGS 128
 #endif
+#ifndef GNN_SPMM_REGS_BF16
+#define GNN_SPMM_REGS_BF16 GNN_SPMM_REGS
+#endif
+template <typename TF>
+struct SpmmRegs {
+  static constexpr int value = TF::bytes == 2 ? GNN_SPMM_REGS_BF16 : GNN_SPMM_REGS;
+};
 
 // Feature vectors in flight per lane (U * R).  Measured on the GCR-reordered C4
 // (profiles/r01_sweep12.txt, r01_sweep19.txt): 8, except 4 when a lane holds two
@@ -30,6 +39,19 @@ struct FeatDepth {
   static constexpr int value = R == 2 ? GNN_SPMM_DEPTH_R2 : ((wide && L <= 2) ? 4 : 8);
 #endif
 };
+
+// host mirror of FeatDepth (feature vectors in flight per lane) for the launcher
+inline int spmm_depth(int es, int vw, int L, int R) {
+  const bool wide = vw * es == 32;
+#if defined(GNN_SPMM_DEPTH8)
+  return wide ? GNN_SPMM_DEPTH8 : 8;
+#else
+  return R == 2 ? GNN_SPMM_DEPTH_R2 : ((wide && L <= 2) ? 4 : 8);
+#endif
+}
+#ifndef GNN_SPMM_VWS_CLAMP
+#define GNN_SPMM_VWS_CLAMP 0  // 1: narrow the sparse copies so a batch is depth/R nonzeros
+#endif
 
 // Aggregators of the node-wise MPP op (Eq. 1): ⊕ = sum (SpMM proper; mean is
 // sum followed by a row scale), max or min of the terms v_i * A[col_i].
@@ -97,7 +119,7 @@ __device__ __forceinline__ void accumulate(float (&acc)[VW], float s, const Feat
 // L lanes per (chunk, K-slice) work item, R VW-wide vectors per lane (plan rule step 2).
 // TF: feature element type (F32 or BF16); accumulation and O are fp32.
 template <typename TF, int VW, int L, int R, int VWS, int AGG>
-__global__ void __launch_bounds__(kMaxThreads, GNN_SPMM_MINB)
+__global__ void __maxnreg__(SpmmRegs<TF>::value)
     spmm_kernel(const SparseArgs a, const void *__restrict__ A, const int64_t lda,
                 float *__restrict__ O, const int64_t ldo) {
   constexpr int ES = TF::bytes;

@@ -67,3 +67,29 @@ def test_header_is_plain_c():
     rc = os.system(f"echo '#include \"gnn_sparse.h\"\nint main(void){{return 0;}}' | "
                    f"/usr/bin/gcc -std=c99 -Wall -Werror -I{ROOT}/include -x c - -o /dev/null")
     assert rc == 0
+
+
+def test_binding_struct_layouts_match_header(tmp_path):
+    """The ctypes mirrors of the ABI structs have the header's size and field offsets
+    (a field added to gnn_plan_opts_t / gnn_plan_info_t must be added to the binding)."""
+    structs = {"gnn_plan_opts_t": gs.PlanOpts, "gnn_plan_info_t": gs._PlanInfo,
+               "gnn_graph_t": gs._Graph, "gnn_reorder_opts_t": gs.ReorderOpts}
+    lines = ["#include <stdio.h>", "#include <stddef.h>", '#include "gnn_sparse.h"',
+             "int main(void) {"]
+    for cname, py in structs.items():
+        lines.append(f'printf("{cname} size %zu\\n", sizeof({cname}));')
+        for fname, _ in py._fields_:
+            lines.append(f'printf("{cname} {fname} %zu\\n", offsetof({cname}, {fname}));')
+    lines.append("return 0; }")
+    src = tmp_path / "layout.c"
+    src.write_text("\n".join(lines))
+    exe = tmp_path / "layout"
+    assert os.system(f"/usr/bin/gcc -std=c99 -I{ROOT}/include {src} -o {exe}") == 0
+    got = {}
+    for line in os.popen(str(exe)).read().splitlines():
+        c, f, v = line.split()
+        got[(c, f)] = int(v)
+    for cname, py in structs.items():
+        assert got[(cname, "size")] == ctypes.sizeof(py), cname
+        for fname, _ in py._fields_:
+            assert got[(cname, fname)] == getattr(py, fname).offset, (cname, fname)

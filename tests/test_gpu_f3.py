@@ -10,7 +10,7 @@ import oracle
 import paper_conf_ipps_fanwc23_b200 as gs
 from paper_conf_ipps_fanwc23_b200 import nn as gnn
 
-from helpers import assert_within, upload
+from helpers import oracle_plan_checked, assert_within, upload
 
 pytestmark = pytest.mark.gpu
 DEV = "cuda"
@@ -139,16 +139,14 @@ def test_randomized_configurations(seed):
         kw["alpha"] = int(rng.choice([1, 3, 8]))
     if rng.random() < 0.2:
         kw["no_locality"] = True
+    if rng.random() < 0.2:  # device-parameter overrides, fed to the oracle as well
+        kw["num_sms"] = int(rng.integers(1, 300))
+        kw["active_blocks_per_sm"] = int(rng.integers(1, 17))
+        kw["l2_bytes"] = int(rng.choice([1 << 20, 40 << 20, 126 << 20]))
     with_val = rng.random() < 0.8
     dg = upload(g, with_val=with_val)
     p = gs.plan(dg, K, feature_dtype="bf16" if bf16 else "f32", **kw)
-    info = p.info()
-    ref_plan = oracle.plan(g.row_ind, K, info["num_sms"], info["active_blocks_per_sm"],
-                           alpha=kw.get("alpha", 2), warps_per_block=kw.get("warps_per_block", 8),
-                           force_chunk=kw.get("force_chunk", 0), force_vw=kw.get("force_vw", 0),
-                           feature_dtype=1 if bf16 else 0, M=M,
-                           l2_bytes=0 if kw.get("no_locality") else info["l2_bytes"])
-    assert info == ref_plan.info
+    oracle_plan_checked(p, g, K, feature_dtype="bf16" if bf16 else "f32", **kw)
     X = torch.from_numpy(gen.features(seed, N, K)).to(DEV)
     A1 = torch.from_numpy(gen.features(seed + 1, M, K)).to(DEV)
     if bf16:

@@ -14,7 +14,7 @@ import oracle
 from gen import configs
 import paper_conf_ipps_fanwc23_b200 as gs
 
-from helpers import assert_within, upload
+from helpers import assert_within, oracle_plan_checked, upload
 
 pytestmark = pytest.mark.gpu
 
@@ -27,21 +27,9 @@ def _x(seed, rows, K, ld=None):
 
 
 def check_plan(p, g, K, **kw):
-    info = p.info()
-    # the locality cap reads the device's L2 size (0 when switched off)
-    l2 = 0 if kw.get("no_locality") else torch.cuda.get_device_properties(0).L2_cache_size
-    assert info["l2_bytes"] == l2 and info["M"] == g.M
-    ref = oracle.plan(g.row_ind, K, info["num_sms"], info["active_blocks_per_sm"],
-                      alpha=kw.get("alpha", 2) or 2,
-                      warps_per_block=kw.get("warps_per_block", 8) or 8,
-                      force_chunk=kw.get("force_chunk", 0), force_vw=kw.get("force_vw", 0),
-                      M=g.M, l2_bytes=l2)
-    assert info == ref.info, (info, ref.info)
-    rf, rl, fl = (t.cpu().numpy() for t in p.arrays())
-    assert np.array_equal(rf, ref.row_first)
-    assert np.array_equal(rl, ref.row_last)
-    assert np.array_equal(fl, ref.flags)
-    return info
+    """Plan info + arrays bit-exact with the oracle, which gets the device parameters
+    from torch and the cuobjdump-derived occupancy (helpers.oracle_plan_checked)."""
+    return oracle_plan_checked(p, g, K, **kw)
 
 
 def run_full(g, K, seed=7, check_sddmm=True, with_val=True, ld_pad=0, **kw):
@@ -378,42 +366,113 @@ def _sampled_rows(g, n, seed):
     return np.unique(np.r_[heavy, rand, 0, g.M - 1])
 
 
+_FULL = {}
+
+
+def full_graph(name, reorder):
+    """Full-size BJ graph (C4 Reddit- / C5 products-shaped), GCR-reordered as bench.py
+    runs it when reorder; cached for the module (generation + Louvain take ~10-20 s)."""
+    key = (name, reorder)
+    if key not in _FULL:
+        g = configs.make_graph(name)
+        perm = None
+        if reorder:
+            perm, _, _ = gs.reorder_gcr(g.row_ptr, g.col_ind)
+            rp, ri, ci, v = gs.permute_graph(g.row_ptr, g.col_ind, g.val, perm)
+            g = gen.Graph(g.M, g.N, rp, ri, ci, v)
+        if len(_FULL) >= 2:
+            _FULL.clear()
+        _FULL[key] = (g, perm)
+    return _FULL[key]
+
+
+def _bench_features(name, g, K, perm):
+    """bench.py's X for this K: the workload's features, rows relabelled by the GCR
+    permutation (X' = P X)."""
+    X = configs.make_features(name, g.N, K)
+    if perm is not None:
+        Xp = np.empty_like(X)
+        Xp[perm] = X
+        X = Xp
+    return X
+
+
+def _sampled_check(name, g, dg, p, X, Xd, K, tag, rows, edges, dtype=None):
+    O = gs.spmm(p, dg, Xd)
+    E = gs.sddmm(p, dg, Xd, Xd)
+    torch.cuda.synchronize()
+    ref, T = oracle.spmm_rows(g, X, rows)
+    assert_within(O[torch.from_numpy(rows).to(DEV)].cpu().numpy(), ref, T,
+                  what=f"{name} spmm K={K} {tag}")
+    r2, T2 = oracle.sddmm_edges(g, X, X, edges)
+    assert_within(E[torch.from_numpy(edges).to(DEV)].cpu().numpy(), r2, T2,
+                  what=f"{name} sddmm K={K} {tag}")
+
+
 @pytest.mark.slow
-@pytest.mark.parametrize("name,Ks,reorder", [("C4", (32, 256), False), ("C4", (64, 128), True),
-                                             ("C5", (256,), True)])
+@pytest.mark.parametrize("name,Ks,reorder", [("C4", (32, 64, 128, 256), True),
+                                             ("C4", (32, 256), False), ("C5", (256,), True)])
 def test_full_size_sampled_parity(name, Ks, reorder):
-    """Full-size Reddit / products-shaped graphs, in bench.py's launch configuration
-    (default plan), checked on sampled output rows (SpMM) and edges (SDDMM) that the
-    oracle computes one by one, plus the global plan arrays bit-exactly."""
-    g = configs.make_graph(name)
-    perm = None
-    if reorder:
-        perm, _, _ = gs.reorder_gcr(g.row_ptr, g.col_ind)
-        rp, ri, ci, v = gs.permute_graph(g.row_ptr, g.col_ind, g.val, perm)
-        g = gen.Graph(g.M, g.N, rp, ri, ci, v)
+    """Full-size Reddit / products-shaped graphs in bench.py's launch configuration
+    (default plan; C4 GCR-reordered at every bench K, the headline config), checked on
+    sampled output rows (SpMM) and edges (SDDMM) that the oracle computes one by one,
+    plus the global plan arrays bit-exactly (device parameters derived independently)."""
+    g, perm = full_graph(name, reorder)
     dg = upload(g)
     rows = _sampled_rows(g, 300, 1)
     edges = np.unique(np.r_[np.random.default_rng(2).choice(g.nnz, 20000, replace=False),
-                            g.row_ptr[rows[:50]]])
+                            g.row_ptr[rows[:50]], g.nnz - 1])
     for K in Ks:
-        X = configs.make_features(name, g.N, K)
+        X = _bench_features(name, g, K, perm)
         Xd = torch.from_numpy(X).to(DEV)
         p = gs.plan(dg, K)
         check_plan(p, g, K)
-        O = gs.spmm(p, dg, Xd)
-        E = gs.sddmm(p, dg, Xd, Xd)
-        torch.cuda.synchronize()
-        ref, T = oracle.spmm_rows(g, X, rows)
-        assert_within(O[torch.from_numpy(rows).to(DEV)].cpu().numpy(), ref, T,
-                      what=f"{name} spmm K={K}")
-        r2 = np.empty(edges.size)
-        T2 = np.empty(edges.size)
-        for j, i in enumerate(edges):
-            a, b = oracle.sddmm(g.row_ind, g.col_ind, g.val, X, X, i0=int(i), i1=int(i) + 1)
-            r2[j], T2[j] = a[0], b[0]
-        assert_within(E[torch.from_numpy(edges).to(DEV)].cpu().numpy(), r2, T2,
-                      what=f"{name} sddmm K={K}")
-        del O, E, Xd
+        _sampled_check(name, g, dg, p, X, Xd, K, "default plan", rows, edges)
+        del Xd
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("name", ["C4", "C5"])
+def test_full_size_paper_rule_plan(name):
+    """The paper's DTP rule exactly (no_locality: InEq. 5 over the candidate set, no
+    B200 cap / floor) at full C4 / C5 size: plan bit-exact with the oracle at every
+    width bench.py runs, C* equal to the brute-force largest candidate with >= alpha full
+    waves, and outputs within the bar on samples under that plan."""
+    g, perm = full_graph(name, True)
+    dg = upload(g)
+    rows = _sampled_rows(g, 150, 5)
+    edges = np.unique(np.random.default_rng(6).choice(g.nnz, 5000, replace=False))
+    Ks = (32, 64, 128, 256) if name == "C4" else (256,)
+    for K in Ks:
+        p = gs.plan(dg, K, no_locality=True)
+        info = check_plan(p, g, K, no_locality=True)
+        FW = info["num_sms"] * info["active_blocks_per_sm"]
+        S, G, W = info["slices"], info["groups"], info["warps_per_block"]
+        cdiv = lambda a, b: -(-a // b)
+        blocks = lambda C: cdiv(cdiv(cdiv(g.nnz, C) * S, G), W)  # InEq. 5 RHS, P:254
+        ok = [C for C in (8, 32, 64, 128, 256, 512) if blocks(C) >= 2 * FW]
+        assert info["chunk"] == info["chunk_dtp"] == (max(ok) if ok else 8)
+        if K in (32, 256):
+            X = _bench_features(name, g, K, perm)
+            Xd = torch.from_numpy(X).to(DEV)
+            _sampled_check(name, g, dg, p, X, Xd, K, "paper rule", rows, edges)
+            del Xd
+
+
+@pytest.mark.slow
+def test_full_size_bf16_bench_config():
+    """bench.py's bf16 leg at full size (C4, GCR, K = 32 and 256): exact-input parity
+    (the oracle gets the bf16 values) on samples."""
+    g, perm = full_graph("C4", True)
+    dg = upload(g)
+    rows = _sampled_rows(g, 150, 7)
+    edges = np.unique(np.random.default_rng(8).choice(g.nnz, 5000, replace=False))
+    for K in (32, 256):
+        Xb = torch.from_numpy(_bench_features("C4", g, K, perm)).to(torch.bfloat16)
+        X = Xb.float().numpy()
+        p = gs.plan(dg, K, feature_dtype="bf16")
+        check_plan(p, g, K, feature_dtype="bf16")
+        _sampled_check("C4", g, dg, p, X, Xb.to(DEV), K, "bf16", rows, edges)
 
 
 # ------------------------------------------------------------ bf16 (f2) ----
@@ -433,10 +492,7 @@ def test_bf16_features_parity(K):
     g = gen.powerlaw_graph(4000, 120000, gamma=2.2, n_comm=6, seed=500 + K)
     dg = upload(g)
     p = gs.plan(dg, K, feature_dtype="bf16")
-    info = p.info()
-    ref = oracle.plan(g.row_ind, K, info["num_sms"], info["active_blocks_per_sm"],
-                      feature_dtype=1, M=g.M, l2_bytes=info["l2_bytes"])
-    assert info == ref.info
+    check_plan(p, g, K, feature_dtype="bf16")
     Xb, Xexact, X32 = _bf16_pair(600 + K, g.N, K)
     A1b, A1exact, A132 = _bf16_pair(700 + K, g.M, K)
     O = gs.spmm(p, dg, Xb).cpu().numpy()
@@ -589,6 +645,33 @@ def test_run_host_full_size_sampled_parity():
             a, b = oracle.sddmm(g.row_ind, g.col_ind, g.val, X, X, i0=int(e), i1=int(e) + 1)
             r2[i], T2[i] = a[0], b[0]
         assert_within(E.numpy()[edges], r2, T2, what=f"run_host C4 sddmm K={K}")
+
+
+@pytest.mark.slow
+def test_run_host_multi_full_size_bench_config():
+    """bench.py's e2e headline exactly: one gnn_run_host_multi call over K = 32..256 on
+    the GCR-reordered full C4 graph with the default piece count, NaN-prefilled pinned
+    outputs; sampled rows / edges of every width against the oracle (and no element of
+    any output left unwritten)."""
+    g, perm = full_graph("C4", True)
+    Ks = (32, 64, 128, 256)
+    runner = gs.HostRunner(g.M, g.N, g.row_ind, g.col_ind, g.val, max(Ks), device=DEV,
+                           Ks=Ks).pin()
+    Xs = [torch.from_numpy(_bench_features("C4", g, K, perm)).pin_memory() for K in Ks]
+    Os = [torch.full((g.M, K), float("nan")).pin_memory() for K in Ks]
+    Es = [torch.full((g.nnz,), float("nan")).pin_memory() for _ in Ks]
+    runner.run_multi(Xs, Ks, Os, Es, upload_graph=True)
+    torch.cuda.synchronize()
+    rows = _sampled_rows(g, 200, 9)
+    edges = np.unique(np.r_[np.random.default_rng(10).choice(g.nnz, 5000, replace=False),
+                            g.row_ptr[rows[:50]], g.nnz - 1])
+    for j, K in enumerate(Ks):
+        assert not torch.isnan(Os[j]).any() and not torch.isnan(Es[j]).any(), K
+        X = Xs[j].numpy()
+        ref, T = oracle.spmm_rows(g, X, rows)
+        assert_within(Os[j].numpy()[rows], ref, T, what=f"run_host_multi C4 spmm K={K}")
+        r2, T2 = oracle.sddmm_edges(g, X, X, edges)
+        assert_within(Es[j].numpy()[edges], r2, T2, what=f"run_host_multi C4 sddmm K={K}")
 
 
 def _run_multi_check(g, Ks, pieces=None, skip_o=(), seed=950):
@@ -780,3 +863,28 @@ def test_plan_spmm_sddmm_one_call():
     torch.cuda.synchronize()
     assert torch.equal(E2, E)  # SDDMM writes each output once: bit-reproducible
     assert_within(O2.cpu().numpy(), r, T, what="one-call spmm only")  # (atomics: not bitwise)
+
+
+def test_binding_rejects_undersized_or_mistyped_operands():
+    """The Python layer checks every dense operand's dtype, shape and device before a
+    pointer reaches a kernel (an undersized tensor would be read / written out of
+    bounds)."""
+    g = configs.make_graph("C1")
+    dg = upload(g)
+    K = 32
+    p = gs.plan(dg, K)
+    X = torch.zeros((g.N, K), device=DEV)
+    bad = [lambda: gs.spmm(p, dg, X[: g.N - 1]),
+           lambda: gs.spmm(p, dg, torch.zeros((g.N, K - 8), device=DEV)),
+           lambda: gs.spmm(p, dg, X, out=torch.empty((g.M - 1, K), device=DEV)),
+           lambda: gs.sddmm(p, dg, X[: g.M - 1], X),
+           lambda: gs.sddmm(p, dg, X, X, out=torch.empty(g.nnz - 1, device=DEV)),
+           lambda: gs.sddmm(p, dg, X, X, out=torch.empty(g.nnz, dtype=torch.float64,
+                                                          device=DEV)),
+           lambda: gs.StepRunner(DEV)(dg, X.to(torch.bfloat16), None,
+                                      torch.empty(g.nnz, device=DEV)),
+           lambda: gs.StepRunner(DEV)(dg, X, torch.empty((g.M, K - 8), device=DEV), None),
+           lambda: gs.StepRunner(DEV)(dg, X, None, torch.empty(g.nnz - 1, device=DEV))]
+    for f in bad:
+        with pytest.raises(ValueError):
+            f()

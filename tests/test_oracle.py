@@ -293,11 +293,12 @@ def test_plan_dtp_maximality_bruteforce(nnz, K, alpha, abs_):
 #   the rows fit, 32,768): C = 256 -> 48,496 rows > 32,768; C = 128 -> 24,248 -> 128.
 # Degree 100 (M = 100,000), fp32: C = 512 -> 24,248 > 16,384; C = 256 -> 12,124 -> 256.
 # Degree 500 (M = 20,000): C = 512 -> 4,849 rows -> 512.  L2 off -> 512.
-# L2 = 1 MiB: 256 rows fit; even C = 8 (37,888 nnz -> 757 rows) does not -> 8, which the
-# step-5c chunk floor (on with the cap) raises to 64.
+# L2 = 1 MiB: 256 rows fit; even C = 8 (37,888 nnz -> 757 rows) does not -> 8.  The
+# step-5c chunk floor does NOT raise it: it applies only where InEq. (5) itself chose
+# fewer than 64 (here C_dtp = 512; the cap, not a lack of parallelism, decided).
 @pytest.mark.parametrize("M,dtype,l2,expect", [
     (200_000, 0, 64 << 20, 128), (200_000, 1, 64 << 20, 128), (100_000, 0, 64 << 20, 256),
-    (200_000, 0, 0, 512), (20_000, 0, 64 << 20, 512), (200_000, 0, 1 << 20, 64)])
+    (200_000, 0, 0, 512), (20_000, 0, 64 << 20, 512), (200_000, 0, 1 << 20, 8)])
 def test_plan_locality_cap_worked_examples(M, dtype, l2, expect):
     p = oracle.plan(np.zeros(10_000_000, np.int32), 256, num_sms=148, active_blocks_per_sm=2,
                     feature_dtype=dtype, M=M, l2_bytes=l2)
@@ -308,8 +309,8 @@ def test_plan_locality_cap_worked_examples(M, dtype, l2, expect):
 
 def test_plan_locality_cap_monotone():
     """More L2 never shrinks C*, more rows per nonzero never grows it, the cap never
-    exceeds the DTP choice except through the step-5c floor of 64, and an unbounded L2
-    gives DTP floored at 64 (no L2 model: DTP exactly)."""
+    exceeds the DTP choice, an unbounded L2 gives DTP exactly, and where DTP itself chose
+    8 or 32 the step-5c floor gives 64 whatever the L2 (no L2 model: DTP exactly)."""
     rng = np.random.default_rng(77)
     cands = [8, 32, 64, 128, 256, 512]
     for _ in range(60):
@@ -329,7 +330,10 @@ def test_plan_locality_cap_monotone():
         prev = 0
         for l2 in (1 << 16, 1 << 20, 16 << 20, 64 << 20, 126 << 20, 1 << 40):
             c = chunk(M, l2)["chunk"]
-            assert c in cands and c <= max(base["chunk"], 64) and c >= max(prev, 64)
+            if base["chunk"] < 64:
+                assert c == 64
+            else:
+                assert c in cands and c <= base["chunk"] and c >= prev
             prev = c
         assert prev == max(base["chunk"], 64)
         c_small_m = chunk(max(1, M // 4), 64 << 20)["chunk"]
@@ -410,6 +414,41 @@ def test_shard_edges(nnz, P):
     b = oracle.shard_edges(nnz, P)
     assert b[0] == 0 and b[-1] == nnz and (np.diff(b) >= 0).all()
     assert (np.diff(b) <= -(-nnz // P)).all()
+
+
+# Hand-worked floor(p * nnz / P) bounds (SURVEY §8(c) "Shards"), chosen where
+# floor and ceil (and rounding) give different answers: 10/3 = 3.33 -> 3, 20/3 = 6.67 -> 6
+# (ceil would give [0, 4, 7, 10], rounding [0, 3, 7, 10]); 7 edges over 8 ranks leave
+# rank 0 empty (floor(7/8) = 0) and rank 7 holds one edge (floor(49/8) = 6).
+@pytest.mark.parametrize("nnz,P,expect", [
+    (10, 3, [0, 3, 6, 10]),
+    (7, 8, [0, 0, 1, 2, 3, 4, 5, 6, 7]),
+    (11, 4, [0, 2, 5, 8, 11]),
+    (5, 2, [0, 2, 5]),
+    (1, 3, [0, 0, 0, 1]),
+    (0, 2, [0, 0, 0]),
+])
+def test_shard_edges_hand_worked(nnz, P, expect):
+    assert list(oracle.shard_edges(nnz, P)) == expect
+
+
+def test_shard_edges_no_int64_overflow_at_full_scale():
+    # p * nnz exceeds 2^31 at C4/C5 sizes; the bound must still be the exact floor
+    nnz, P = 126_167_053, 8
+    b = oracle.shard_edges(nnz, P)
+    assert list(b) == [p * nnz // P for p in range(P + 1)]
+    assert b[5] == 78_854_408  # 5 * 126,167,053 / 8 = 78,854,408.125
+
+
+def test_assert_within_rejects_nan_and_inf():
+    from helpers import assert_within
+    ref = np.array([1.0, 2.0]); T = np.array([1.0, 2.0])
+    assert assert_within(np.array([1.0, 2.0]), ref, T) == 0.0
+    for bad in (np.nan, np.inf, -np.inf):
+        with pytest.raises(AssertionError):
+            assert_within(np.array([1.0, bad]), ref, T)
+    with pytest.raises(AssertionError):  # a NaN where sum|terms| == 0 fails too
+        assert_within(np.array([np.nan]), np.array([0.0]), np.array([0.0]))
 
 
 def test_csr_to_coo_matches_repeat():

@@ -20,7 +20,7 @@ import numpy as np, torch
 import gen, oracle
 import paper_conf_ipps_fanwc23_b200 as gs
 from gen import configs
-res = {"lib": os.environ["GNN_LIB_PATH"], "dtype": DTYPE, "force_chunk": FCHUNK}
+res = {"lib": os.environ["GNN_LIB_PATH"], "dtype": DTYPE, "force_chunk": FCHUNK, "wpb": WPB}
 # parity on a small graph
 g = gen.powerlaw_graph(4000, 200000, gamma=2.2, n_comm=5, seed=3)
 dg = gs.DeviceGraph.from_arrays(g.M, g.N, g.row_ind, g.col_ind, g.val, g.row_ptr)
@@ -35,13 +35,24 @@ for K in (32, 64, 128, 256):
     worst = max(worst, float((np.abs(O - r) / np.maximum(T, 1e-300)).max()),
                 float((np.abs(E - r2) / np.maximum(T2, 1e-300)).max()))
 res["parity_worst_err_over_T"] = worst
-g = configs.make_graph(WL)
 perm = None
-if REORDER:
-    perm, comm, q = gs.reorder_gcr(g.row_ptr, g.col_ind)
-    rp, ri, ci, v = gs.permute_graph(g.row_ptr, g.col_ind, g.val, perm)
-    g = gen.Graph(g.M, g.N, rp, ri, ci, v)
-    res["modularity"] = q
+cache = os.environ.get("GNN_SWEEP_CACHE")  # per-session scratch: the graph is deterministic
+cfile = cache and os.path.join(cache, f"{WL}_{int(REORDER)}.npz")
+if cfile and os.path.exists(cfile):
+    z = np.load(cfile)
+    g = gen.Graph(int(z["M"]), int(z["N"]), z["rp"], z["ri"], z["ci"], z["v"])
+    perm = z["perm"] if REORDER else None
+else:
+    g = configs.make_graph(WL)
+    if REORDER:
+        perm, comm, q = gs.reorder_gcr(g.row_ptr, g.col_ind)
+        rp, ri, ci, v = gs.permute_graph(g.row_ptr, g.col_ind, g.val, perm)
+        g = gen.Graph(g.M, g.N, rp, ri, ci, v)
+        res["modularity"] = q
+    if cfile:
+        os.makedirs(cache, exist_ok=True)
+        np.savez(cfile, M=g.M, N=g.N, rp=g.row_ptr, ri=g.row_ind, ci=g.col_ind, v=g.val,
+                 perm=perm if perm is not None else np.zeros(0, np.int32))
 dg = gs.DeviceGraph.from_arrays(g.M, g.N, g.row_ind, g.col_ind, g.val, g.row_ptr)
 flush = torch.empty(64 * 1024 * 1024, device="cuda")
 for K, fvw in ([(k, 0) for k in KS] + [(k, 8) for k in KS if VW8 and k % 8 == 0 and k < 256]
@@ -52,7 +63,7 @@ for K, fvw in ([(k, 0) for k in KS] + [(k, 8) for k in KS if VW8 and k % 8 == 0 
     if DTYPE == "bf16":
         X = X.to(torch.bfloat16)
     O = torch.empty((g.M, K), device="cuda"); E = torch.empty(g.nnz, device="cuda")
-    p = gs.plan(dg, K, force_vw=fvw, feature_dtype=DTYPE, force_chunk=FCHUNK)
+    p = gs.plan(dg, K, force_vw=fvw, feature_dtype=DTYPE, force_chunk=FCHUNK, warps_per_block=WPB)
     ts, td = [], []
     for it in range(REPS + 2):
         flush.fill_(it)
@@ -62,7 +73,7 @@ for K, fvw in ([(k, 0) for k in KS] + [(k, 8) for k in KS if VW8 and k % 8 == 0 
         if it >= 2:
             ts.append(a.elapsed_time(b)); td.append(b.elapsed_time(c))
     res[f"K{K}" + (f"_vw{fvw}" if fvw else "")] = {"spmm_ms": round(min(ts), 4), "sddmm_ms": round(min(td), 4),
-                    "spmm_med": round(sorted(ts)[len(ts)//2], 4), "info": {k: p.info()[k] for k in ("chunk", "active_blocks_per_sm")}}
+                    "spmm_med": round(sorted(ts)[len(ts)//2], 4), "info": {k: p.info()[k] for k in ("chunk", "active_blocks_per_sm", "warps_per_block")}}
 print("RESULT " + json.dumps(res), flush=True)
 '''
 
@@ -78,10 +89,11 @@ def main():
     ap.add_argument("--reorder", action="store_true")
     ap.add_argument("--dtype", default="f32", choices=["f32", "bf16"])
     ap.add_argument("--force-chunk", type=int, default=0)
+    ap.add_argument("--wpb", type=int, default=0, help="plan warps_per_block (0 = default 8)")
     ap.add_argument("libs", nargs="+")
     a = ap.parse_args()
     code = CHILD.replace("ROOT", repr(ROOT)).replace("WL", repr(a.workload)).replace(
-        "KS", repr([int(k) for k in a.K.split(",")])).replace("REPS", str(a.reps)).replace("VW8", str(a.vw8)).replace("REORDER", str(a.reorder)).replace("DTYPE", repr(a.dtype)).replace("FCHUNK", str(a.force_chunk)).replace("ALTVW", str(a.alt_vw))
+        "KS", repr([int(k) for k in a.K.split(",")])).replace("REPS", str(a.reps)).replace("VW8", str(a.vw8)).replace("REORDER", str(a.reorder)).replace("DTYPE", repr(a.dtype)).replace("FCHUNK", str(a.force_chunk)).replace("ALTVW", str(a.alt_vw)).replace("WPB", str(a.wpb))
     for lib in a.libs:
         env = dict(os.environ, GNN_LIB_PATH=os.path.abspath(lib))
         r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
