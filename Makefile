@@ -21,7 +21,7 @@ gen/libgnngen.so: gen/gen.c gen/gen.h
 
 # no fast-math, no FMA contraction: the oracle must round exactly as written
 oracle/liboracle.so: oracle/oracle.c oracle/oracle.h
-	$(HOSTCC) -O2 -ffp-contract=off -fno-fast-math -fPIC -shared -o $@ oracle/oracle.c -lm
+	$(HOSTCC) -O2 -ffp-contract=off -fno-fast-math -fopenmp -fPIC -shared -o $@ oracle/oracle.c -lm
 
 $(OBJDIR)/%.o: $(PKG)/csrc/% $(CUHDR)
 	@mkdir -p $(OBJDIR)

@@ -53,11 +53,18 @@ def _load():
     lib.oracle_csr_to_coo.argtypes = [vp, i64, vp]
     lib.oracle_modularity.argtypes = [vp, vp, i64, vp, i32]
     lib.oracle_modularity.restype = ctypes.c_double
+    lib.oracle_threads.argtypes = [ctypes.c_int]
+    lib.oracle_threads.restype = ctypes.c_int
     for f in ("oracle_spmm", "oracle_spmm_agg", "oracle_sddmm", "oracle_plan", "oracle_shard_rows",
               "oracle_shard_edges", "oracle_csr_to_coo"):
         getattr(lib, f).restype = ctypes.c_int
     _lib = lib
     return lib
+
+
+def threads(n: int = 0) -> int:
+    """Set the oracle's OpenMP thread count (n > 0); returns the count in effect."""
+    return int(_load().oracle_threads(n))
 
 
 def _i32(a):

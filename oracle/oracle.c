@@ -1,7 +1,9 @@
 /*
  * oracle.c -- TEST INFRASTRUCTURE ONLY (see oracle.h).  Plain C, fp64, no
  * blocking / fusion / reordering beyond what the paper's algorithms state.
- * Compiled with -O2 -ffp-contract=off (no FMA contraction, no fast-math).
+ * Compiled with -O2 -ffp-contract=off (no FMA contraction, no fast-math) -fopenmp: SpMM
+ * runs one contiguous range of whole rows per thread, SDDMM splits the nonzeros; neither
+ * changes any sum's order, so results are identical for every thread count.
  */
 #include "oracle.h"
 
@@ -9,16 +11,27 @@
 #include <stddef.h>
 #include <stdlib.h>
 #include <string.h>
+#ifdef _OPENMP
+#include <omp.h>
+#endif
+
+/* Thread count of the OpenMP loops below (timing / determinism tests); 0 = unchanged. */
+int oracle_threads(int n) {
+#ifdef _OPENMP
+  if (n > 0) omp_set_num_threads(n);
+  return omp_get_max_threads();
+#else
+  (void)n;
+  return 1;
+#endif
+}
 
 /* ------------------------------------------------------------ SpMM ------ */
-/* Algorithm 1. */
-int oracle_spmm(int64_t i0, int64_t i1, const int32_t *row_ind, const int32_t *col_ind,
-                const float *val, int64_t K, const float *A, int64_t lda, int64_t r0,
-                int64_t nrows, double *O, double *T) {
-  if (i0 < 0 || i1 < i0 || K < 1 || lda < K || nrows < 0) return -1;
-  memset(O, 0, sizeof(double) * (size_t)(nrows * K));
-  if (T) memset(T, 0, sizeof(double) * (size_t)(nrows * K));
-  for (int64_t i = i0; i < i1; ++i) {                       /* line 1 */
+/* Algorithm 1 over nonzeros [s, e). */
+static int spmm_range(int64_t s, int64_t e, const int32_t *row_ind, const int32_t *col_ind,
+                      const float *val, int64_t K, const float *A, int64_t lda, int64_t r0,
+                      int64_t nrows, double *O, double *T) {
+  for (int64_t i = s; i < e; ++i) {                         /* line 1 */
     int64_t r = row_ind[i], c = col_ind[i];                 /* line 2 */
     double v = val ? (double)val[i] : 1.0;
     if (r < r0 || r >= r0 + nrows || c < 0) return -1;
@@ -31,6 +44,36 @@ int oracle_spmm(int64_t i0, int64_t i1, const int32_t *row_ind, const int32_t *c
     }
   }
   return 0;
+}
+
+/* Algorithm 1 over [i0, i1).  With OpenMP the nonzeros are cut into one contiguous range
+ * per thread, each cut moved forward to the next row start, so every row is summed by one
+ * thread in nonzero order: the result is the serial loop's, bit for bit, for any thread
+ * count (row_ind is non-decreasing). */
+int oracle_spmm(int64_t i0, int64_t i1, const int32_t *row_ind, const int32_t *col_ind,
+                const float *val, int64_t K, const float *A, int64_t lda, int64_t r0,
+                int64_t nrows, double *O, double *T) {
+  if (i0 < 0 || i1 < i0 || K < 1 || lda < K || nrows < 0) return -1;
+  memset(O, 0, sizeof(double) * (size_t)(nrows * K));
+  if (T) memset(T, 0, sizeof(double) * (size_t)(nrows * K));
+  int nt = 1;
+#ifdef _OPENMP
+  nt = omp_get_max_threads();
+  if ((i1 - i0) < 65536) nt = 1;
+#endif
+  int rc = 0;
+#pragma omp parallel num_threads(nt) reduction(| : rc)
+  {
+    int t = 0;
+#ifdef _OPENMP
+    t = omp_get_thread_num();
+#endif
+    int64_t s = i0 + (i1 - i0) * t / nt, e = i0 + (i1 - i0) * (t + 1) / nt;
+    while (s > i0 && s < i1 && row_ind[s] == row_ind[s - 1]) ++s;  /* own whole rows */
+    while (e > i0 && e < i1 && row_ind[e] == row_ind[e - 1]) ++e;
+    if (s < e) rc |= spmm_range(s, e, row_ind, col_ind, val, K, A, lda, r0, nrows, O, T);
+  }
+  return rc ? -1 : 0;
 }
 
 /* ------------------------------------------------ aggregated SpMM ------ */
@@ -130,10 +173,13 @@ int oracle_sddmm(int64_t i0, int64_t i1, const int32_t *row_ind, const int32_t *
                  const float *val, int64_t K, const float *A1, int64_t lda1,
                  const float *A2T, int64_t lda2, double *out, double *T) {
   if (i0 < 0 || i1 < i0 || K < 1 || lda1 < K || lda2 < K) return -1;
+  int rc = 0;
+  /* every output is independent: OpenMP over the nonzeros changes no arithmetic */
+#pragma omp parallel for schedule(static) reduction(| : rc) if (i1 - i0 >= 16384)
   for (int64_t i = i0; i < i1; ++i) {                       /* line 1 */
     int64_t r = row_ind[i], c = col_ind[i];                 /* line 2 */
     double v = val ? (double)val[i] : 1.0;
-    if (r < 0 || c < 0) return -1;
+    if (r < 0 || c < 0) { rc |= 1; continue; }
     const float *a1 = A1 + r * lda1;
     const float *a2 = A2T + c * lda2;                       /* A2[k][c] = A2T[c][k] */
     double acc = 0.0, tabs = 0.0;
@@ -145,7 +191,7 @@ int oracle_sddmm(int64_t i0, int64_t i1, const int32_t *row_ind, const int32_t *
     out[i - i0] = acc * v;                                  /* line 6 */
     if (T) T[i - i0] = fabs(v) * tabs;
   }
-  return 0;
+  return rc ? -1 : 0;
 }
 
 /* ------------------------------------------------------------ plan ------ */

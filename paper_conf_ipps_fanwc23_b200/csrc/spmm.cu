@@ -95,8 +95,25 @@ SpmmFn pick_spmm(int dtype, int vw, int L, int R, int vws, int agg = kAggSum) {
   return pick_spmm_f32(vw, L, R, vws);
 }
 
+#ifndef GNN_SPMM_BF16_R2_WIDEN
+#define GNN_SPMM_BF16_R2_WIDEN 1  // measured: bf16 K=256 SpMM 4.30 -> 3.96 ms (r01_sweep43)
+#endif
+#ifndef GNN_SPMM_F32_R2_WIDEN
+#define GNN_SPMM_F32_R2_WIDEN 1  // measured at 80 registers: C4 K=256 5.94 -> 5.87 ms, C5
+                                 // 8.74 -> 8.61 (r02_s1; at 128 registers C5 lost 16%)
+#endif
+// The lane shape the sum kernel is launched with: rows of two vectors per lane (R = 2)
+// run as one vector per lane on twice the lanes -- half the accumulators per lane, each
+// output element summed in the same order (identical results).
+bool spmm_widen(int dtype, int agg, int lanes, int vecs) {
+  return agg == kAggSum && vecs == 2 && lanes <= 16 &&
+         ((dtype == GNN_BF16 && GNN_SPMM_BF16_R2_WIDEN) ||
+          (dtype == GNN_F32 && GNN_SPMM_F32_R2_WIDEN));
+}
+
 // Cached per (device, dtype, vw, lanes, vecs, wpb): the occupancy API is a host-side
 // query but not free, and plans are rebuilt every step in graph-sampling training (C3).
+// The query is for the kernel the sum launcher actually runs (after the widen remap).
 int spmm_active_blocks_per_sm(int dtype, int vw, int lanes, int vecs, int wpb) {
   static std::atomic<int> cache[64][2][5][6][2][17];
   int dev = 0;
@@ -110,6 +127,10 @@ int spmm_active_blocks_per_sm(int dtype, int vw, int lanes, int vecs, int wpb) {
   std::atomic<int> &slot = cache[dev][dtype][iv][il][vecs - 1][wpb];
   int n = slot.load(std::memory_order_relaxed);
   if (n > 0) return n;
+  if (spmm_widen(dtype, kAggSum, lanes, vecs)) {
+    lanes *= 2;
+    vecs = 1;
+  }
   SpmmFn f = pick_spmm(dtype, vw, lanes, vecs, 1);
   if (!f) return 0;
   // the plan's vw_sparse is not known yet: size the tiles for the widest (4)
@@ -235,19 +256,7 @@ gnn_status_t launch_spmm(const Plan *p, const gnn_graph_t *g, const void *A, int
   if (dtype == GNN_BF16 && in.vecs == 2 && vws > 2) vws = 2;
 #endif
   int lanes = in.lanes, vecs = in.vecs;
-#ifndef GNN_SPMM_BF16_R2_WIDEN
-#define GNN_SPMM_BF16_R2_WIDEN 1  // measured: bf16 K=256 SpMM 4.30 -> 3.96 ms (r01_sweep43)
-#endif
-#ifndef GNN_SPMM_F32_R2_WIDEN
-#define GNN_SPMM_F32_R2_WIDEN 0
-#endif
-  // Rows of two vectors per lane (R = 2) run as one vector per lane on twice the lanes:
-  // half the accumulators per lane (no spill with 2-wide sparse copies), half the
-  // nonzeros in flight per warp; each output element is summed in the same order, so the
-  // results are identical.
-  if (agg == kAggSum && vecs == 2 && lanes <= 16 &&
-      ((dtype == GNN_BF16 && GNN_SPMM_BF16_R2_WIDEN) ||
-       (dtype == GNN_F32 && GNN_SPMM_F32_R2_WIDEN))) {
+  if (spmm_widen(dtype, agg, lanes, vecs)) {
     lanes *= 2;
     vecs = 1;
     vws = effective_vws(in.vw_sparse, g, nullptr);
@@ -255,7 +264,7 @@ gnn_status_t launch_spmm(const Plan *p, const gnn_graph_t *g, const void *A, int
   }
 #if GNN_SPMM_VWS_CLAMP
   {
-    int d = spmm_depth(ES, VW, lanes, vecs) / vecs;
+    int d = spmm_depth(ES, VW, lanes, vecs, agg) / vecs;
     if (d < 1) d = 1;
     while (vws > d) vws >>= 1;
   }

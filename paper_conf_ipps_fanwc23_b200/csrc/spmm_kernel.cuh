@@ -8,45 +8,46 @@
 
 namespace gnn {
 
-// Feature rows in flight per lane (U) and the register budget, per instantiation.
-// Measured on C4 (profiles/r01_sweep4.txt): with 256-bit loads U = 4 is best while
-// several chunks share a warp (L <= 8), U = 8 once a group spans >= 16 lanes.
-// Register budget per thread (the occupancy lever of PAPER.md P:392, "register pressure"
-// at large K): 128 = 2 resident blocks of 8 warps per SM, 80 = 3, 64 = 4.
-#ifndef GNN_SPMM_REGS
-#define GNN_SPMM_REGS 128
-#endif
-#ifndef GNN_SPMM_REGS_BF16
-#define GNN_SPMM_REGS_BF16 GNN_SPMM_REGS
-#endif
-template <typename TF>
-struct SpmmRegs {
-  static constexpr int value = TF::bytes == 2 ? GNN_SPMM_REGS_BF16 : GNN_SPMM_REGS;
-};
-
-// Feature vectors in flight per lane (U * R).  Measured on the GCR-reordered C4
-// (profiles/r01_sweep12.txt, r01_sweep19.txt): 8, except 4 when a lane holds two
-// vectors per row (R = 2) or a row is only 2 lanes wide.
+// Register budget and feature vectors in flight per lane (U * R), per instantiation --
+// the occupancy lever of PAPER.md P:392 ("register pressure" at large K).  Measured on
+// the GCR-reordered C4 and C5 (profiles/r02_s1_sweep_*.txt, 4-warp blocks):
+//   fp32 rows of one 256-bit vector per lane (every K once rows of two vectors run on
+//   twice the lanes, below): 80 registers (3 resident 8-warp blocks / 6 of 4 warps per SM
+//   instead of 2 / 4) with 4 vectors in flight instead of 8: C4 K=32 0.890 -> 0.849 ms,
+//   K=64 1.594 -> 1.510, K=128 2.974 -> 2.942, K=256 5.942 -> 5.871, C5 K=256 8.74 -> 8.61;
+//   bf16 rows of >= 8 lanes: 96 registers, 4 in flight (5 resident 4-warp blocks): C4
+//   K=256 3.91 -> 3.75 ms; everything else (narrow bf16 rows, max / min, two-vector rows
+//   that stay so) keeps 128 registers and the round-1 depths (r01_sweep4 / 12 / 19).
+// GNN_SPMM_REGS / GNN_SPMM_DEPTH8 / GNN_SPMM_DEPTH_R2 override the table (build sweeps).
 #ifndef GNN_SPMM_DEPTH_R2
 #define GNN_SPMM_DEPTH_R2 4
 #endif
-template <typename TF, int VW, int L, int R>
-struct FeatDepth {
+template <typename TF, int VW, int L, int R, int AGG>
+struct SpmmTune {
   static constexpr bool wide = VW * TF::bytes == 32;  // 256-bit vectors
-#if defined(GNN_SPMM_DEPTH8)
-  static constexpr int value = wide ? GNN_SPMM_DEPTH8 : 8;
+  static constexpr bool f32 = TF::bytes == 4;
+  static constexpr bool lean = AGG == 0 && R == 1 && wide && (f32 || L >= 8);
+#if defined(GNN_SPMM_REGS)
+  static constexpr int regs = GNN_SPMM_REGS;
 #else
-  static constexpr int value = R == 2 ? GNN_SPMM_DEPTH_R2 : ((wide && L <= 2) ? 4 : 8);
+  static constexpr int regs = lean ? (f32 ? 80 : 96) : 128;
+#endif
+#if defined(GNN_SPMM_DEPTH8)
+  static constexpr int depth = wide ? GNN_SPMM_DEPTH8 : 8;
+#else
+  static constexpr int depth = R == 2 ? GNN_SPMM_DEPTH_R2 : ((lean || (wide && L <= 2)) ? 4 : 8);
 #endif
 };
 
-// host mirror of FeatDepth (feature vectors in flight per lane) for the launcher
-inline int spmm_depth(int es, int vw, int L, int R) {
+// host mirror of SpmmTune::depth (feature vectors in flight per lane) for the launcher
+inline int spmm_depth(int es, int vw, int L, int R, int agg) {
   const bool wide = vw * es == 32;
+  const bool lean = agg == 0 && R == 1 && wide && (es == 4 || L >= 8);
 #if defined(GNN_SPMM_DEPTH8)
+  (void)lean;
   return wide ? GNN_SPMM_DEPTH8 : 8;
 #else
-  return R == 2 ? GNN_SPMM_DEPTH_R2 : ((wide && L <= 2) ? 4 : 8);
+  return R == 2 ? GNN_SPMM_DEPTH_R2 : ((lean || (wide && L <= 2)) ? 4 : 8);
 #endif
 }
 #ifndef GNN_SPMM_VWS_CLAMP
@@ -119,7 +120,7 @@ __device__ __forceinline__ void accumulate(float (&acc)[VW], float s, const Feat
 // L lanes per (chunk, K-slice) work item, R VW-wide vectors per lane (plan rule step 2).
 // TF: feature element type (F32 or BF16); accumulation and O are fp32.
 template <typename TF, int VW, int L, int R, int VWS, int AGG>
-__global__ void __maxnreg__(SpmmRegs<TF>::value)
+__global__ void __maxnreg__((SpmmTune<TF, VW, L, R, AGG>::regs))
     spmm_kernel(const SparseArgs a, const void *__restrict__ A, const int64_t lda,
                 float *__restrict__ O, const int64_t ldo) {
   constexpr int ES = TF::bytes;
@@ -128,7 +129,7 @@ __global__ void __maxnreg__(SpmmRegs<TF>::value)
   using Tiles = TilesFor<L, VWS>;
   constexpr int T = Tiles::T;  // nonzeros per tile per group
   // U nonzeros per batch: FeatDepth vectors in flight per lane, whole sparse vectors
-  constexpr int D = FeatDepth<TF, VW, L, R>::value / R;
+  constexpr int D = SpmmTune<TF, VW, L, R, AGG>::depth / R;
   constexpr int U = D > T ? T : (D < VWS ? VWS : D);
   static_assert(T % U == 0 && U % VWS == 0, "tile / prefetch shape");
   const int lane = threadIdx.x & 31;

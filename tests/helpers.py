@@ -78,7 +78,11 @@ def kernel_resources(lib_path):
 def expected_active_blocks(lib_path, dtype, vw, lanes, vecs, wpb):
     """Resident blocks/SM of spmm_kernel<dtype, vw, lanes, vecs, 1, sum> at wpb warps per
     block with the plan's tile smem (sized for 4-wide sparse vectors: 2 stages x 3 arrays
-    x (32 / lanes) groups x (4 * lanes + 4) words per warp)."""
+    x (32 / lanes) groups x (4 * lanes + 4) words per warp).  Rows of two
+    vectors per lane on <= 16 lanes are launched as one vector per lane on twice the
+    lanes ("widen"), so that is the kernel whose occupancy counts."""
+    if vecs == 2 and lanes <= 16:
+        lanes, vecs = 2 * lanes, 1
     regs, static_smem = kernel_resources(lib_path)[("spmm", dtype, vw, lanes, vecs, 1, 0)]
     S = B200_SM
     per_warp_regs = -(-regs * 32 // S["reg_unit"]) * S["reg_unit"]
@@ -116,7 +120,7 @@ def oracle_plan_checked(p, g, K, **kw):
     assert (info["num_sms"], info["active_blocks_per_sm"], info["l2_bytes"]) == (nsm, abs_, l2)
     dt = kw.get("feature_dtype", 0)
     ref = oracle.plan(g.row_ind, K, nsm, abs_, alpha=kw.get("alpha", 2) or 2,
-                      warps_per_block=kw.get("warps_per_block", 8) or 8,
+                      warps_per_block=kw.get("warps_per_block") or 4,  # library default
                       force_chunk=kw.get("force_chunk", 0), force_vw=kw.get("force_vw", 0),
                       feature_dtype=1 if dt in (1, "bf16") else 0, M=g.M, l2_bytes=l2)
     assert info == ref.info, (info, ref.info)

@@ -95,7 +95,7 @@ def test_forced_vector_width(vw):
     run_full(g, 64, force_vw=vw)
 
 
-@pytest.mark.parametrize("wpb,alpha", [(1, 1), (4, 2), (16, 8)])
+@pytest.mark.parametrize("wpb,alpha", [(1, 1), (8, 2), (16, 8)])
 def test_block_shape_and_alpha(wpb, alpha):
     g = gen.powerlaw_graph(5000, 200000, seed=300 + wpb)
     run_full(g, 64, warps_per_block=wpb, alpha=alpha)

@@ -576,3 +576,27 @@ def test_extremum_backward_ties_go_to_the_first_term():
     # min: col 0 -> nonzero 0 (value 1); col 1 -> nonzero 2 (value -1)
     np.testing.assert_array_equal(dA, [[10.0 + 30.0, 40.0], [0.0, 0.0], [0.0, 20.0]])
     np.testing.assert_array_equal(dval, [10.0, 0.0, -20.0, 30.0])
+
+
+def test_parallel_oracle_is_bitwise_serial():
+    """OpenMP changes no sum's order: SpMM (whole rows per thread, cuts moved to row
+    starts, incl. a hub row longer than a thread's share) and SDDMM give identical bits
+    with 1 and with many threads."""
+    g = gen.powerlaw_graph(3000, 200_000, gamma=2.1, n_comm=5, seed=91)
+    ri = g.row_ind.copy()
+    ri[: g.nnz // 3] = 0  # a hub spanning several threads' ranges
+    ri.sort()
+    X = gen.features(92, g.N, 24)
+    nmax = oracle.threads()
+    try:
+        res = []
+        for n in (1, 3, max(4, nmax)):
+            oracle.threads(n)
+            O, T = oracle.spmm(ri, g.col_ind, g.val, X, M=g.M)
+            E, T2 = oracle.sddmm(ri, g.col_ind, g.val, X, X)
+            res.append((O, T, E, T2))
+        for r in res[1:]:
+            for a, b in zip(res[0], r):
+                assert np.array_equal(a, b)
+    finally:
+        oracle.threads(nmax)
