@@ -9,6 +9,7 @@ PKG     := paper_conf_ipps_fanwc23_b200
 ARCH    := -gencode arch=compute_100a,code=sm_100a
 NVFLAGS := -ccbin /usr/bin/g++ $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC \
            -Xcompiler -fvisibility=hidden -Iinclude --expt-relaxed-constexpr -Xptxas -v
+GITSHA  := $(shell git -C $(CURDIR) rev-parse --short=12 HEAD 2>/dev/null || echo unknown)$(shell git -C $(CURDIR) diff --quiet HEAD -- $(PKG)/csrc include 2>/dev/null || echo +dirty)
 CUSRC   := $(wildcard $(PKG)/csrc/*.cu) $(wildcard $(PKG)/csrc/*.cpp)
 CUHDR   := $(wildcard $(PKG)/csrc/*.cuh) include/gnn_sparse.h
 OBJDIR  := $(if $(TAG),/tmp/gnn_obj_$(TAG),build/obj)
@@ -26,6 +27,11 @@ oracle/liboracle.so: oracle/oracle.c oracle/oracle.h
 $(OBJDIR)/%.o: $(PKG)/csrc/% $(CUHDR)
 	@mkdir -p $(OBJDIR)
 	$(NVCC) $(NVFLAGS) $(DEFS) -c -o $@ $< 2> $@.ptxas.log || (cat $@.ptxas.log; exit 1)
+
+# the version string carries the commit; rebuilt whenever HEAD moves
+$(OBJDIR)/util.cu.o: $(PKG)/csrc/util.cu $(CUHDR) .git/HEAD $(wildcard .git/refs/heads/*)
+	@mkdir -p $(OBJDIR)
+	$(NVCC) $(NVFLAGS) $(DEFS) -DGNN_GIT_SHA='"$(GITSHA)"' -c -o $@ $< 2> $@.ptxas.log || (cat $@.ptxas.log; exit 1)
 
 $(PKG)/libgnnsparse.so: $(OBJS)
 	$(NVCC) $(ARCH) -shared -cudart static -o $@ $(OBJS)

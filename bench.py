@@ -97,29 +97,39 @@ def load_peaks():
     return 6650.0, "fallback (B200_PROFILING.md)"
 
 
-def probe_own_stream(X, idx, K, reps=3):
+def probe_own_stream(X, idx, K, chunk=0, reps=3):
     """The gather ceiling of a kernel (SURVEY §8(d) peak #2): gnn_probe_gather -- the
     same 256-bit row loads as the kernels, no arithmetic, no stores -- over THIS
     workload's own column-index stream and feature matrix, so its L2 hits and misses are
-    the workload's.  GB/s counted as (4K gathered + 4 index) bytes per entry; median of
+    the workload's.  Two traversals are timed: grid-stride (gnn_probe_gather) and the
+    kernels' chunk order at chunk size `chunk` (gnn_probe_gather_chunked); the faster is
+    the ceiling.  GB/s counted as (4K gathered + 4 index) bytes per entry; median of
     `reps` timed runs after one warm-up.  None if the probe does not cover K / dtype."""
     import torch
     import paper_conf_ipps_fanwc23_b200 as gs
     if K not in (32, 64, 128, 256) or X.dtype != torch.float32 or idx.numel() == 0:
         return None
     sink = torch.zeros(1, device=X.device)
-    ts = []
-    for it in range(reps + 1):
-        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        a.record()
-        gs.probe_gather(X, idx, sink)
-        b.record()
-        torch.cuda.synchronize()
-        if it:
-            ts.append(a.elapsed_time(b))
-    ms = statistics.median(ts)
-    return {"GBps": round(idx.numel() * (4 * K + 4) / ms / 1e6, 1), "ms": round(ms, 4),
-            "entries": int(idx.numel())}
+    out = {"entries": int(idx.numel())}
+    for tag, ch in (("grid_stride", 0), ("chunked", chunk)):
+        if tag == "chunked" and not chunk:
+            continue
+        ts = []
+        for it in range(reps + 1):
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record()
+            gs.probe_gather(X, idx, sink, chunk=ch)
+            b.record()
+            torch.cuda.synchronize()
+            if it:
+                ts.append(a.elapsed_time(b))
+        ms = statistics.median(ts)
+        out[tag] = {"GBps": round(idx.numel() * (4 * K + 4) / ms / 1e6, 1), "ms": round(ms, 4)}
+    best = max((v for k, v in out.items() if isinstance(v, dict)), key=lambda v: v["GBps"])
+    out["GBps"] = best["GBps"]
+    if chunk:
+        out["chunk"] = chunk
+    return out
 
 
 def load_ncu_traffic():
@@ -443,7 +453,7 @@ def roofline_for(name, reorder, r, Ks, world, args, dtype="f32"):
     achieved = dbytes / (dms * 1e-3) / 1e9
     gsh = g_sp if dkind == "spmm" else g_sd
     X = r["X"][dK]
-    probe = probe_own_stream(X, gsh.col_ind, dK)
+    probe = probe_own_stream(X, gsh.col_ind, dK, chunk=r["detail"][f"K{dK}"]["chunk"])
     hbm, hbm_src = load_peaks()
     step_ms = float(sum(r["step_ms"])) / args.steps
     tkey = f"{name}{'+gcr' if reorder else ''}:{dkind}:K{dK}"
@@ -458,9 +468,10 @@ def roofline_for(name, reorder, r, Ks, world, args, dtype="f32"):
                               "dram__bytes_write.sum of one committed `ncu --set full` capture "
                               "(cold cache), not measured in this run") if traffic else None,
            "kernel": f"{dkind} K={dK} ({name}{', GCR-reordered' if reorder else ''}, {dtype})",
-           "peak_source": ("gnn_probe_gather over this workload's own col_ind stream and X "
-                           "(same 256-bit row loads, no arithmetic; measured in this run, "
-                           "(4K + 4) B per entry)"),
+           "peak_source": ("pure-gather probe over this workload's own col_ind stream and X "
+                           "(same 256-bit row loads, no arithmetic, no stores; the faster of a "
+                           "grid-stride and the kernels' chunk-order traversal; measured in "
+                           "this run, (4K + 4) B per entry)"),
            "probe": probe,
            "algorithmic_bytes_per_launch": int(dbytes),
            "byte_model": "per nnz 12 B sparse (+4 B out for SDDMM) + eb*K B gathered feature "
@@ -780,7 +791,7 @@ def c3_block(args, dev, world, rank):
     Xcat = torch.cat([X for (_, _, X, _, _) in subs])
     offs = np.cumsum([0] + [g.N for (g, _, _, _, _) in subs[:-1]])
     idx = torch.cat([dg.col_ind + int(o) for (_, dg, _, _, _), o in zip(subs, offs)])
-    probe = probe_own_stream(Xcat, idx, K)
+    probe = probe_own_stream(Xcat, idx, K, chunk=64)
     del Xcat, idx
     per_sub_bytes = nbytes / nsteps
     step_ms_mean = tot_ms / nsteps

@@ -16,7 +16,10 @@
  *   - Dense matrices are row-major fp32 with a leading dimension (pitch, in
  *     elements) >= K ("row-major ... FP32").
  *   - The caller owns every buffer (graph arrays, features, outputs and the plan
- *     workspace); the library never allocates device memory.
+ *     workspace); the library never allocates device memory, except gnn_validate (an
+ *     8-byte stream-ordered result flag, freed before it returns).
+ *   - GNN_VALIDATE=1 in the environment makes gnn_plan_create (and everything built on
+ *     it) run gnn_validate on the graph first -- a debug switch that synchronises.
  *   - Every call is asynchronous on the given stream (a cudaStream_t; NULL = the
  *     legacy default stream) and never synchronises the host, except
  *     gnn_validate().  Launch errors are returned as GNN_ERR_CUDA; faults inside a
@@ -320,14 +323,18 @@ GNN_API gnn_status_t gnn_run_host_multi(const gnn_graph_t *graph_host, int32_t u
                                         void *workspace, size_t ws_bytes, gnn_stream_t stream);
 
 /* One message-passing step on DEVICE data in one call (BJ configs[2]: a new sampled
- * subgraph every step, re-planned every step): gnn_plan_create into `workspace`
- * (gnn_plan_workspace_bytes bytes; host DTP + plan kernel, no sync), then O = S X
- * (gnn_spmm, if O) and out[i] = val[i] <X[row_i], X[col_i]> (gnn_sddmm with A1 = the
- * graph's rows of X, i.e. X + row_base * ldx, A2T = X, if out).  The SDDMM runs on a
- * per-thread side stream forked from `stream` after the plan and joined back, so the two
- * kernels overlap; `stream` is ordered after both.  The plan handle is internal and
- * released before return (its arrays stay in `workspace`).  fp32; same alignment and
- * error rules as gnn_spmm / gnn_sddmm.  Device pointers. */
+ * subgraph every step, re-planned every step): the host half of gnn_plan_create (DTP:
+ * C* and the launch shape, no sync), then O = S X (gnn_spmm, if O) and
+ * out[i] = val[i] <X[row_i], X[col_i]> (gnn_sddmm with A1 = the graph's rows of X, i.e.
+ * X + row_base * ldx, A2T = X, if out).  The per-chunk boundary table the plan kernel
+ * would write (row_first / row_last / flags, Algo 3 lines 2-3) is recomputed
+ * from row_ind inside the kernels instead, so no plan kernel runs and `workspace`'s
+ * plan arrays are NOT written (deterministic plans excepted: they run the plan kernel
+ * for their fix-up pass).  The SDDMM runs on a per-thread side stream forked from
+ * `stream` and joined back, so the two kernels overlap; the SpMM is a programmatic
+ * dependent launch of its split-row pre-zero.  `stream` is ordered after both.
+ * workspace: gnn_plan_workspace_bytes bytes.  fp32; same alignment and error rules as
+ * gnn_spmm / gnn_sddmm.  Device pointers. */
 GNN_API gnn_status_t gnn_plan_spmm_sddmm(const gnn_graph_t *graph, int32_t K,
                                          const gnn_plan_opts_t *opts, const float *X,
                                          int64_t ldx, float *O, int64_t ldo, float *out,
@@ -342,6 +349,14 @@ GNN_API gnn_status_t gnn_plan_spmm_sddmm(const gnn_graph_t *graph, int32_t K,
  * K in {32, 64, 128, 256}; X 32-byte aligned with ld % 8 == 0; idx in [0, rows). */
 GNN_API gnn_status_t gnn_probe_gather(const float *X, int64_t ld, const int32_t *idx, int64_t n,
                                       int32_t K, float *sink, gnn_stream_t stream);
+/* The same pure gather in the kernels' traversal order: one lane group (K/8 lanes, 8 fp32
+ * per lane) per `chunk` consecutive entries of idx, one group per chunk over the whole
+ * grid of 4-warp blocks (as gnn_spmm / gnn_sddmm launch a plan of chunk size C*), so the
+ * rows in flight -- and the L2 hit rate on a workload's own index stream -- are the
+ * kernels'.  Same argument rules as gnn_probe_gather; chunk >= 1. */
+GNN_API gnn_status_t gnn_probe_gather_chunked(const float *X, int64_t ld, const int32_t *idx,
+                                              int64_t n, int32_t K, int32_t chunk, float *sink,
+                                              gnn_stream_t stream);
 
 /* Split a (row-shard) hybrid CSR/COO by the owner of each column, for overlapping the
  * X all-gather with SpMM: column c belongs to block c / blk, P blocks.

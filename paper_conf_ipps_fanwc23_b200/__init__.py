@@ -74,7 +74,7 @@ EXPORTS = ["gnn_plan_workspace_bytes", "gnn_plan_create", "gnn_plan_info", "gnn_
            "gnn_transpose",
            "gnn_shard_rows", "gnn_shard_edges", "gnn_split_col_blocks",
            "gnn_reorder_gcr", "gnn_permute_graph", "gnn_permute_rows",
-           "gnn_probe_gather", "gnn_run_host_workspace_bytes", "gnn_run_host",
+           "gnn_probe_gather", "gnn_probe_gather_chunked", "gnn_run_host_workspace_bytes", "gnn_run_host",
            "gnn_run_host_multi_workspace_bytes", "gnn_run_host_multi", "gnn_csr_to_coo", "gnn_validate", "gnn_last_error",
            "gnn_version"]
 
@@ -132,6 +132,8 @@ def lib():
     L.gnn_permute_graph.argtypes = [vp, vp, vp, i64, vp, vp, vp, vp, vp]
     L.gnn_permute_rows.argtypes = [vp, i64, i64, i64, vp, vp, i64, vp]
     L.gnn_probe_gather.argtypes = [vp, i64, vp, i64, i32, vp, vp]
+    if hasattr(L, "gnn_probe_gather_chunked"):
+        L.gnn_probe_gather_chunked.argtypes = [vp, i64, vp, i64, i32, i32, vp, vp]
     L.gnn_validate.argtypes = [P(_Graph), vp]
     L.gnn_last_error.argtypes = []
     L.gnn_last_error.restype = ctypes.c_char_p
@@ -140,6 +142,7 @@ def lib():
     for f in ("gnn_plan_create", "gnn_plan_info", "gnn_plan_arrays", "gnn_spmm", "gnn_sddmm",
               "gnn_shard_rows", "gnn_shard_edges", "gnn_csr_to_coo", "gnn_validate",
               "gnn_reorder_gcr", "gnn_permute_graph", "gnn_permute_rows", "gnn_probe_gather",
+              "gnn_probe_gather_chunked",
               "gnn_spmm_bf16", "gnn_sddmm_bf16", "gnn_spmm_ex", "gnn_transpose",
               "gnn_split_col_blocks", "gnn_run_host", "gnn_run_host_multi"):
         if hasattr(L, f):
@@ -533,10 +536,18 @@ def permute_rows(X: torch.Tensor, perm: torch.Tensor, out: torch.Tensor | None =
 
 
 def probe_gather(X: torch.Tensor, idx: torch.Tensor, sink: torch.Tensor | None = None,
-                 stream=None) -> None:
-    """gnn_probe_gather: pure row gather X[idx] (measurement utility)."""
+                 stream=None, chunk: int = 0) -> None:
+    """gnn_probe_gather: pure row gather X[idx] (measurement utility); chunk > 0 selects
+    gnn_probe_gather_chunked (the kernels' traversal: one lane group per chunk)."""
     if sink is None:
         sink = torch.zeros(1, device=X.device)
+    _dense(X, "X", rows=1)
+    if idx.dtype != torch.int32 or not idx.is_contiguous() or idx.device != X.device:
+        raise ValueError("idx must be a contiguous int32 tensor on X's device")
+    if chunk:
+        _check(lib().gnn_probe_gather_chunked(_ptr(X), X.stride(0), _ptr(idx), idx.numel(),
+                                              X.shape[1], chunk, _ptr(sink), _stream(stream)))
+        return
     _check(lib().gnn_probe_gather(_ptr(X), X.stride(0), _ptr(idx), idx.numel(), X.shape[1],
                                   _ptr(sink), _stream(stream)))
 

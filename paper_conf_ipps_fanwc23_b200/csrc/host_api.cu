@@ -394,10 +394,12 @@ GNN_API gnn_status_t gnn_run_host(const gnn_graph_t *gh, int32_t upload_graph, c
 
 // ----------------------------------------------------------------------------------
 // One message-passing step on device-resident data in ONE call (BJ configs[2]: a new
-// sampled subgraph every step, re-planned every step): plan (host DTP + plan kernel) ->
-// SpMM and SDDMM.  The SDDMM runs on a per-thread, per-device side stream forked from
-// `stream` after the plan and joined back before return, so the two kernels' tails
-// overlap on graphs that fill only a few waves; no allocation, no host sync.
+// sampled subgraph every step, re-planned every step): host DTP, then SpMM and SDDMM with
+// the per-chunk boundary table recomputed inside the kernels (no plan kernel).  The SDDMM
+// runs on a per-thread, per-device side stream forked from `stream` and joined back
+// before return, so the two kernels overlap on graphs that fill only a few waves; the
+// SpMM overlaps its pre-zero through a programmatic dependent launch.  No allocation, no
+// host sync.
 namespace gnn {
 namespace {
 struct SideStream {
@@ -441,14 +443,23 @@ GNN_API gnn_status_t gnn_plan_spmm_sddmm(const gnn_graph_t *g, int32_t K,
     return fail(GNN_ERR_INVALID_ARG, "gnn_plan_spmm_sddmm: NULL graph / no output");
   if (opts && opts->feature_dtype != GNN_F32)
     return fail(GNN_ERR_UNSUPPORTED, "gnn_plan_spmm_sddmm: fp32 features only");
+  // Host DTP only: no plan kernel.  The kernels derive each chunk's boundary rows and flags
+  // from row_ind themselves (the plan kernel's arithmetic), so the SDDMM -- which
+  // never needs them -- starts at once on the side stream, and the SpMM is launched as a
+  // programmatic dependent of the split-row pre-zero.  Deterministic plans keep the plan
+  // kernel (their fix-up pass reads the arrays).
+  // GNN_STEP_PLAN_KERNEL=1 restores the plan-kernel path (A/B measurements)
+  const char *pk = getenv("GNN_STEP_PLAN_KERNEL");
+  const bool det = (opts && opts->deterministic) || (pk && pk[0] == '1');
   gnn_plan_t plan = nullptr;
-  if (gnn_status_t st = gnn_plan_create(g, K, opts, workspace, ws_bytes, stream, &plan))
+  if (gnn_status_t st = plan_create(g, K, opts, workspace, ws_bytes, stream, &plan, det))
     return st;
   struct Guard {
     gnn_plan_t p;
     ~Guard() { gnn_plan_destroy(p); }
   } guard{plan};
-  const Plan *p = reinterpret_cast<const Plan *>(plan);
+  Plan *p = reinterpret_cast<Plan *>(plan);
+  p->inline_plan = !det;
   cudaStream_t s = (cudaStream_t)stream;
   SideStream *side = nullptr;
   const bool fork = O && out && g->nnz > 0;

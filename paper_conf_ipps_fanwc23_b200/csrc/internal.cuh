@@ -32,6 +32,7 @@ struct Plan {
   float *carry;  // deterministic plans: [num_chunks][2][K] split-row partials, else null
   int64_t M;
   int64_t row_base;
+  bool inline_plan = false;  // kernels recompute the boundary table (gnn_plan_spmm_sddmm)
 };
 
 // Kernel parameter block shared by the SpMM / SDDMM launchers.
@@ -54,7 +55,33 @@ struct SparseArgs {
   float *carry;   // deterministic: split-row partials [chunk][first|last][K] (no atomics)
   int64_t c_begin, c_end;  // chunk range of this launch (default [0, num_chunks)); the
                            // pipelined host path launches a plan piece by piece
+  int32_t inline_plan;     // 1: no plan arrays -- each chunk derives its boundary rows and
+                           // flags from row_ind (the plan kernel's arithmetic) itself
 };
+
+#ifdef __CUDACC__
+// Boundary rows and continuation flags of chunk c (Algo 3 lines 2-3): from the
+// plan arrays, or -- inline plans -- recomputed from row_ind exactly as plan_kernel does.
+__device__ __forceinline__ void chunk_rows(const SparseArgs &a, int64_t c, int32_t &rf,
+                                           int32_t &rl, uint32_t &fl) {
+  if (a.inline_plan) {
+    const int64_t s = c * a.chunk;
+    const int64_t e = s + a.chunk < a.nnz ? s + a.chunk : a.nnz;
+    rf = __ldg(a.row_ind + s);
+    rl = __ldg(a.row_ind + e - 1);
+    fl = (s > 0 && __ldg(a.row_ind + s - 1) == rf ? 1u : 0u) |
+         (e < a.nnz && __ldg(a.row_ind + e) == rl ? 2u : 0u);
+  } else {
+    rf = a.row_first[c];
+    rl = a.row_last[c];
+    fl = a.flags[c];
+  }
+}
+// last row of chunk c - 1 (c > 0)
+__device__ __forceinline__ int32_t prev_chunk_last_row(const SparseArgs &a, int64_t c) {
+  return a.inline_plan ? __ldg(a.row_ind + c * a.chunk - 1) : a.row_last[c - 1];
+}
+#endif
 
 // Occupancy (active blocks / SM) of the SpMM kernel for a feature width/lane count;
 // DTP's ActiveblocksPerSM (Eq. 3) -- defined in spmm.cu.

@@ -4,6 +4,7 @@
 // and last row and whether those rows continue into the neighbouring chunks (the
 // node boundaries the hybrid-parallel kernels must respect).
 #include <cuda_runtime.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <new>
@@ -180,6 +181,11 @@ gnn_status_t plan_create(const gnn_graph_t *g, int32_t K, const gnn_plan_opts_t 
     return fail(GNN_ERR_INVALID_ARG, "gnn_plan_create: bad graph descriptor");
   gnn_plan_info_t info;
   if (gnn_status_t st = make_info(g->M, g->nnz, K, opts, &info)) return st;
+  // GNN_VALIDATE=1: check the graph's contents (sortedness, index ranges) before planning
+  // -- a debug switch: gnn_validate synchronises the stream
+  const char *v = getenv("GNN_VALIDATE");
+  if (v && v[0] == '1' && g->nnz > 0)
+    if (gnn_status_t st = gnn_validate(g, stream)) return st;
   const int64_t nch = info.num_chunks;
   const int32_t det = opts ? opts->deterministic : 0;
   const size_t need = ws_bytes_for(nch, K, det);

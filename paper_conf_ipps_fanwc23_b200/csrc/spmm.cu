@@ -33,12 +33,15 @@ namespace gnn {
 template <int VW>
 __global__ void spmm_prezero_kernel(const SparseArgs a, float *__restrict__ O,
                                     const int64_t ldo, const float init) {
+  // let a programmatic dependent (the SpMM of gnn_plan_spmm_sddmm) launch right away
+  asm volatile("griddepcontrol.launch_dependents;");
   const int64_t c = a.c_begin + (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5);
   const int lane = threadIdx.x & 31;
   if (c >= a.c_end) return;
-  const uint32_t fl = a.flags[c];
+  int32_t rf, rl;
+  uint32_t fl;
+  chunk_rows(a, c, rf, rl, fl);
   if (!(fl & 2u)) return;
-  const int32_t rf = a.row_first[c], rl = a.row_last[c];
   if ((fl & 1u) && rf == rl) return;
   float *o = O + ((int64_t)rl - a.row_base) * ldo;
   float z[VW];
@@ -199,6 +202,7 @@ SparseArgs make_args(const Plan *p, const gnn_graph_t *g) {
   a.carry = nullptr;
   a.c_begin = 0;
   a.c_end = a.num_chunks;
+  a.inline_plan = p->inline_plan ? 1 : 0;
   return a;
 }
 
@@ -303,7 +307,24 @@ gnn_status_t launch_spmm(const Plan *p, const gnn_graph_t *g, const void *A, int
   }
   const int64_t per_block = (int64_t)(32 / lanes) * in.warps_per_block;  // items / block
   const int64_t grid = (nch * in.slices + per_block - 1) / per_block;
-  f<<<(unsigned)grid, threads, smem, s>>>(a, A, lda, O, ldo);
+  if (p->inline_plan) {
+    // programmatic dependent launch: the SpMM starts while the pre-zero drains and waits
+    // for it only before its first atomic flush (spmm_kernel, griddepcontrol.wait)
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)grid);
+    cfg.blockDim = dim3(threads);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, f, a, A, lda, O, ldo);
+    if (e != cudaSuccess) return cuda_fail(e, "gnn_spmm launch (PDL)");
+  } else {
+    f<<<(unsigned)grid, threads, smem, s>>>(a, A, lda, O, ldo);
+  }
   if (a.carry) {
     const int64_t blocks = (a.num_chunks * 32 + 255) / 256;
     if (agg == kAggMax) spmm_fixup_kernel<1><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo);

@@ -155,11 +155,7 @@ __global__ void __maxnreg__((SpmmTune<TF, VW, L, R, AGG>::regs))
   const int n = item_ok ? (int)(min(cs + (int64_t)a.chunk, a.nnz) - cs) : 0;  // nnz here
   int32_t rf = 0, rl = 0;
   uint32_t fl = 0;
-  if (item_ok) {
-    rf = a.row_first[c];
-    rl = a.row_last[c];
-    fl = a.flags[c];
-  }
+  if (item_ok) chunk_rows(a, c, rf, rl, fl);
   // feature row c of A starts at Ab + c * ldaB (IMAD.WIDE.U32 per gather)
   const char *__restrict__ Ab = reinterpret_cast<const char *>(A) + (int64_t)k0 * ES;
   const uint32_t ldaB = (uint32_t)lda * (uint32_t)ES;
@@ -172,7 +168,15 @@ __global__ void __maxnreg__((SpmmTune<TF, VW, L, R, AGG>::regs))
       if (col_ok[r]) st_zero<VW>(Ok + (row - a.row_base) * ldo + r * Lg * VW);
   };
   float acc[R][VW];
+  // Launched as a programmatic dependent of the pre-zero kernel (gnn_plan_spmm_sddmm):
+  // everything up to the first flush of a row shared with another chunk overlaps the
+  // pre-zero; that flush waits for it (griddepcontrol.wait is a no-op otherwise).
+  bool pdl_waited = false;
   auto flush = [&](int32_t row) {
+    if (!pdl_waited && ((row == rf && (fl & 1u)) || (row == rl && (fl & 2u)))) {
+      asm volatile("griddepcontrol.wait;" ::: "memory");
+      pdl_waited = true;
+    }
     if (a.carry) {  // deterministic plan: split rows go to this chunk's partial slots
       const bool shared = (row == rf && (fl & 1u)) || (row == rl && (fl & 2u));
       if (shared) {
@@ -192,7 +196,7 @@ __global__ void __maxnreg__((SpmmTune<TF, VW, L, R, AGG>::regs))
 
   // empty rows between the previous chunk's last row and ours are ours to zero
   if (item_ok) {
-    const int64_t prev = (c == 0) ? a.row_base - 1 : (int64_t)a.row_last[c - 1];
+    const int64_t prev = (c == 0) ? a.row_base - 1 : (int64_t)prev_chunk_last_row(a, c);
     for (int64_t r = prev + 1; r < rf; ++r) zero_row(r);
   }
 

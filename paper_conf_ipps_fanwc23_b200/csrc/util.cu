@@ -109,7 +109,12 @@ extern "C" {
 
 GNN_API const char *gnn_last_error(void) { return g_err; }
 
-GNN_API const char *gnn_version(void) { return "gnnsparse 0.1 (sm_100a)"; }
+#ifndef GNN_GIT_SHA
+#define GNN_GIT_SHA "unknown"
+#endif
+// the commit the library was built from (Makefile: git rev-parse; "+dirty" for a tree with
+// uncommitted changes) -- the GPU box's snapshot has no .git, bench.py reports this
+GNN_API const char *gnn_version(void) { return "gnnsparse 0.2 (sm_100a) git " GNN_GIT_SHA; }
 
 GNN_API gnn_status_t gnn_shard_rows(const int32_t *row_ptr_host, int64_t M, int32_t P,
                                     int64_t *bounds) {

@@ -85,8 +85,10 @@ def expected_active_blocks(lib_path, dtype, vw, lanes, vecs, wpb):
         lanes, vecs = 2 * lanes, 1
     regs, static_smem = kernel_resources(lib_path)[("spmm", dtype, vw, lanes, vecs, 1, 0)]
     S = B200_SM
+    # the register file is split over the SM's 4 sub-partitions; a warp's registers
+    # (allocated in 256-register units) come from one of them
     per_warp_regs = -(-regs * 32 // S["reg_unit"]) * S["reg_unit"]
-    by_regs = (S["regs"] // per_warp_regs) // wpb
+    by_regs = (4 * ((S["regs"] // 4) // per_warp_regs)) // wpb
     dyn = wpb * 2 * 3 * (32 // lanes) * (4 * lanes + 4) * 4
     by_smem = S["smem"] // (dyn + static_smem)
     by_threads = S["threads"] // (32 * wpb)

@@ -888,3 +888,45 @@ def test_binding_rejects_undersized_or_mistyped_operands():
     for f in bad:
         with pytest.raises(ValueError):
             f()
+
+
+def test_validate_env_switch(monkeypatch):
+    """GNN_VALIDATE=1 makes gnn_plan_create check the graph first (a decreasing row_ind
+    is reported as GNN_ERR_INPUT_CHECK); unset, the same call plans without a check."""
+    g = configs.make_graph("C1")
+    ri = g.row_ind.copy()
+    ri[10], ri[11] = ri[11] + 1, ri[10]  # not non-decreasing
+    dg = gs.DeviceGraph.from_arrays(g.M, g.N, ri, g.col_ind, g.val, None, device=DEV)
+    monkeypatch.setenv("GNN_VALIDATE", "1")
+    with pytest.raises(gs.GnnError) as e:
+        gs.plan(dg, 32)
+    assert e.value.status == 5
+    monkeypatch.delenv("GNN_VALIDATE")
+    gs.plan(dg, 32)
+
+
+@pytest.mark.parametrize("plan_kernel", ["0", "1"])
+def test_one_call_step_inline_plan_matches_oracle(monkeypatch, plan_kernel):
+    """gnn_plan_spmm_sddmm with the boundary table recomputed inside the kernels (and the
+    PDL SpMM) against the oracle, on graphs with hubs split over many chunks, empty rows
+    and a row shard; the plan-kernel path (GNN_STEP_PLAN_KERNEL=1) likewise."""
+    monkeypatch.setenv("GNN_STEP_PLAN_KERNEL", plan_kernel)
+    rng = np.random.default_rng(77)
+    for t in range(4):
+        M = int(rng.integers(100, 3000))
+        nnz = int(rng.integers(1000, 60000))
+        rows = np.sort(rng.integers(0, M, nnz))
+        rows[: nnz // 4] = rows[0]  # a hub
+        g = gen.from_coo(M, M, rows, rng.integers(0, M, nnz), gen.uniform_values(80 + t, nnz))
+        K = int(rng.choice([32, 64, 128, 256]))
+        dg = upload(g)
+        X = torch.from_numpy(_x(90 + t, g.N, K)).to(DEV)
+        O = torch.full((g.M, K), float("nan"), device=DEV)
+        E = torch.full((g.nnz,), float("nan"), device=DEV)
+        gs.StepRunner(DEV)(dg, X, O, E)
+        torch.cuda.synchronize()
+        Xh = X.cpu().numpy()
+        ref, T = oracle.spmm(g.row_ind, g.col_ind, g.val, Xh, M=g.M)
+        assert_within(O.cpu().numpy(), ref, T, what=f"one-call spmm t={t}")
+        r2, T2 = oracle.sddmm(g.row_ind, g.col_ind, g.val, Xh, Xh)
+        assert_within(E.cpu().numpy(), r2, T2, what=f"one-call sddmm t={t}")
