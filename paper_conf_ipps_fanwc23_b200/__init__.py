@@ -50,7 +50,8 @@ class PlanOpts(ctypes.Structure):
                 ("force_chunk", ctypes.c_int32), ("force_vw", ctypes.c_int32),
                 ("deterministic", ctypes.c_int32), ("feature_dtype", ctypes.c_int32),
                 ("no_locality", ctypes.c_int32), ("num_sms", ctypes.c_int32),
-                ("active_blocks_per_sm", ctypes.c_int32), ("l2_bytes", ctypes.c_int64)]
+                ("active_blocks_per_sm", ctypes.c_int32), ("l2_bytes", ctypes.c_int64),
+                ("hub_rows", ctypes.c_int64)]
 
 
 class _PlanInfo(ctypes.Structure):
@@ -64,7 +65,8 @@ class _PlanInfo(ctypes.Structure):
 class ReorderOpts(ctypes.Structure):
     """gnn_reorder_opts_t; zero fields take defaults (3 levels, 20 passes, 1e-6, 1.0)."""
     _fields_ = [("max_levels", ctypes.c_int32), ("max_passes", ctypes.c_int32),
-                ("min_gain", ctypes.c_double), ("resolution", ctypes.c_double)]
+                ("min_gain", ctypes.c_double), ("resolution", ctypes.c_double),
+                ("hub_rows", ctypes.c_int64)]
 
 
 EXPORTS = ["gnn_plan_workspace_bytes", "gnn_plan_create", "gnn_plan_info", "gnn_plan_arrays",
@@ -271,25 +273,27 @@ def _dtype_code(d):
 
 def _opts(alpha=0, warps_per_block=0, force_chunk=0, force_vw=0, feature_dtype=0,
           deterministic=False, no_locality=False, num_sms=0, active_blocks_per_sm=0,
-          l2_bytes=0):
+          l2_bytes=0, hub_rows=0):
     return PlanOpts(alpha, warps_per_block, force_chunk, force_vw, int(bool(deterministic)),
                     _dtype_code(feature_dtype), int(bool(no_locality)), num_sms,
-                    active_blocks_per_sm, l2_bytes)
+                    active_blocks_per_sm, l2_bytes, hub_rows)
 
 
 def plan(graph: DeviceGraph, K: int, alpha: int = 0, warps_per_block: int = 0,
          force_chunk: int = 0, force_vw: int = 0, feature_dtype=GNN_F32,
          deterministic: bool = False, no_locality: bool = False, num_sms: int = 0,
-         active_blocks_per_sm: int = 0, l2_bytes: int = 0, stream=None) -> Plan:
+         active_blocks_per_sm: int = 0, l2_bytes: int = 0, hub_rows: int = 0,
+         stream=None) -> Plan:
     """gnn_plan_create: DTP/HVMA chunking + the GPU plan kernel (no host sync).
     feature_dtype: fp32 (default) or bf16 feature matrices.
     deterministic: split rows summed in chunk order without atomics (bit-reproducible).
     no_locality: plain DTP (InEq. 5), without the L2 locality cap and the chunk floor
     (DESIGN.md §3 steps 5b, 5c).  num_sms / active_blocks_per_sm / l2_bytes: device-
-    parameter overrides for the plan arithmetic only (0 = the device's)."""
+    parameter overrides for the plan arithmetic only (0 = the device's).  hub_rows: feature
+    rows [0, hub_rows) gathered with an L2 evict_last policy (reorder_gcr(hub_rows=))."""
     L = lib()
     o = _opts(alpha, warps_per_block, force_chunk, force_vw, feature_dtype, deterministic,
-              no_locality, num_sms, active_blocks_per_sm, l2_bytes)
+              no_locality, num_sms, active_blocks_per_sm, l2_bytes, hub_rows)
     nbytes = L.gnn_plan_workspace_bytes(graph.M, graph.nnz, K, ctypes.byref(o))
     if nbytes == ctypes.c_size_t(-1).value:
         _check(GNN_ERR_INVALID_ARG)
@@ -489,16 +493,18 @@ def validate(graph: DeviceGraph, stream=None) -> None:
 
 
 # ---------------------------------------------------------------- reorder ---
-def reorder_gcr(row_ptr, col_ind, max_levels=0, max_passes=0, min_gain=0.0, resolution=0.0):
+def reorder_gcr(row_ptr, col_ind, max_levels=0, max_passes=0, min_gain=0.0, resolution=0.0,
+                hub_rows=0):
     """gnn_reorder_gcr (host): Louvain-based GCR permutation of a square symmetric graph.
-    Returns (perm, community, modularity) with perm[old] = new."""
+    Returns (perm, community, modularity) with perm[old] = new.  hub_rows > 0 places the
+    hub_rows highest-degree nodes first (a contiguous hub block of X)."""
     rp = np.ascontiguousarray(row_ptr, dtype=np.int32)
     ci = np.ascontiguousarray(col_ind, dtype=np.int32)
     n = rp.shape[0] - 1
     perm = np.empty(n, np.int32)
     comm = np.empty(n, np.int32)
     q = ctypes.c_double(0.0)
-    o = ReorderOpts(max_levels, max_passes, min_gain, resolution)
+    o = ReorderOpts(max_levels, max_passes, min_gain, resolution, hub_rows)
     _check(lib().gnn_reorder_gcr(rp.ctypes.data, ci.ctypes.data, n, ctypes.byref(o),
                                  perm.ctypes.data, comm.ctypes.data, ctypes.byref(q)))
     return perm, comm, q.value

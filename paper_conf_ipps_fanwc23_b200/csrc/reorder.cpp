@@ -260,6 +260,23 @@ GNN_API gnn_status_t gnn_reorder_gcr(const int32_t *row_ptr, const int32_t *col_
       }
       return a < b;
     });
+    if (o.hub_rows > 0) {
+      // hub block (B200 addition, DESIGN.md §5 "hub block"): the hub_rows nodes of largest
+      // degree (ties: smaller id) move to the front, in the hierarchical order among
+      // themselves; the rest keep theirs.  Their feature rows then form one contiguous
+      // block of X that the kernels can keep L2-resident (plan option hub_rows).
+      const int64_t H = o.hub_rows < n ? o.hub_rows : n;
+      std::vector<int32_t> byd(n);
+      for (int64_t i = 0; i < n; ++i) byd[i] = (int32_t)i;
+      auto deg = [&](int32_t v) { return (int64_t)row_ptr[v + 1] - row_ptr[v]; };
+      std::nth_element(byd.begin(), byd.begin() + (H - 1), byd.end(), [&](int32_t a, int32_t b) {
+        const int64_t da = deg(a), db = deg(b);
+        return da != db ? da > db : a < b;
+      });
+      std::vector<char> hub(n, 0);
+      for (int64_t i = 0; i < H; ++i) hub[byd[i]] = 1;
+      std::stable_partition(order.begin(), order.end(), [&](int32_t v) { return hub[v] != 0; });
+    }
     for (int64_t p = 0; p < n; ++p) perm[order[p]] = (int32_t)p;
     if (comm_out) {
       for (int64_t i = 0; i < n; ++i) comm_out[i] = L ? path[L - 1][i] : (int32_t)i;

@@ -203,6 +203,7 @@ SparseArgs make_args(const Plan *p, const gnn_graph_t *g) {
   a.c_begin = 0;
   a.c_end = a.num_chunks;
   a.inline_plan = p->inline_plan ? 1 : 0;
+  a.hub_rows = p->hub_rows;
   return a;
 }
 

@@ -86,3 +86,21 @@ def test_permute_graph_rejects_non_bijection():
     bad = np.zeros(100, np.int32)
     with pytest.raises(gs.GnnError):
         gs.permute_graph(g.row_ptr, g.col_ind, g.val, bad)
+
+
+@pytest.mark.parametrize("H", [1, 50, 400])
+def test_hub_block_first(H):
+    """hub_rows = H: the H highest-degree nodes (ties: smaller id) take new ids [0, H); hubs
+    and non-hubs each keep the relative order of the plain GCR permutation; bijection."""
+    g = gen.powerlaw_graph(3000, 60000, gamma=2.1, n_comm=6, seed=21)
+    p0, c0, q0 = gs.reorder_gcr(g.row_ptr, g.col_ind)
+    p1, c1, q1 = gs.reorder_gcr(g.row_ptr, g.col_ind, hub_rows=H)
+    assert sorted(p1) == list(range(g.N))
+    assert np.array_equal(c0, c1) and q0 == q1
+    deg = np.diff(g.row_ptr.astype(np.int64))
+    top = sorted(range(g.N), key=lambda v: (-deg[v], v))[:H]
+    assert set(np.flatnonzero(p1 < H)) == set(top)
+    hub = p1 < H
+    for mask in (hub, ~hub):
+        nodes = np.flatnonzero(mask)
+        assert np.array_equal(np.argsort(p1[nodes]), np.argsort(p0[nodes]))
