@@ -45,9 +45,9 @@ variant: $(OBJS)
 	cat $(OBJDIR)/*.ptxas.log > build/ptxas_$(TAG).log
 
 # measurement probes (tools/microbench.py), not part of the product
-micro: build/libgnnmicro.so
-build/libgnnmicro.so: tools/microbench.cu
-	@mkdir -p build
+micro: variants/libgnnmicro.so
+variants/libgnnmicro.so: tools/microbench.cu
+	@mkdir -p variants
 	$(NVCC) $(ARCH) -O3 -shared -Xcompiler -fPIC -o $@ $<
 
 clean:

@@ -71,6 +71,18 @@ def sddmm_bytes(nnz, M, K, eb=4):
     return nnz * (16 + eb * K) + eb * K * M
 
 
+def shard_kernel_bytes(g, spec, K, eb=4):
+    """Algorithmic bytes of one rank's SpMM row shard and SDDMM edge shard at width K
+    (DESIGN.md §7): SpMM over rows [r0, r1) with nonzeros [e0, e1); SDDMM over edges
+    [f0, f1), whose A1 reads are the rows that edge range spans (each rank reads a row
+    split between two edge shards -- counting g.M on every rank would count the A1 term
+    P times)."""
+    sp_nnz, sp_rows = spec.e1 - spec.e0, spec.r1 - spec.r0
+    sd_nnz = spec.f1 - spec.f0
+    sd_rows = (int(g.row_ind[spec.f1 - 1]) - int(g.row_ind[spec.f0]) + 1) if sd_nnz else 0
+    return spmm_bytes(sp_nnz, sp_rows, K, eb), sddmm_bytes(sd_nnz, sd_rows, K, eb), sd_rows
+
+
 def plan_bytes(nch):
     return nch * (16 + 9)
 
@@ -367,14 +379,10 @@ def time_path(args, g, perm, name, Ks, dev, world, rank, dtype="f32", xmode=None
         step_ms.append(tot)
     my_bytes, my_flops, detail = 0, 0, {}
     eb = 2 if dtype == "bf16" else 4
-    # A1 rows this rank's SDDMM edge shard reads (its row span; the whole graph at P = 1):
-    # counting g.M on every rank would count the A1 term P times in the aggregate
-    sd_rows = (int(g.row_ind[spec.f1 - 1]) - int(g.row_ind[spec.f0]) + 1) if sdg.nnz else 0
     kb = {}
     for K in Ks:
         info = gs.plan(spg, K, feature_dtype=dtype).info()
-        b_sp = spmm_bytes(spg.nnz, spg.M, K, eb)
-        b_sd = sddmm_bytes(sdg.nnz, sd_rows, K, eb)
+        b_sp, b_sd, sd_rows = shard_kernel_bytes(g, spec, K, eb)
         kb[K] = {"spmm": b_sp, "sddmm": b_sd}
         my_bytes += b_sp + b_sd + plan_bytes(info["num_chunks"])
         my_flops += spmm_flops(spg.nnz, K) + sddmm_flops(sdg.nnz, K)
@@ -424,6 +432,20 @@ def init_dist(world, local):
         ncores = os.cpu_count() or 1
         os.environ["OMP_NUM_THREADS"] = str(max(1, ncores // world))
     return dev
+
+
+def per_rank_bytes(r, world, dev):
+    """This path's algorithmic bytes per step on every rank (list, rank order)."""
+    import torch
+    import torch.distributed as dist
+    if world == 1:
+        return [int(r["bytes"])]
+    rank = dist.get_rank()
+    t = torch.zeros(world, dtype=torch.float64,
+                    device=dev if dist.get_backend() == "nccl" else "cpu")
+    t[rank] = float(r["bytes"])
+    dist.all_reduce(t)
+    return [int(x) for x in t.tolist()]
 
 
 def aggregate(r, args, world, dev):
@@ -501,6 +523,7 @@ def measure_workload(args, name, Ks, reorder, dev, world, rank, legs=("bf16", "n
         g, perm, reorder_info = g0, None, None
     r = time_path(args, g, perm, name, Ks, dev, world, rank)
     tot_ms, tot_bytes, tot_flops = aggregate(r, args, world, dev)
+    by_rank = per_rank_bytes(r, world, dev)
     roof = roofline_for(name, reorder, r, Ks, world, args)
     step_ms = [float(x) for x in r["step_ms"]]
     block = {"value": round(tot_bytes / (tot_ms * 1e-3) / 1e9, 2), "unit": "GB/s",
@@ -513,6 +536,11 @@ def measure_workload(args, name, Ks, reorder, dev, world, rank, legs=("bf16", "n
                                     + (", GCR-reordered offline" if reorder else ""),
                         "K": Ks, "nnz": g.nnz, "M": g.M, "N": g.N, "degree": g.degree_stats(),
                         "graph_gen_s": round(gen_s, 1), "reorder": reorder_info},
+             "bytes_per_step": {"by_rank": by_rank, "total": int(sum(by_rank)),
+                                "note": "SpMM row shard + SDDMM edge shard of each rank; "
+                                        "the total exceeds one GPU's by the A1 rows of "
+                                        "rows split between edge shards (each rank reads "
+                                        "them)"},
              "roofline": roof, "gpu_launches": r["launches"] * args.steps,
              "clocks": r["clocks"], "kernels": r["detail"]}
     del r
@@ -627,7 +655,7 @@ def run_ours(args):
                            l2="flushed between timed steps (256 MiB write, outside events)",
                            parallelism=f"rowshard-spmm/edgeshard-sddmm x{world}",
                            xmode=args.xmode),
-            "gflops": head["gflops"],
+            "gflops": head["gflops"], "bytes_per_step": head["bytes_per_step"],
             "roofline": head["roofline"], "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": head["gpu_launches"], "clocks": head["clocks"],
             "kernels": head["kernels"], "no_reorder": head.get("no_reorder"),

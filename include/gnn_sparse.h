@@ -92,11 +92,6 @@ typedef struct {
   int32_t num_sms;              /* NumSM of Eq. 4                                      */
   int32_t active_blocks_per_sm; /* ActiveblocksPerSM of Eq. 3 (else the occupancy API) */
   int64_t l2_bytes;             /* L2 bytes of step 5b (no_locality still disables it) */
-  /* Hub block (B200 addition): feature rows [0, hub_rows) -- the highest-
-   * degree nodes after gnn_reorder_gcr with its hub_rows option -- are gathered with an
-   * L2 evict_last policy so they stay resident while the rest streams; 0 = off.  A launch
-   * attribute only: results and plan info are unchanged. */
-  int64_t hub_rows;
 } gnn_plan_opts_t;
 
 /* What the plan decided (all integers; bit-exact with the oracle's plan). */
@@ -258,7 +253,9 @@ typedef struct {
   double resolution;
   int64_t hub_rows;  /* > 0: the hub_rows nodes of largest degree (ties: smaller id) are
                         placed first, in the community order among themselves, so their
-                        feature rows form one block X[0, hub_rows) (plan option hub_rows) */
+                        feature rows form one contiguous block X[0, hub_rows) (DESIGN.md §5:
+                        measured on C5 with and without an L2 evict_last hint on that block:
+                        no gain; kept for experiments) */
 } gnn_reorder_opts_t;
 GNN_API gnn_status_t gnn_reorder_gcr(const int32_t *row_ptr_host, const int32_t *col_ind_host,
                                      int64_t n, const gnn_reorder_opts_t *opts,

@@ -50,8 +50,7 @@ class PlanOpts(ctypes.Structure):
                 ("force_chunk", ctypes.c_int32), ("force_vw", ctypes.c_int32),
                 ("deterministic", ctypes.c_int32), ("feature_dtype", ctypes.c_int32),
                 ("no_locality", ctypes.c_int32), ("num_sms", ctypes.c_int32),
-                ("active_blocks_per_sm", ctypes.c_int32), ("l2_bytes", ctypes.c_int64),
-                ("hub_rows", ctypes.c_int64)]
+                ("active_blocks_per_sm", ctypes.c_int32), ("l2_bytes", ctypes.c_int64)]
 
 
 class _PlanInfo(ctypes.Structure):
@@ -273,27 +272,25 @@ def _dtype_code(d):
 
 def _opts(alpha=0, warps_per_block=0, force_chunk=0, force_vw=0, feature_dtype=0,
           deterministic=False, no_locality=False, num_sms=0, active_blocks_per_sm=0,
-          l2_bytes=0, hub_rows=0):
+          l2_bytes=0):
     return PlanOpts(alpha, warps_per_block, force_chunk, force_vw, int(bool(deterministic)),
                     _dtype_code(feature_dtype), int(bool(no_locality)), num_sms,
-                    active_blocks_per_sm, l2_bytes, hub_rows)
+                    active_blocks_per_sm, l2_bytes)
 
 
 def plan(graph: DeviceGraph, K: int, alpha: int = 0, warps_per_block: int = 0,
          force_chunk: int = 0, force_vw: int = 0, feature_dtype=GNN_F32,
          deterministic: bool = False, no_locality: bool = False, num_sms: int = 0,
-         active_blocks_per_sm: int = 0, l2_bytes: int = 0, hub_rows: int = 0,
-         stream=None) -> Plan:
+         active_blocks_per_sm: int = 0, l2_bytes: int = 0, stream=None) -> Plan:
     """gnn_plan_create: DTP/HVMA chunking + the GPU plan kernel (no host sync).
     feature_dtype: fp32 (default) or bf16 feature matrices.
     deterministic: split rows summed in chunk order without atomics (bit-reproducible).
     no_locality: plain DTP (InEq. 5), without the L2 locality cap and the chunk floor
     (DESIGN.md §3 steps 5b, 5c).  num_sms / active_blocks_per_sm / l2_bytes: device-
-    parameter overrides for the plan arithmetic only (0 = the device's).  hub_rows: feature
-    rows [0, hub_rows) gathered with an L2 evict_last policy (reorder_gcr(hub_rows=))."""
+    parameter overrides for the plan arithmetic only (0 = the device's)."""
     L = lib()
     o = _opts(alpha, warps_per_block, force_chunk, force_vw, feature_dtype, deterministic,
-              no_locality, num_sms, active_blocks_per_sm, l2_bytes, hub_rows)
+              no_locality, num_sms, active_blocks_per_sm, l2_bytes)
     nbytes = L.gnn_plan_workspace_bytes(graph.M, graph.nnz, K, ctypes.byref(o))
     if nbytes == ctypes.c_size_t(-1).value:
         _check(GNN_ERR_INVALID_ARG)

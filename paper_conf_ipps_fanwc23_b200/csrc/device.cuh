@@ -29,11 +29,6 @@ __device__ __forceinline__ uint64_t l2_evict_first() {
   asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
   return pol;
 }
-__device__ __forceinline__ uint64_t l2_evict_normal() {
-  uint64_t pol;
-  asm("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(pol));
-  return pol;
-}
 __device__ __forceinline__ uint64_t l2_evict_last() {
   uint64_t pol;
   asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
@@ -84,27 +79,6 @@ __device__ __forceinline__ void ld_feat<8>(const float *p, float (&x)[8]) {
                  "=f"(x[6]), "=f"(x[7])
                : "l"(p));
 #endif
-}
-
-// The same loads with an explicit L2 policy (hub block rows: evict_last).
-template <int VW>
-__device__ __forceinline__ void ld_feat_hint(const float *p, uint64_t pol, float (&x)[VW]) {
-  if constexpr (VW == 8) {
-    asm("ld.global.nc.L2::cache_hint.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
-        : "=f"(x[0]), "=f"(x[1]), "=f"(x[2]), "=f"(x[3]), "=f"(x[4]), "=f"(x[5]), "=f"(x[6]),
-          "=f"(x[7])
-        : "l"(p), "l"(pol));
-  } else if constexpr (VW == 4) {
-    asm("ld.global.nc.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;"
-        : "=f"(x[0]), "=f"(x[1]), "=f"(x[2]), "=f"(x[3])
-        : "l"(p), "l"(pol));
-  } else if constexpr (VW == 2) {
-    asm("ld.global.nc.L2::cache_hint.v2.f32 {%0,%1}, [%2], %3;"
-        : "=f"(x[0]), "=f"(x[1])
-        : "l"(p), "l"(pol));
-  } else {
-    asm("ld.global.nc.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(x[0]) : "l"(p), "l"(pol));
-  }
 }
 
 // ------------------------------------------------------------- outputs ----
@@ -244,9 +218,6 @@ struct FeatVec<F32, VW> {
   __device__ __forceinline__ void load(const char *p) {
     ld_feat<VW>(reinterpret_cast<const float *>(p), r);
   }
-  __device__ __forceinline__ void load_hint(const char *p, uint64_t pol) {
-    ld_feat_hint<VW>(reinterpret_cast<const float *>(p), pol, r);
-  }
   __device__ __forceinline__ void zero() {
 #pragma unroll
     for (int v = 0; v < VW; ++v) r[v] = 0.f;
@@ -274,60 +245,12 @@ struct FeatVec<BF16, VW> {
       asm("ld.global.nc.b32 %0, [%1];" : "=r"(r[0]) : "l"(p));
     }
   }
-  __device__ __forceinline__ void load_hint(const char *p, uint64_t pol) {
-    if constexpr (VW == 16) {
-      asm("ld.global.nc.L2::cache_hint.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
-          : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
-            "=r"(r[7])
-          : "l"(p), "l"(pol));
-    } else if constexpr (VW == 8) {
-      asm("ld.global.nc.L2::cache_hint.v4.b32 {%0,%1,%2,%3}, [%4], %5;"
-          : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3])
-          : "l"(p), "l"(pol));
-    } else if constexpr (VW == 4) {
-      asm("ld.global.nc.L2::cache_hint.v2.b32 {%0,%1}, [%2], %3;"
-          : "=r"(r[0]), "=r"(r[1])
-          : "l"(p), "l"(pol));
-    } else {
-      asm("ld.global.nc.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(r[0]) : "l"(p), "l"(pol));
-    }
-  }
   __device__ __forceinline__ void zero() {
 #pragma unroll
     for (int v = 0; v < VW / 2; ++v) r[v] = 0u;
   }
   __device__ __forceinline__ float get(int v) const {
     return (v & 1) ? __uint_as_float(r[v >> 1] & 0xffff0000u) : __uint_as_float(r[v >> 1] << 16);
-  }
-};
-
-// Gather of feature row `col` at p: rows of the hub block [0, hub_rows) carry an L2
-// evict_last policy (kept resident across the kernel), the others evict_normal.  Off
-// (hub_rows == 0, the default) it is the plain load.
-#ifndef GNN_HUB_HINT
-#define GNN_HUB_HINT 1
-#endif
-struct HubPolicy {
-  uint64_t hub, rest;
-  int64_t rows;
-  __device__ __forceinline__ void init(int64_t hub_rows) {
-    rows = hub_rows;
-#if GNN_HUB_HINT
-    if (rows) {
-      hub = l2_evict_last();
-      rest = l2_evict_normal();
-    }
-#endif
-  }
-  template <typename TF, int VW>
-  __device__ __forceinline__ void gather(FeatVec<TF, VW> &x, const char *p, uint32_t col) const {
-#if GNN_HUB_HINT
-    if (rows) {
-      x.load_hint(p, (int64_t)col < rows ? hub : rest);
-      return;
-    }
-#endif
-    x.load(p);
   }
 };
 

@@ -33,7 +33,6 @@ struct Plan {
   int64_t M;
   int64_t row_base;
   bool inline_plan = false;  // kernels recompute the boundary table (gnn_plan_spmm_sddmm)
-  int64_t hub_rows = 0;      // opts.hub_rows: L2-resident hub block of the feature rows
 };
 
 // Kernel parameter block shared by the SpMM / SDDMM launchers.
@@ -58,7 +57,6 @@ struct SparseArgs {
                            // pipelined host path launches a plan piece by piece
   int32_t inline_plan;     // 1: no plan arrays -- each chunk derives its boundary rows and
                            // flags from row_ind (the plan kernel's arithmetic) itself
-  int64_t hub_rows;        // gathers of feature rows [0, hub_rows) carry L2 evict_last
 };
 
 #ifdef __CUDACC__

@@ -69,7 +69,7 @@ gnn_status_t make_info(int64_t M, int64_t nnz, int32_t K, const gnn_plan_opts_t 
   const int32_t G = 32 / L;
   // step 3: FullWaveSize (Eqs. 3-4) from the occupancy of the SpMM kernel, unless the
   // caller overrides the device parameters (tests feed the same values to the oracle)
-  if (o.num_sms < 0 || o.active_blocks_per_sm < 0 || o.l2_bytes < 0 || o.hub_rows < 0)
+  if (o.num_sms < 0 || o.active_blocks_per_sm < 0 || o.l2_bytes < 0)
     return fail(GNN_ERR_INVALID_ARG, "plan: negative device-parameter override");
   DeviceInfo d;
   if (gnn_status_t st = device_info(&d)) return st;
@@ -198,7 +198,6 @@ gnn_status_t plan_create(const gnn_graph_t *g, int32_t K, const gnn_plan_opts_t 
   p->row_ind = g->row_ind;
   p->M = g->M;
   p->row_base = g->row_base;
-  p->hub_rows = opts ? opts->hub_rows : 0;
   char *w = (char *)workspace;
   p->row_first = (int32_t *)w;
   p->row_last = (int32_t *)(w + align256(sizeof(int32_t) * nch));

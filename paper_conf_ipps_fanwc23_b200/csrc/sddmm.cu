@@ -10,9 +10,12 @@
 // with a transposed butterfly that reduces U nonzeros at once (WarpReduce, line 12),
 // scale by val_i after the sum (Algo 2 line 6) and store: the U results of a
 // batch land in consecutive lanes, so the store is coalesced; each output is written
-// exactly once (plain stores, deterministic).  Tiles whose nonzeros all share one
-// row (for every group of the warp) take a fast path with no per-nonzero row or
-// bounds logic; the next tile's sparse entries are prefetched into registers.
+// exactly once (plain stores, deterministic).  The sparse entries come from the same
+// per-warp cp.async shared-memory ring as SpMM's (one tile ahead of use); tiles whose
+// nonzeros all share one row (for every group of the warp) take a fast path with no
+// per-nonzero row or bounds logic, and single-slice rows issue the next batch's gathers
+// before this batch's butterfly (software pipelining).  SDDMM never reads the plan's
+// boundary table, only its chunk size and lane shape.
 #include "sddmm_kernel.cuh"
 
 namespace gnn {

@@ -163,8 +163,6 @@ __global__ void __maxnreg__(SddmmRegs<TF>::value)
 
   const float *__restrict__ vi = a.val ? a.val + cs : nullptr;
   float *__restrict__ oc = out + cs;
-  HubPolicy hp;
-  hp.init(a.hub_rows);
   // sparse tiles: per-warp double-buffered shared-memory ring (TMA bulk copies, or
   // cp.async for narrow sparse vectors), one tile ahead of use
   extern __shared__ int32_t gnn_smem[];
@@ -247,7 +245,7 @@ __global__ void __maxnreg__(SddmmRegs<TF>::value)
               const char *rowp = A2l + (uint64_t)cj[u] * ld2B;
 #pragma unroll
               for (int r = 0; r < R; ++r) {
-                if (lane_ok[r] && (FAST || u < valid)) hp.gather(x[u][r], rowp + r * Lg * VW * ES, cj[u]);
+                if (lane_ok[r] && (FAST || u < valid)) x[u][r].load(rowp + r * Lg * VW * ES);
                 else x[u][r].zero();
               }
             }
@@ -282,11 +280,10 @@ __global__ void __maxnreg__(SddmmRegs<TF>::value)
       auto load_batch = [&](int jj) {
 #pragma unroll
         for (int u = 0; u < U; ++u) {
-          const uint32_t col = (uint32_t)s_col[jj + u];
-          const char *rowp = A2l + (uint64_t)col * ld2B;
+          const char *rowp = A2l + (uint64_t)(uint32_t)s_col[jj + u] * ld2B;
 #pragma unroll
           for (int r = 0; r < R; ++r) {
-            if (lane_ok[r]) hp.gather(x[u][r], rowp + r * Lg * VW * ES, col);
+            if (lane_ok[r]) x[u][r].load(rowp + r * Lg * VW * ES);
             else x[u][r].zero();
           }
         }
@@ -322,11 +319,10 @@ __global__ void __maxnreg__(SddmmRegs<TF>::value)
         const int valid = n - (tb + jj);
 #pragma unroll
         for (int u = 0; u < U; ++u) {
-          const uint32_t col = (uint32_t)s_col[jj + u];
-          const char *rowp = A2l + (uint64_t)col * ld2B;
+          const char *rowp = A2l + (uint64_t)(uint32_t)s_col[jj + u] * ld2B;
 #pragma unroll
           for (int r = 0; r < R; ++r) {
-            if (lane_ok[r] && u < valid) hp.gather(x[u][r], rowp + r * Lg * VW * ES, col);
+            if (lane_ok[r] && u < valid) x[u][r].load(rowp + r * Lg * VW * ES);
             else x[u][r].zero();
           }
         }

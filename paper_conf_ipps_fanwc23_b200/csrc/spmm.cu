@@ -1,22 +1,21 @@
 // spmm.cu -- hybrid-parallel SpMM for sm_100a (O = S A; Algorithm 1
 // is the definition, Algorithm 3 P:168-195 the prior-art GPU design).
 //
-// Work decomposition: the plan cuts the nnz into chunks of C*
-// consecutive nonzeros (equal work per unit, hybrid node/edge parallelism).
-// Each (chunk, K-slice) work item is owned by a lane group of L lanes; every lane
-// holds VW consecutive feature columns, so one group gathers L*VW columns of a
-// source row per nonzero with one vector load per lane (128-bit, or 256-bit at
-// VW = 8).  G = 32/L groups share a warp.  Per tile of T = L*vw_sparse nonzeros the
-// group loads (row, col, val) coalesced and vectorised, then broadcasts them
-// nonzero by nonzero with width-L shuffles; U feature rows are in flight per lane
-// before the FMAs consume them, and the next tile's sparse entries are prefetched into
-// registers.  Tiles whose nonzeros all belong to one row (for every group of the warp;
+// Work decomposition: the plan cuts the nnz into chunks of C* consecutive
+// nonzeros (equal work per unit, hybrid node/edge parallelism).  Each (chunk,
+// K-slice) work item is owned by a lane group of L lanes; every lane holds VW consecutive
+// feature columns, so one group gathers L*VW columns of a source row per nonzero with one
+// vector load per lane (256-bit at VW = 8 fp32 / 16 bf16).  G = 32/L groups share a warp.
+// The chunk's (row, col, val) entries are staged through a per-warp, double-buffered
+// shared-memory ring filled by cp.async one tile ahead of use, and read back as
+// warp-broadcast shared loads; U feature rows are in flight per lane before the FMAs
+// consume them.  Tiles whose nonzeros all belong to one row (for every group of the warp;
 // the common case at high degree) take a fast path with no per-nonzero row or bounds
-// logic; the others run the general row-switch loop.  A row switch ("row-switch procedure")
-// flushes the accumulator: rows wholly inside the chunk get a plain vector store,
-// rows shared with a neighbouring chunk (plan flags) a vector atomic add into a row
-// zeroed beforehand by spmm_prezero_kernel.  Empty rows are written as zeros by the
-// chunk that precedes them, so O is fully overwritten without a memset.
+// logic; the others run the general row-switch loop.  A row switch ("row-switch
+// procedure") flushes the accumulator: rows wholly inside the chunk get a plain vector
+// store, rows shared with a neighbouring chunk (plan flags) a vector atomic add into a row
+// zeroed beforehand by spmm_prezero_kernel.  Empty rows are written as zeros by the chunk
+// that precedes them, so O is fully overwritten without a memset.
 #include <atomic>
 #include <climits>
 
@@ -203,7 +202,6 @@ SparseArgs make_args(const Plan *p, const gnn_graph_t *g) {
   a.c_begin = 0;
   a.c_end = a.num_chunks;
   a.inline_plan = p->inline_plan ? 1 : 0;
-  a.hub_rows = p->hub_rows;
   return a;
 }
 

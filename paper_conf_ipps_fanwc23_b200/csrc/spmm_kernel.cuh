@@ -207,8 +207,6 @@ __global__ void __maxnreg__((SpmmTune<TF, VW, L, R, AGG>::regs))
   int32_t cur = -1;
 
   const float *__restrict__ vi = a.val ? a.val + cs : nullptr;
-  HubPolicy hp;
-  hp.init(a.hub_rows);
   // sparse tiles: per-warp double-buffered shared-memory ring (TMA bulk copies, or
   // cp.async for narrow sparse vectors), one tile ahead of use
   extern __shared__ int32_t gnn_smem[];
@@ -272,7 +270,7 @@ __global__ void __maxnreg__((SpmmTune<TF, VW, L, R, AGG>::regs))
           const char *rowp = Ab + (uint64_t)cj[u] * ldaB;
 #pragma unroll
           for (int r = 0; r < R; ++r) {
-            if (col_ok[r]) hp.gather(x[u][r], rowp + r * Lg * VW * ES, cj[u]);
+            if (col_ok[r]) x[u][r].load(rowp + r * Lg * VW * ES);
             else x[u][r].zero();
           }
         }
@@ -300,7 +298,7 @@ __global__ void __maxnreg__((SpmmTune<TF, VW, L, R, AGG>::regs))
           const char *rowp = Ab + (uint64_t)cj[u] * ldaB;
 #pragma unroll
           for (int r = 0; r < R; ++r) {
-            if (col_ok[r] && tb + jj + u < n) hp.gather(x[u][r], rowp + r * Lg * VW * ES, cj[u]);
+            if (col_ok[r] && tb + jj + u < n) x[u][r].load(rowp + r * Lg * VW * ES);
             else x[u][r].zero();
           }
         }

@@ -154,3 +154,33 @@ def test_gloo_overlapped_block_broadcast_spmm():
         p.join(timeout=240)
         assert p.exitcode == 0
     assert q.get(timeout=10)
+
+
+@pytest.mark.parametrize("P", [1, 2, 3, 8])
+def test_bench_shard_bytes_add_up(P):
+    """bench.py's per-rank byte model (shard_kernel_bytes): SpMM bytes of the P row
+    shards sum to the single-GPU SpMM bytes exactly; SDDMM bytes of the P edge shards
+    sum to the single-GPU SDDMM bytes plus one A1 row (4K B) per row split between two
+    edge shards -- the A1 term is not counted P times (round-1 overcount)."""
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    sys.path.insert(0, root)
+    import bench
+    import gen
+    from paper_conf_ipps_fanwc23_b200 import dist as gdist
+    g = gen.powerlaw_graph(3001, 60000, gamma=2.2, n_comm=5, seed=91)
+    K = 64
+    one = gdist.shard_spec(g.row_ptr, g.N, 0, 1)
+    sp1, sd1, rows1 = bench.shard_kernel_bytes(g, one, K)
+    assert rows1 == g.M and sp1 == bench.spmm_bytes(g.nnz, g.M, K)
+    sp = sd = 0
+    split = 0
+    for r in range(P):
+        s = gdist.shard_spec(g.row_ptr, g.N, r, P)
+        a, b, _ = bench.shard_kernel_bytes(g, s, K)
+        sp += a
+        sd += b
+        if r and s.f0 < g.nnz and s.f0 > 0 and g.row_ind[s.f0] == g.row_ind[s.f0 - 1]:
+            split += 1
+    assert sp == sp1
+    assert sd == sd1 + split * 4 * K

@@ -1,7 +1,9 @@
 """C5 (products-shaped, X = 2.5 GB >> L2) DRAM over-fetch experiments, K = 256:
 GCR order with a hub block of H rows first (reorder_gcr(hub_rows=H)) x gathers of that
-block with an L2 evict_last policy (plan hub_rows), and SpMM split into two K = 128
-column halves (half the bytes per row in flight).  SpMM / SDDMM timed with CUDA events,
+block with an L2 evict_last policy (plan option hub_rows of the library at commit 084431e;
+the hint measured slower and was removed, profiles/r02_s3_c5_hub.txt -- with later
+libraries only hint = 0 runs), and SpMM split into two K = 128 column halves (half the
+bytes per row in flight).  SpMM / SDDMM timed with CUDA events,
 L2 flushed between runs, median of --reps.  One JSON line per setting.
 
     python tools/c5_hub.py [--hubs 0,32768,65536] [--reps 5] [--profile H:hint]
@@ -66,10 +68,12 @@ def main():
             X = X.to(torch.bfloat16)
         O = torch.empty((g.M, K), device="cuda")
         E = torch.empty(g.nnz, device="cuda")
-        for hint in ([0, 1] if H else [0]):
+        has_hint = "hub_rows" in dict(gs.PlanOpts._fields_)
+        for hint in ([0, 1] if H and has_hint else [0]):
             if a.profile and hint != int(a.profile.split(":")[1]):
                 continue
-            p = gs.plan(dg, K, feature_dtype=a.dtype, hub_rows=H if hint else 0)
+            kw = {"hub_rows": H} if hint else {}
+            p = gs.plan(dg, K, feature_dtype=a.dtype, **kw)
             if a.profile:
                 gs.spmm(p, dg, X, out=O)
                 gs.sddmm(p, dg, X, X, out=E)
@@ -82,7 +86,7 @@ def main():
             res["sddmm_ms"] = timed(lambda: gs.sddmm(p, dg, X, X, out=E), a.reps, flush)
             if K % 2 == 0 and a.dtype == "f32":
                 # K-split: two launches over column halves (pitched views, same graph)
-                ph = gs.plan(dg, K // 2, hub_rows=H if hint else 0)
+                ph = gs.plan(dg, K // 2, **kw)
                 Xa, Xb = X[:, :K // 2], X[:, K // 2:]
                 Oa, Ob = O[:, :K // 2], O[:, K // 2:]
 

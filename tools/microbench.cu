@@ -5,7 +5,9 @@
 //   mb_copy  : streaming copy (HBM read+write).
 //   mb_shfl  : warp-shuffle issue rate (8 independent xor-shuffle chains per thread):
 //              the cost of a shuffle-based segmented reduction in SpMM.
-// Not part of the product ABI (built into build/libgnnmicro.so).
+//   mb_fma   : fp32 FMA throughput, scalar FFMA vs packed FFMA2 (fma.rn.f32x2), 16
+//              independent accumulator pairs per thread (SURVEY §8(d) peak #4).
+// Not part of the product ABI (built into variants/libgnnmicro.so).
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -68,7 +70,42 @@ __global__ void shfl_kernel(int iters, float *__restrict__ out) {
   if (s == 1234.5f) out[0] = s;
 }
 
+template <bool PACKED>
+__global__ void fma_kernel(int iters, float *__restrict__ out) {
+  float a[32];
+#pragma unroll
+  for (int j = 0; j < 32; ++j) a[j] = threadIdx.x * 1e-3f + j;
+  const float x0 = 1.0001f, x1 = 0.9999f, s = 1e-7f;
+  for (int it = 0; it < iters; ++it) {
+#pragma unroll
+    for (int j = 0; j < 32; j += 2) {
+      if constexpr (PACKED) {
+        uint64_t d, xx, ss;
+        asm("mov.b64 %0, {%1,%2};" : "=l"(d) : "f"(a[j]), "f"(a[j + 1]));
+        asm("mov.b64 %0, {%1,%2};" : "=l"(xx) : "f"(x0), "f"(x1));
+        asm("mov.b64 %0, {%1,%1};" : "=l"(ss) : "f"(s));
+        asm volatile("fma.rn.f32x2 %0, %1, %2, %0;" : "+l"(d) : "l"(xx), "l"(ss));
+        asm("mov.b64 {%0,%1}, %2;" : "=f"(a[j]), "=f"(a[j + 1]) : "l"(d));
+      } else {
+        asm volatile("fma.rn.f32 %0, %1, %2, %0;" : "+f"(a[j]) : "f"(x0), "f"(s));
+        asm volatile("fma.rn.f32 %0, %1, %2, %0;" : "+f"(a[j + 1]) : "f"(x1), "f"(s));
+      }
+    }
+  }
+  float t = 0.f;
+#pragma unroll
+  for (int j = 0; j < 32; ++j) t += a[j];
+  if (t == 1234.5f) out[0] = t;
+}
+
 extern "C" {
+// 32 fp32 FMAs per thread per iteration either way (16 FFMA2 or 32 FFMA instructions)
+__attribute__((visibility("default"))) int mb_fma(int packed, int blocks, int iters, float *out,
+                                                  void *stream) {
+  if (packed) fma_kernel<true><<<blocks, 256, 0, (cudaStream_t)stream>>>(iters, out);
+  else fma_kernel<false><<<blocks, 256, 0, (cudaStream_t)stream>>>(iters, out);
+  return cudaGetLastError() == cudaSuccess ? 0 : 2;
+}
 __attribute__((visibility("default"))) int mb_shfl(int blocks, int iters, float *out, void *stream) {
   shfl_kernel<<<blocks, 256, 0, (cudaStream_t)stream>>>(iters, out);
   return cudaGetLastError() == cudaSuccess ? 0 : 2;

@@ -11,11 +11,12 @@ import sys
 import torch
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-lib = ctypes.CDLL(os.path.join(ROOT, "build", "libgnnmicro.so"))
+lib = ctypes.CDLL(os.path.join(ROOT, "variants", "libgnnmicro.so"))
 vp, i64, i32 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32
 lib.mb_gather.argtypes = [vp, i64, vp, i64, i32, vp, vp, i32]
 lib.mb_copy.argtypes = [vp, vp, i64, vp, i32]
 lib.mb_shfl.argtypes = [i32, i32, vp, vp]
+lib.mb_fma.argtypes = [i32, i32, i32, vp, vp]
 
 
 def timed(fn, reps=10):
@@ -65,6 +66,14 @@ def main():
     warps = blocks * 8
     res["shfl_warp_instr_per_s"] = round(warps * iters * 8 / (ms * 1e-3), 1)
     res["shfl_per_sm_per_clk_at_1965MHz"] = round(warps * iters * 8 / (ms * 1e-3) / nsm / 1.965e9, 3)
+    # fp32 FMA throughput: scalar FFMA vs packed FFMA2 (SURVEY §8(d) peak #4)
+    res["fma"] = {}
+    for packed, tag in ((0, "FFMA"), (1, "FFMA2")):
+        ms = timed(lambda: lib.mb_fma(packed, blocks, iters, vp(out.data_ptr()), st))
+        flops = blocks * 256 * iters * 32 * 2
+        res["fma"][tag] = {"TFLOPs": round(flops / (ms * 1e-3) / 1e12, 2),
+                           "fma_per_sm_per_clk_at_1965MHz":
+                               round(flops / 2 / (ms * 1e-3) / nsm / 1.965e9, 1)}
     print(json.dumps(res), flush=True)
 
 
