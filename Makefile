@@ -50,7 +50,13 @@ variants/libgnnmicro.so: tools/microbench.cu
 	@mkdir -p variants
 	$(NVCC) $(ARCH) -O3 -shared -Xcompiler -fPIC -o $@ $<
 
+# lane-mapping experiment (tools/interleaved_ab.py), not part of the product
+exp: variants/libgnnexp.so
+variants/libgnnexp.so: tools/spmm_interleaved.cu $(PKG)/csrc/device.cuh
+	@mkdir -p variants
+	$(NVCC) $(ARCH) -O3 -std=c++17 -shared -Xcompiler -fPIC -Iinclude -o $@ $<
+
 clean:
 	rm -rf gen/libgnngen.so oracle/liboracle.so $(PKG)/libgnnsparse.so build/obj*
 
-.PHONY: all clean variant micro
+.PHONY: all clean variant micro exp
