@@ -125,10 +125,12 @@ __device__ __forceinline__ void reduce_scale_store(float (&part)[U], const float
 }
 
 // L here is V, the number of VW-wide vectors in one K-slice (plan lanes x vecs).
+// The kernel body with the block index as a parameter (see spmm_body).
 template <typename TF, int VW, int L, int VWS, int SMAX>
-__global__ void __maxnreg__(SddmmRegs<TF>::value)
-    sddmm_kernel(const SparseArgs a, const void *__restrict__ A1, const int64_t lda1,
-                 const void *__restrict__ A2T, const int64_t lda2, float *__restrict__ out) {
+__device__ __forceinline__ void sddmm_body(const SparseArgs &a, const void *__restrict__ A1,
+                                           const int64_t lda1, const void *__restrict__ A2T,
+                                           const int64_t lda2, float *__restrict__ out,
+                                           const int64_t bid) {
   constexpr int ES = TF::bytes;
   using Sh = SddmmShape<VW, L, SMAX>;
   constexpr int R = Sh::R, Lg = Sh::Lg;
@@ -142,7 +144,7 @@ __global__ void __maxnreg__(SddmmRegs<TF>::value)
   const int g = lane / Lg;
   const int l = lane & (Lg - 1);
   const int64_t c =
-      a.c_begin + ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * G + g;
+      a.c_begin + (bid * (blockDim.x >> 5) + (threadIdx.x >> 5)) * G + g;
   const bool item_ok = c < a.c_end;
   if (!__any_sync(kFull, item_ok)) return;
   const int64_t cs = c * a.chunk;
@@ -169,7 +171,7 @@ __global__ void __maxnreg__(SddmmRegs<TF>::value)
   Tiles tiles;
   {
     const int64_t c0 =
-        a.c_begin + ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * G;
+        a.c_begin + (bid * (blockDim.x >> 5) + (threadIdx.x >> 5)) * G;
     tiles.init(gnn_smem + (threadIdx.x >> 5) * Tiles::WARP_WORDS, lane, a.row_ind, a.col_ind,
                a.val, [&](int gg, int64_t &cs_, int &n_) {
                  const int64_t cc = c0 + gg;
@@ -360,6 +362,13 @@ __global__ void __maxnreg__(SddmmRegs<TF>::value)
     if (fast) run_tile(std::true_type{});
     else run_tile(std::false_type{});
   }
+}
+
+template <typename TF, int VW, int L, int VWS, int SMAX>
+__global__ void __maxnreg__(SddmmRegs<TF>::value)
+    sddmm_kernel(const SparseArgs a, const void *__restrict__ A1, const int64_t lda1,
+                 const void *__restrict__ A2T, const int64_t lda2, float *__restrict__ out) {
+  sddmm_body<TF, VW, L, VWS, SMAX>(a, A1, lda1, A2T, lda2, out, blockIdx.x);
 }
 
 using SddmmFn = void (*)(const SparseArgs, const void *__restrict__, const int64_t,

@@ -119,10 +119,12 @@ __device__ __forceinline__ void accumulate(float (&acc)[VW], float s, const Feat
 
 // L lanes per (chunk, K-slice) work item, R VW-wide vectors per lane (plan rule step 2).
 // TF: feature element type (F32 or BF16); accumulation and O are fp32.
+// The kernel body with the block index as a parameter (bid), so a fused launch can run it
+// on a sub-range of its blocks (step_fused.cu).
 template <typename TF, int VW, int L, int R, int VWS, int AGG>
-__global__ void __maxnreg__((SpmmTune<TF, VW, L, R, AGG>::regs))
-    spmm_kernel(const SparseArgs a, const void *__restrict__ A, const int64_t lda,
-                float *__restrict__ O, const int64_t ldo) {
+__device__ __forceinline__ void spmm_body(const SparseArgs &a, const void *__restrict__ A,
+                                          const int64_t lda, float *__restrict__ O,
+                                          const int64_t ldo, const int64_t bid) {
   constexpr int ES = TF::bytes;
   constexpr int Lg = L;
   constexpr int G = 32 / Lg;
@@ -136,7 +138,7 @@ __global__ void __maxnreg__((SpmmTune<TF, VW, L, R, AGG>::regs))
   const int g = lane / Lg;
   const int l = lane & (Lg - 1);
   const int64_t item =
-      a.c_begin * a.slices + ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * G + g;
+      a.c_begin * a.slices + (bid * (blockDim.x >> 5) + (threadIdx.x >> 5)) * G + g;
   const bool item_ok = item < a.c_end * a.slices;
   if (!__any_sync(kFull, item_ok)) return;  // warp-uniform exit
 
@@ -213,7 +215,7 @@ __global__ void __maxnreg__((SpmmTune<TF, VW, L, R, AGG>::regs))
   Tiles tiles;
   {
     const int64_t item0 =
-        a.c_begin * a.slices + ((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * G;
+        a.c_begin * a.slices + (bid * (blockDim.x >> 5) + (threadIdx.x >> 5)) * G;
     tiles.init(gnn_smem + (threadIdx.x >> 5) * Tiles::WARP_WORDS, lane, a.row_ind, a.col_ind,
                a.val, [&](int gg, int64_t &cs_, int &n_) {
                  const int64_t it = item0 + gg;
@@ -328,6 +330,13 @@ __global__ void __maxnreg__((SpmmTune<TF, VW, L, R, AGG>::regs))
   if (item_ok && c == a.num_chunks - 1) {
     for (int64_t r = (int64_t)rl + 1; r < a.row_base + a.M; ++r) zero_row(r);
   }
+}
+
+template <typename TF, int VW, int L, int R, int VWS, int AGG>
+__global__ void __maxnreg__((SpmmTune<TF, VW, L, R, AGG>::regs))
+    spmm_kernel(const SparseArgs a, const void *__restrict__ A, const int64_t lda,
+                float *__restrict__ O, const int64_t ldo) {
+  spmm_body<TF, VW, L, R, VWS, AGG>(a, A, lda, O, ldo, blockIdx.x);
 }
 
 using SpmmFn = void (*)(const SparseArgs, const void *__restrict__, const int64_t,
