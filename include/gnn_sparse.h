@@ -158,7 +158,9 @@ GNN_API void gnn_plan_destroy(gnn_plan_t plan);
  * A, O must be 4*vw_feat-byte aligned and lda, ldo multiples of vw_feat, else
  * GNN_ERR_UNSUPPORTED (re-plan with force_vw).  A and O must not overlap.
  * Rows split across chunks are combined with vector atomic adds, so the fp32
- * summation order of such rows is not deterministic (tolerance: DESIGN.md). */
+ * summation order of such rows is not deterministic (tolerance: DESIGN.md), and the
+ * vector atomics flush SUBNORMAL partial sums to zero: for data whose partial sums can be
+ * subnormal use a deterministic plan (plain fp32 adds, exact for subnormals). */
 GNN_API gnn_status_t gnn_spmm(gnn_plan_t plan, const gnn_graph_t *graph, const float *A,
                               int64_t lda, float *O, int64_t ldo, gnn_stream_t stream);
 
@@ -374,6 +376,19 @@ GNN_API gnn_status_t gnn_split_col_blocks(const int32_t *row_ind_host, const int
                                           int64_t blk, int32_t *row_ind_out,
                                           int32_t *col_ind_out, float *val_out,
                                           int64_t *bounds);
+
+/* --------------------------------------------------------- autograd helpers -- */
+/* dst[i] = src[idx[i]] for i in [0, n) (device arrays): the edge values of S^T in the
+ * transposed order (idx = gnn_transpose's edge_perm) for the backward dX = S^T dO with
+ * trainable edge values. */
+GNN_API gnn_status_t gnn_gather_f32(const float *src, const int32_t *idx, int64_t n, float *dst,
+                                    gnn_stream_t stream);
+/* Y[r][0:K] = X[r][0:K] / max(1, row_ptr[r+1] - row_ptr[r]) for r in [0, M) (device; Y may
+ * be X): the backward of the mean aggregator, dX = S^T (dO / deg) (Eq. 1 with (+) = mean,
+ * P:23-31; rows without nonzeros carry no gradient). */
+GNN_API gnn_status_t gnn_scale_rows_inv_degree(const int32_t *row_ptr, int64_t M, int32_t K,
+                                               const float *X, int64_t ldx, float *Y,
+                                               int64_t ldy, gnn_stream_t stream);
 
 /* ------------------------------------------------------------- helpers ---- */
 /* Decode CSR offsets into the hybrid format's RowInd (Fig. 2d):

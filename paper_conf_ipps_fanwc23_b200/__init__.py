@@ -72,7 +72,7 @@ EXPORTS = ["gnn_plan_workspace_bytes", "gnn_plan_create", "gnn_plan_info", "gnn_
            "gnn_plan_destroy", "gnn_spmm", "gnn_sddmm", "gnn_spmm_bf16", "gnn_sddmm_bf16",
            "gnn_spmm_ex", "gnn_spmm_extremum_backward", "gnn_plan_spmm_sddmm",
            "gnn_transpose_workspace_bytes",
-           "gnn_transpose",
+           "gnn_transpose", "gnn_gather_f32", "gnn_scale_rows_inv_degree",
            "gnn_shard_rows", "gnn_shard_edges", "gnn_split_col_blocks",
            "gnn_reorder_gcr", "gnn_permute_graph", "gnn_permute_rows",
            "gnn_probe_gather", "gnn_probe_gather_chunked", "gnn_run_host_workspace_bytes", "gnn_run_host",
@@ -113,6 +113,9 @@ def lib():
         L.gnn_transpose_workspace_bytes.argtypes = [i64]
         L.gnn_transpose_workspace_bytes.restype = ctypes.c_size_t
         L.gnn_transpose.argtypes = [P(_Graph), vp, ctypes.c_size_t, vp, vp, vp, vp, vp, vp]
+    if hasattr(L, "gnn_gather_f32"):
+        L.gnn_gather_f32.argtypes = [vp, vp, i64, vp, vp]
+        L.gnn_scale_rows_inv_degree.argtypes = [vp, i64, i32, vp, i64, vp, i64, vp]
     L.gnn_shard_rows.argtypes = [vp, i64, i32, vp]
     L.gnn_shard_edges.argtypes = [i64, i32, vp]
     if hasattr(L, "gnn_run_host"):
@@ -145,7 +148,8 @@ def lib():
               "gnn_reorder_gcr", "gnn_permute_graph", "gnn_permute_rows", "gnn_probe_gather",
               "gnn_probe_gather_chunked",
               "gnn_spmm_bf16", "gnn_sddmm_bf16", "gnn_spmm_ex", "gnn_transpose",
-              "gnn_split_col_blocks", "gnn_run_host", "gnn_run_host_multi"):
+              "gnn_split_col_blocks", "gnn_run_host", "gnn_run_host_multi", "gnn_gather_f32",
+              "gnn_scale_rows_inv_degree"):
         if hasattr(L, f):
             getattr(L, f).restype = st
     _lib = L
@@ -425,6 +429,31 @@ def transpose(graph: DeviceGraph, stream=None):
                            _ptr(vt), _ptr(perm), _stream(stream)))
     gt = DeviceGraph(graph.N, graph.M, ri, ci, vt if graph.val is not None else None, rp, 0)
     return gt, perm
+
+
+def gather_values(src: torch.Tensor, idx: torch.Tensor, stream=None) -> torch.Tensor:
+    """gnn_gather_f32: src[idx] on the device (fp32 values, int32 indices)."""
+    if (src.dtype != torch.float32 or not src.is_cuda or not src.is_contiguous()
+            or idx.dtype != torch.int32 or not idx.is_contiguous() or idx.device != src.device):
+        raise ValueError("gather_values: contiguous fp32 src and int32 idx on one CUDA device")
+    out = torch.empty(idx.numel(), dtype=torch.float32, device=src.device)
+    _check(lib().gnn_gather_f32(_ptr(src), _ptr(idx), idx.numel(), _ptr(out), _stream(stream)))
+    return out
+
+
+def scale_rows_inv_degree(graph: DeviceGraph, X: torch.Tensor, out: torch.Tensor | None = None,
+                          stream=None) -> torch.Tensor:
+    """gnn_scale_rows_inv_degree: X[r] / max(1, deg r) (the mean aggregator's backward)."""
+    if graph.row_ptr is None:
+        raise ValueError("scale_rows_inv_degree needs the graph's row_ptr")
+    _dense(X, "X", rows=graph.M, device=graph.row_ind.device)
+    if out is None:
+        out = torch.empty_like(X)
+    _dense(out, "out", rows=graph.M, cols=X.shape[1], device=X.device)
+    _check(lib().gnn_scale_rows_inv_degree(_ptr(graph.row_ptr), graph.M, X.shape[1], _ptr(X),
+                                           X.stride(0), _ptr(out), out.stride(0),
+                                           _stream(stream)))
+    return out
 
 
 def sddmm(p: Plan, graph: DeviceGraph, A1: torch.Tensor, A2T: torch.Tensor,

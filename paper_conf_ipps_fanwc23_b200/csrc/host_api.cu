@@ -420,7 +420,12 @@ gnn_status_t side_stream(SideStream **out) {
       cudaEventDestroy(t.join);
       t.s = nullptr;
     }
-    e = cudaStreamCreateWithFlags(&t.s, cudaStreamNonBlocking);
+    // GNN_STEP_SIDE_PRIO=low: the SDDMM's side stream below the caller's (experiment)
+    const char *pr = getenv("GNN_STEP_SIDE_PRIO");
+    int lo = 0, hi = 0;
+    cudaDeviceGetStreamPriorityRange(&lo, &hi);
+    e = cudaStreamCreateWithPriority(&t.s, cudaStreamNonBlocking,
+                                     (pr && pr[0] == 'l') ? lo : 0);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&t.fork, cudaEventDisableTiming);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&t.join, cudaEventDisableTiming);
     if (e != cudaSuccess) return cuda_fail(e, "gnn_plan_spmm_sddmm side stream");
@@ -461,6 +466,16 @@ GNN_API gnn_status_t gnn_plan_spmm_sddmm(const gnn_graph_t *g, int32_t K,
   Plan *p = reinterpret_cast<Plan *>(plan);
   p->inline_plan = !det;
   cudaStream_t s = (cudaStream_t)stream;
+  // both outputs: one fused launch where the shape has an instance and K <= 64 (measured:
+  // C3 K=32 0.0402 -> 0.0366 ms, but K=128 0.0682 -> 0.0736: the fused kernel runs the
+  // SpMM half at SDDMM's 128-register budget; r02_s8).  GNN_STEP_FUSED=0 / 1: never /
+  // whenever an instance exists.
+  const char *fz = getenv("GNN_STEP_FUSED");
+  const bool fuse = fz ? fz[0] == '1' : K <= 64;
+  if (O && out && !det && fuse) {
+    const gnn_status_t st = launch_step_fused(p, g, X, ldx, O, ldo, out, stream);
+    if (st != GNN_ERR_UNSUPPORTED) return st;
+  }
   SideStream *side = nullptr;
   const bool fork = O && out && g->nnz > 0;
   if (fork) {
@@ -470,12 +485,20 @@ GNN_API gnn_status_t gnn_plan_spmm_sddmm(const gnn_graph_t *g, int32_t K,
     if (e != cudaSuccess) return cuda_fail(e, "gnn_plan_spmm_sddmm fork");
   }
   gnn_status_t st = GNN_OK;
-  if (out)  // A1 = the graph's own rows of X (row_base), A2T = all of X
-    st = launch_sddmm(p, g, X ? X + g->row_base * ldx : nullptr, ldx, X, ldx, out,
-                      fork ? side->s : s, GNN_F32, "gnn_plan_spmm_sddmm sddmm", -1, 0);
-  if (st == GNN_OK && O)
-    st = launch_spmm(p, g, X, ldx, O, ldo, s, GNN_F32, GNN_AGG_SUM, 0,
-                     "gnn_plan_spmm_sddmm spmm", -1, 0);
+  // GNN_STEP_SPMM_FIRST=1 enqueues the SpMM (the longer kernel) before the SDDMM (experiment)
+  const char *sf = getenv("GNN_STEP_SPMM_FIRST");
+  const bool spmm_first = sf && sf[0] == '1';
+  auto run_sddmm = [&]() {  // A1 = the graph's own rows of X (row_base), A2T = all of X
+    return launch_sddmm(p, g, X ? X + g->row_base * ldx : nullptr, ldx, X, ldx, out,
+                        fork ? side->s : s, GNN_F32, "gnn_plan_spmm_sddmm sddmm", -1, 0);
+  };
+  auto run_spmm = [&]() {
+    return launch_spmm(p, g, X, ldx, O, ldo, s, GNN_F32, GNN_AGG_SUM, 0,
+                       "gnn_plan_spmm_sddmm spmm", -1, 0);
+  };
+  if (spmm_first && O) st = run_spmm();
+  if (st == GNN_OK && out) st = run_sddmm();
+  if (st == GNN_OK && O && !spmm_first) st = run_spmm();
   if (fork) {  // join even after an error, so `stream` covers everything enqueued
     cudaError_t e = cudaEventRecord(side->join, side->s);
     if (e == cudaSuccess) e = cudaStreamWaitEvent(s, side->join, 0);

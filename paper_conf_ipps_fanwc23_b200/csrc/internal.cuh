@@ -105,6 +105,11 @@ gnn_status_t plan_create(const gnn_graph_t *g, int32_t K, const gnn_plan_opts_t 
                          void *workspace, size_t ws_bytes, gnn_stream_t stream, gnn_plan_t *out,
                          bool launch);
 gnn_status_t launch_plan_range(const Plan *p, gnn_stream_t stream, int64_t c0, int64_t c1);
+// The one-call step as one launch (step_fused.cu); GNN_ERR_UNSUPPORTED = no fused instance
+// for this shape (nothing launched).
+gnn_status_t launch_step_fused(const Plan *p, const gnn_graph_t *g, const float *X,
+                               int64_t ldx, float *O, int64_t ldo, float *out,
+                               gnn_stream_t stream);
 gnn_status_t launch_sddmm(const Plan *p, const gnn_graph_t *g, const void *A1, int64_t lda1,
                           const void *A2T, int64_t lda2, float *out, gnn_stream_t stream,
                           int dtype, const char *who, int64_t c0, int64_t c1);

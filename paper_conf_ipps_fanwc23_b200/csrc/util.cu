@@ -101,6 +101,28 @@ __global__ void permute_rows_kernel(const float *__restrict__ X, int64_t ldx, in
   }
 }
 
+// dst[i] = src[idx[i]] (grid-stride, coalesced over i)
+__global__ void gather_f32_kernel(const float *__restrict__ src, const int32_t *__restrict__ idx,
+                                  int64_t n, float *__restrict__ dst) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride)
+    dst[i] = src[idx[i]];
+}
+
+// Y[r][:K] = X[r][:K] / max(1, row_ptr[r+1] - row_ptr[r]); one warp per row
+__global__ void scale_rows_inv_degree_kernel(const int32_t *__restrict__ row_ptr, int64_t M,
+                                             int32_t K, const float *__restrict__ X,
+                                             int64_t ldx, float *__restrict__ Y, int64_t ldy) {
+  const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t r = warp; r < M; r += nwarps) {
+    const int32_t cnt = row_ptr[r + 1] - row_ptr[r];
+    const float s = 1.0f / (float)(cnt > 1 ? cnt : 1);
+    for (int k = lane; k < K; k += 32) Y[r * ldy + k] = X[r * ldx + k] * s;
+  }
+}
+
 }  // namespace gnn
 
 using namespace gnn;
@@ -207,6 +229,36 @@ GNN_API gnn_status_t gnn_permute_rows(const float *X, int64_t ldx, int64_t n, in
                                                                          ldy);
   cudaError_t e = cudaGetLastError();
   return e == cudaSuccess ? GNN_OK : cuda_fail(e, "permute_rows launch");
+}
+
+GNN_API gnn_status_t gnn_gather_f32(const float *src, const int32_t *idx, int64_t n, float *dst,
+                                    gnn_stream_t stream) {
+  if (n < 0 || (n > 0 && (!src || !idx || !dst)))
+    return fail(GNN_ERR_INVALID_ARG, "gnn_gather_f32: bad arguments");
+  if (n == 0) return GNN_OK;
+  DeviceInfo d;
+  if (gnn_status_t st = device_info(&d)) return st;
+  int64_t blocks = (n + 255) / 256;
+  if (blocks > (int64_t)d.num_sms * 16) blocks = (int64_t)d.num_sms * 16;
+  gather_f32_kernel<<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>(src, idx, n, dst);
+  cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? GNN_OK : cuda_fail(e, "gather launch");
+}
+
+GNN_API gnn_status_t gnn_scale_rows_inv_degree(const int32_t *row_ptr, int64_t M, int32_t K,
+                                               const float *X, int64_t ldx, float *Y,
+                                               int64_t ldy, gnn_stream_t stream) {
+  if (M < 0 || K < 1 || (M > 0 && (!row_ptr || !X || !Y || ldx < K || ldy < K)))
+    return fail(GNN_ERR_INVALID_ARG, "gnn_scale_rows_inv_degree: bad arguments");
+  if (M == 0) return GNN_OK;
+  DeviceInfo d;
+  if (gnn_status_t st = device_info(&d)) return st;
+  int64_t blocks = (M * 32 + 255) / 256;
+  if (blocks > (int64_t)d.num_sms * 16) blocks = (int64_t)d.num_sms * 16;
+  scale_rows_inv_degree_kernel<<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>(
+      row_ptr, M, K, X, ldx, Y, ldy);
+  cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? GNN_OK : cuda_fail(e, "scale rows launch");
 }
 
 GNN_API gnn_status_t gnn_validate(const gnn_graph_t *g, gnn_stream_t stream) {

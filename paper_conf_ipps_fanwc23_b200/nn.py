@@ -20,7 +20,8 @@ import math
 
 import torch
 
-from . import DeviceGraph, plan, sddmm, spmm, spmm_extremum_backward, transpose
+from . import (DeviceGraph, gather_values, plan, scale_rows_inv_degree, sddmm, spmm,
+               spmm_extremum_backward, transpose)
 
 
 class SparseOp:
@@ -31,7 +32,6 @@ class SparseOp:
         self.g = graph
         self.gt, self.perm = (transpose(graph) if need_transpose else (None, None))
         self._plans = {}
-        self._cnt = None
 
     def plan_for(self, which: str, K: int, dtype=torch.float32):
         key = (which, K, dtype)
@@ -41,19 +41,10 @@ class SparseOp:
             self._plans[key] = p
         return p
 
-    def counts(self) -> torch.Tensor:
-        """Nonzeros per row (mean aggregation), from row_ptr."""
-        if self._cnt is None:
-            rp = self.g.row_ptr
-            if rp is None:
-                raise ValueError("mean aggregation needs the graph's row_ptr")
-            self._cnt = (rp[1:] - rp[:-1]).to(torch.float32)
-        return self._cnt
-
     def with_val(self, val, transposed=False) -> DeviceGraph:
         g = self.gt if transposed else self.g
-        if val is not None and transposed:
-            val = val[self.perm.long()].contiguous()
+        if val is not None and transposed:  # S^T's values in transposed order (edge_perm)
+            val = gather_values(val.contiguous(), self.perm)
         return DeviceGraph(g.M, g.N, g.row_ind, g.col_ind, val, g.row_ptr, g.row_base)
 
 
@@ -81,9 +72,8 @@ class _SpMMFunction(torch.autograd.Function):
             dval = torch.zeros(op.g.nnz, dtype=torch.float32, device=X.device) if need_v else None
             dX, dval = spmm_extremum_backward(g, agg, X, O, dO, dval=dval)
             return (dX if ctx.needs_input_grad[0] else None), dval, None, None
-        if agg == "mean":
-            cnt = op.counts()
-            dO = dO / torch.clamp(cnt, min=1.0)[:, None]
+        if agg == "mean":  # dX = S^T (dO / deg): the row scale runs in the library
+            dO = scale_rows_inv_degree(op.g, dO)
         K = dO.shape[1]
         dX = dval = None
         if ctx.needs_input_grad[0]:

@@ -905,20 +905,22 @@ def test_validate_env_switch(monkeypatch):
     gs.plan(dg, 32)
 
 
-@pytest.mark.parametrize("plan_kernel", ["0", "1"])
-def test_one_call_step_inline_plan_matches_oracle(monkeypatch, plan_kernel):
-    """gnn_plan_spmm_sddmm with the boundary table recomputed inside the kernels (and the
-    PDL SpMM) against the oracle, on graphs with hubs split over many chunks, empty rows
-    and a row shard; the plan-kernel path (GNN_STEP_PLAN_KERNEL=1) likewise."""
-    monkeypatch.setenv("GNN_STEP_PLAN_KERNEL", plan_kernel)
+@pytest.mark.parametrize("mode", ["fused", "two_kernels", "plan_kernel"])
+def test_one_call_step_inline_plan_matches_oracle(monkeypatch, mode):
+    """gnn_plan_spmm_sddmm against the oracle on graphs with hubs split over many chunks
+    and empty rows, in its three forms: one fused SpMM+SDDMM launch (default), the two
+    kernels on two streams (GNN_STEP_FUSED=0), both with the boundary table recomputed in
+    the kernels and a PDL SpMM, and the plan-kernel path (GNN_STEP_PLAN_KERNEL=1)."""
+    monkeypatch.setenv("GNN_STEP_FUSED", "0" if mode == "two_kernels" else "1")
+    monkeypatch.setenv("GNN_STEP_PLAN_KERNEL", "1" if mode == "plan_kernel" else "0")
     rng = np.random.default_rng(77)
-    for t in range(4):
+    for t in range(6):
         M = int(rng.integers(100, 3000))
         nnz = int(rng.integers(1000, 60000))
         rows = np.sort(rng.integers(0, M, nnz))
         rows[: nnz // 4] = rows[0]  # a hub
         g = gen.from_coo(M, M, rows, rng.integers(0, M, nnz), gen.uniform_values(80 + t, nnz))
-        K = int(rng.choice([32, 64, 128, 256]))
+        K = int(rng.choice([32, 64, 128, 256])) if t else 24  # (24: no fused instance)
         dg = upload(g)
         X = torch.from_numpy(_x(90 + t, g.N, K)).to(DEV)
         O = torch.full((g.M, K), float("nan"), device=DEV)
@@ -930,3 +932,32 @@ def test_one_call_step_inline_plan_matches_oracle(monkeypatch, plan_kernel):
         assert_within(O.cpu().numpy(), ref, T, what=f"one-call spmm t={t}")
         r2, T2 = oracle.sddmm(g.row_ind, g.col_ind, g.val, Xh, Xh)
         assert_within(E.cpu().numpy(), r2, T2, what=f"one-call sddmm t={t}")
+
+
+def test_subnormal_partials_atomic_ftz_vs_deterministic():
+    """Documented limit (reading 28, device.cuh): the vector atomics that combine a
+    row split across chunks (REDG.E.ADD.F32x4) flush subnormal operands to zero.  With
+    subnormal features a split row may lose its partial sums on the default plan, while
+    rows owned by one chunk are exact; a deterministic plan (split rows summed in chunk
+    order by plain fp32 adds, no atomics) keeps them: exact here (sums of subnormals are
+    exact until they leave the subnormal range)."""
+    M = N = 64
+    rows = np.r_[np.zeros(2000, np.int64), np.repeat(np.arange(1, M), 3)]
+    rng = np.random.default_rng(5)
+    g = gen.from_coo(M, N, rows, rng.integers(0, N, rows.size), np.ones(rows.size, np.float32))
+    K = 32
+    X = (rng.integers(1, 4, (N, K)).astype(np.float64) * 2.0 ** -140).astype(np.float32)
+    assert (X != 0).all() and (np.abs(X) < np.finfo(np.float32).tiny).all()  # subnormal
+    ref, T = oracle.spmm(g.row_ind, g.col_ind, g.val, X, M=g.M)
+    dg = upload(g)
+    Xd = torch.from_numpy(X).to(DEV)
+    det = gs.spmm(gs.plan(dg, K, deterministic=True), dg, Xd).cpu().numpy()
+    assert np.array_equal(det.astype(np.float64), ref)
+    p = gs.plan(dg, K)
+    C = p.info()["chunk"]
+    first, last = g.row_ptr[:-1] // C, (g.row_ptr[1:] - 1) // C
+    split = first != last                                     # rows spanning chunks
+    assert split[0]
+    O = gs.spmm(p, dg, Xd).cpu().numpy().astype(np.float64)
+    assert np.array_equal(O[~split], ref[~split])             # rows owned by one chunk
+    assert (O[split] >= 0).all() and (O[split] <= ref[split]).all()  # flushed partials

@@ -1,7 +1,8 @@
-"""C3 (sampled subgraphs, K = 128) one-call step A/B: the inline-plan path of
-gnn_plan_spmm_sddmm (no plan kernel, PDL SpMM) against the plan-kernel path
-(GNN_STEP_PLAN_KERNEL=1), alternated A/B/A/B on the same resident subgraphs, L2 flushed
-between steps, CUDA events around each step.  Prints one JSON line.
+"""C3 (sampled subgraphs, K = 128) one-call step A/B/C: gnn_plan_spmm_sddmm as one fused
+SpMM+SDDMM launch (default), as two kernels on two streams with the boundary table
+recomputed in-kernel (GNN_STEP_FUSED=0), and with the plan kernel (GNN_STEP_PLAN_KERNEL=1),
+alternated on the same resident subgraphs, L2 flushed between steps, CUDA events around
+each step.  Prints one JSON line.
 
     python tools/c3_ab.py [--graphs 20] [--steps 2000] [--rounds 3]
 """
@@ -39,10 +40,15 @@ def main():
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
     stream = torch.cuda.current_stream()
     run = gs.StepRunner(dev)
-    res = {"inline": [], "plan_kernel": []}
+    # (GNN_STEP_FUSED, GNN_STEP_PLAN_KERNEL, GNN_STEP_SPMM_FIRST)
+    modes = {"fused": ("1", "0", "0"), "two_kernels": ("0", "0", "0"),
+             "two_kernels_spmm_first": ("0", "0", "1"), "plan_kernel": ("0", "1", "0")}
+    res = {m: [] for m in modes}
     for rnd in range(a.rounds):
-        for mode in ("inline", "plan_kernel"):
-            os.environ["GNN_STEP_PLAN_KERNEL"] = "1" if mode == "plan_kernel" else "0"
+        for mode, (fz, pk, sf) in modes.items():
+            os.environ["GNN_STEP_FUSED"] = fz
+            os.environ["GNN_STEP_PLAN_KERNEL"] = pk
+            os.environ["GNN_STEP_SPMM_FIRST"] = sf
             for s in subs:
                 run(*s)
             torch.cuda.synchronize()
@@ -56,9 +62,10 @@ def main():
             torch.cuda.synchronize()
             res[mode].append(statistics.mean(x.elapsed_time(y) for x, y in ev))
     os.environ.pop("GNN_STEP_PLAN_KERNEL", None)
+    os.environ.pop("GNN_STEP_FUSED", None)
+    os.environ.pop("GNN_STEP_SPMM_FIRST", None)
     print(json.dumps({"K": K, "graphs": a.graphs, "steps": a.steps,
-                      "inline_ms": [round(x, 4) for x in res["inline"]],
-                      "plan_kernel_ms": [round(x, 4) for x in res["plan_kernel"]]}))
+                      **{f"{m}_ms": [round(x, 4) for x in v] for m, v in res.items()}}))
 
 
 if __name__ == "__main__":
