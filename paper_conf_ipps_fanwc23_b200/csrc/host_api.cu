@@ -466,12 +466,12 @@ GNN_API gnn_status_t gnn_plan_spmm_sddmm(const gnn_graph_t *g, int32_t K,
   Plan *p = reinterpret_cast<Plan *>(plan);
   p->inline_plan = !det;
   cudaStream_t s = (cudaStream_t)stream;
-  // both outputs: one fused launch where the shape has an instance and K <= 64 (measured:
-  // C3 K=32 0.0402 -> 0.0366 ms, but K=128 0.0682 -> 0.0736: the fused kernel runs the
-  // SpMM half at SDDMM's 128-register budget; r02_s8).  GNN_STEP_FUSED=0 / 1: never /
-  // whenever an instance exists.
+  // both outputs: one fused launch where the shape has an instance and K <= 32 (measured on
+  // 20 C3 subgraphs: K=32 0.0402 -> 0.0367 ms, but K=64 0.0489 -> 0.0523 and K=128 0.0684
+  // -> 0.0738: the fused kernel runs the SpMM half at SDDMM's 128-register budget;
+  // profiles/r02_s9_c3_fused_ab.txt).  GNN_STEP_FUSED=0 / 1: never / whenever possible.
   const char *fz = getenv("GNN_STEP_FUSED");
-  const bool fuse = fz ? fz[0] == '1' : K <= 64;
+  const bool fuse = fz ? fz[0] == '1' : K <= 32;
   if (O && out && !det && fuse) {
     const gnn_status_t st = launch_step_fused(p, g, X, ldx, O, ldo, out, stream);
     if (st != GNN_ERR_UNSUPPORTED) return st;
