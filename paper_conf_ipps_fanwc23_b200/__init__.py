@@ -367,12 +367,16 @@ def spmm_extremum_backward(graph: DeviceGraph, agg: str, A: torch.Tensor, O: tor
     Accumulates into dA (N x K) / dval (nnz) when given, else returns fresh zeroed ones."""
     if agg not in ("max", "min"):
         raise ValueError("agg must be 'max' or 'min'")
-    for t, n in ((A, "A"), (O, "O"), (dO, "dO")):
-        _dense(t, n)
-    K = A.shape[1]
+    dev = graph.row_ind.device
+    K = A.shape[1] if torch.is_tensor(A) and A.dim() == 2 else 0
+    _dense(A, "A", rows=graph.N if graph.nnz else 0, device=dev)
+    for t, n in ((O, "O"), (dO, "dO")):
+        _dense(t, n, rows=graph.M, cols=K, device=dev)
     if dA is None:
         dA = torch.zeros((graph.N, K), dtype=torch.float32, device=A.device)
-    _dense(dA, "dA")
+    _dense(dA, "dA", rows=graph.N, cols=K, device=dev)
+    if dval is not None:
+        _vec_out(dval, "dval", graph.nnz, dev)
     g = graph.desc()
     _check(lib().gnn_spmm_extremum_backward(ctypes.byref(g), AGG[agg], K, _ptr(A), A.stride(0),
                                             _ptr(O), O.stride(0), _ptr(dO), dO.stride(0),
@@ -561,7 +565,10 @@ def permute_rows(X: torch.Tensor, perm: torch.Tensor, out: torch.Tensor | None =
     _dense(X, "X")
     if out is None:
         out = torch.empty_like(X)
+    _dense(out, "out", rows=X.shape[0], cols=X.shape[1], device=X.device)
     perm = perm.to(device=X.device, dtype=torch.int32).contiguous()
+    if perm.numel() != X.shape[0]:
+        raise ValueError("permute_rows: perm must have one entry per row of X")
     _check(lib().gnn_permute_rows(_ptr(X), X.stride(0), X.shape[0], X.shape[1], _ptr(perm),
                                   _ptr(out), out.stride(0), _stream(stream)))
     return out
@@ -625,11 +632,16 @@ class HostRunner:
                            self.row_base)
         return self
 
+    def _check_host(self, X_host, K, O_host, out_host):
+        for t, n in ((X_host, self.N * K), (O_host, self.M * K), (out_host, self.nnz)):
+            if t is not None and (t.is_cuda or not t.is_contiguous() or t.dtype != torch.float32
+                                  or t.numel() < n):
+                raise ValueError("host buffers must be contiguous fp32 CPU tensors of "
+                                 "N*K (X), M*K (O) and nnz (out) elements")
+
     def run(self, X_host: torch.Tensor, K: int, O_host=None, out_host=None, upload_graph=True,
             stream=None):
-        for t in (X_host, O_host, out_host):
-            if t is not None and (t.is_cuda or not t.is_contiguous() or t.dtype != torch.float32):
-                raise ValueError("host buffers must be contiguous fp32 CPU tensors")
+        self._check_host(X_host, K, O_host, out_host)
         _check(lib().gnn_run_host(ctypes.byref(self.desc), int(upload_graph), _ptr(X_host), K,
                                   _ptr(O_host), _ptr(out_host), ctypes.byref(self.opts),
                                   _ptr(self.ws), self.ws_bytes, _stream(stream)))
@@ -641,9 +653,10 @@ class HostRunner:
         n = len(Ks)
         O_hosts = O_hosts or [None] * n
         out_hosts = out_hosts or [None] * n
-        for t in list(X_hosts) + list(O_hosts) + list(out_hosts):
-            if t is not None and (t.is_cuda or not t.is_contiguous() or t.dtype != torch.float32):
-                raise ValueError("host buffers must be contiguous fp32 CPU tensors")
+        if not (len(X_hosts) == len(O_hosts) == len(out_hosts) == n):
+            raise ValueError("run_multi: one X / O / out entry per width")
+        for X_host, K, O_host, out_host in zip(X_hosts, Ks, O_hosts, out_hosts):
+            self._check_host(X_host, K, O_host, out_host)
         vp = ctypes.c_void_p
         karr = (ctypes.c_int32 * n)(*Ks)
         xa = (vp * n)(*[_ptr(t) for t in X_hosts])
