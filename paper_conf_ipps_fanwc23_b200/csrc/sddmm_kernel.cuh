@@ -13,10 +13,12 @@ namespace gnn {
 // SDDMM spreads them over Lg = V / Rsd lanes with Rsd vectors per lane, so each dot
 // product is reduced over Lg lanes and 32 / Lg nonzeros are in flight per warp step;
 // U = nonzeros per batch per group, U * Rsd = 8 feature vectors in flight per lane.
-// Measured on the GCR-reordered C4 (profiles/r01_sweep8.txt): Rsd = 2 from V = 8 on
-// (K=64: 2.07 -> 1.94 ms, K=128: 4.82 -> 3.61 ms, K=256: 8.85 -> 7.05 ms), 1 below.
+// Measured on the GCR-reordered C4: Rsd = 2 from V = 16 on (round 1, r01_sweep8: K=128
+// 4.82 -> 3.61 ms, K=256 8.85 -> 7.05 ms); at V = 8 (K = 64) round 1 also preferred 2
+// (2.07 -> 1.94 ms), the round-2 kernels prefer 1 (8 lanes x 1 vector, 8 in flight:
+// 1.652 -> 1.544 ms, profiles/r02_s13_sweep_c4_sddmm_r1_k64.txt).
 #ifndef GNN_SDDMM_R2_FROM
-#define GNN_SDDMM_R2_FROM 8  // smallest V that uses Rsd = 2
+#define GNN_SDDMM_R2_FROM 16  // smallest V that uses Rsd = 2
 #endif
 #ifndef GNN_SDDMM_UR
 #define GNN_SDDMM_UR 8       // U * Rsd: feature vectors in flight per lane
