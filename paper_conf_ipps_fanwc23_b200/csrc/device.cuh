@@ -81,15 +81,6 @@ __device__ __forceinline__ void ld_feat<8>(const float *p, float (&x)[8]) {
 #endif
 }
 
-// 16-byte global -> shared copy of FEATURE data (no L2 hint; .cg: L2 only, no L1 fill);
-// src_bytes < 16 zero-fills the rest.
-__device__ __forceinline__ void cp_async_feat16(void *smem_dst, const void *gsrc, int src_bytes) {
-  const uint32_t d = (uint32_t)__cvta_generic_to_shared(smem_dst);
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(d), "l"(gsrc),
-               "r"(src_bytes)
-               : "memory");
-}
-
 // ------------------------------------------------------------- outputs ----
 #ifndef GNN_OUT_STREAMING
 #define GNN_OUT_STREAMING 0  // outputs stored with the streaming (.cs, evict-first) policy
@@ -232,22 +223,6 @@ struct FeatVec<F32, VW> {
     for (int v = 0; v < VW; ++v) r[v] = 0.f;
   }
   __device__ __forceinline__ float get(int v) const { return r[v]; }
-  // staged gathers (SpmmTune::stage): the row slice was copied into shared memory by
-  // cp.async; issue / read back this lane's VW elements
-  __device__ __forceinline__ void stage_issue(float *sm, const char *p) const {
-#pragma unroll
-    for (int h = 0; h < VW; h += 4) cp_async_feat16(sm + h, p + 4 * h, 16);
-  }
-  __device__ __forceinline__ void stage_read(const float *sm) {
-#pragma unroll
-    for (int h = 0; h < VW; h += 4) {
-      const float4 t = *reinterpret_cast<const float4 *>(sm + h);
-      r[h] = t.x;
-      r[h + 1] = t.y;
-      r[h + 2] = t.z;
-      r[h + 3] = t.w;
-    }
-  }
 };
 
 template <int VW>

@@ -136,9 +136,7 @@ int spmm_active_blocks_per_sm(int dtype, int vw, int lanes, int vecs, int wpb) {
   SpmmFn f = pick_spmm(dtype, vw, lanes, vecs, 1);
   if (!f) return 0;
   // the plan's vw_sparse is not known yet: size the tiles for the widest (4)
-  const size_t smem = (size_t)wpb * (spmm_tile_bytes_per_warp(lanes, 4) +
-                                     spmm_stage_bytes_per_warp(dtype == GNN_BF16 ? 2 : 4, vw,
-                                                               lanes, vecs, kAggSum));
+  const size_t smem = (size_t)wpb * spmm_tile_bytes_per_warp(lanes, 4);
   // only ever raise the per-function limit above the 48 KB default (a smaller value would
   // make later launches with more warps per block fail); launches re-raise it as needed
   if (smem > 48 * 1024 &&
@@ -301,9 +299,7 @@ gnn_status_t launch_spmm(const Plan *p, const gnn_graph_t *g, const void *A, int
       default: spmm_prezero_kernel<8><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, init); break;
     }
   }
-  const size_t smem = (size_t)in.warps_per_block * (spmm_tile_bytes_per_warp(lanes, vws) +
-                                                    spmm_stage_bytes_per_warp(ES, VW, lanes,
-                                                                              vecs, agg));
+  const size_t smem = (size_t)in.warps_per_block * spmm_tile_bytes_per_warp(lanes, vws);
   if (smem > 48 * 1024) {
     cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return cuda_fail(e, "gnn_spmm smem attribute");

@@ -37,30 +37,7 @@ struct SpmmTune {
 #else
   static constexpr int depth = R == 2 ? GNN_SPMM_DEPTH_R2 : ((lean || (wide && L <= 2)) ? 4 : 8);
 #endif
-  // > 0: nonzeros per batch whose feature rows are staged through shared memory by
-  // cp.async instead of loaded into registers (experiment, GNN_SPMM_SMEM_STAGE)
-#if defined(GNN_SPMM_SMEM_STAGE)
-  static constexpr int stage = (lean && f32) ? GNN_SPMM_SMEM_STAGE : 0;
-#else
-  static constexpr int stage = 0;
-#endif
-#if defined(GNN_SPMM_STAGE_REGS) && !defined(GNN_SPMM_REGS)
-  static constexpr int kregs = stage ? GNN_SPMM_STAGE_REGS : regs;
-#else
-  static constexpr int kregs = regs;
-#endif
 };
-
-// host mirror: dynamic shared memory per warp of the feature stage (0 when not staged)
-inline int spmm_stage_bytes_per_warp(int es, int vw, int L, int R, int agg) {
-#if defined(GNN_SPMM_SMEM_STAGE)
-  const bool lean = agg == 0 && R == 1 && vw * es == 32 && (es == 4 || L >= 8);
-  return (lean && es == 4) ? GNN_SPMM_SMEM_STAGE * 32 * R * vw * es : 0;
-#else
-  (void)es; (void)vw; (void)L; (void)R; (void)agg;
-  return 0;
-#endif
-}
 
 // host mirror of SpmmTune::depth (feature vectors in flight per lane) for the launcher
 inline int spmm_depth(int es, int vw, int L, int R, int agg) {
@@ -154,10 +131,8 @@ __device__ __forceinline__ void spmm_body(const SparseArgs &a, const void *__res
   using Tiles = TilesFor<L, VWS>;
   constexpr int T = Tiles::T;  // nonzeros per tile per group
   // U nonzeros per batch: FeatDepth vectors in flight per lane, whole sparse vectors
-  using Tune = SpmmTune<TF, VW, L, R, AGG>;
-  constexpr int D = Tune::stage ? Tune::stage : Tune::depth / R;
+  constexpr int D = SpmmTune<TF, VW, L, R, AGG>::depth / R;
   constexpr int U = D > T ? T : (D < VWS ? VWS : D);
-  constexpr bool STAGED = Tune::stage > 0;
   static_assert(T % U == 0 && U % VWS == 0, "tile / prefetch shape");
   const int lane = threadIdx.x & 31;
   const int g = lane / Lg;
@@ -254,12 +229,6 @@ __device__ __forceinline__ void spmm_body(const SparseArgs &a, const void *__res
                cs, n);
   }
   tiles.issue(0, 0, lane);
-  // staged gathers: this lane's [U][R] row slices, after every warp's tile ring
-  float *stg = nullptr;
-  if constexpr (STAGED)
-    stg = reinterpret_cast<float *>(gnn_smem + (blockDim.x >> 5) * Tiles::WARP_WORDS) +
-          ((int64_t)(threadIdx.x >> 5) * U * R * 32 + lane) * VW;
-  auto stage_slot = [&](int u, int r) { return stg + (u * R + r) * 32 * VW; };
 
   const int ntiles = (a.chunk + T - 1) / T;  // warp-uniform trip count
   for (int t = 0; t < ntiles; ++t) {
@@ -297,41 +266,20 @@ __device__ __forceinline__ void spmm_body(const SparseArgs &a, const void *__res
           cj[u] = (uint32_t)s_col[jj + u];
           vj[u] = vi ? s_val[jj + u] : 1.f;
         }
-        if constexpr (STAGED) {
+        FeatVec<TF, VW> x[U][R];
 #pragma unroll
-          for (int u = 0; u < U; ++u) {
-            const char *rowp = Ab + (uint64_t)cj[u] * ldaB;
+        for (int u = 0; u < U; ++u) {
+          const char *rowp = Ab + (uint64_t)cj[u] * ldaB;
 #pragma unroll
-            for (int r = 0; r < R; ++r)
-              if (col_ok[r]) FeatVec<TF, VW>().stage_issue(stage_slot(u, r), rowp + r * Lg * VW * ES);
+          for (int r = 0; r < R; ++r) {
+            if (col_ok[r]) x[u][r].load(rowp + r * Lg * VW * ES);
+            else x[u][r].zero();
           }
-          cp_async_commit();
-          cp_async_wait<0>();
-#pragma unroll
-          for (int u = 0; u < U; ++u)
-#pragma unroll
-            for (int r = 0; r < R; ++r) {
-              FeatVec<TF, VW> x;
-              if (col_ok[r]) x.stage_read(stage_slot(u, r));
-              else x.zero();
-              accumulate<AGG, TF, VW>(acc[r], vj[u], x);
-            }
-        } else {
-          FeatVec<TF, VW> x[U][R];
-#pragma unroll
-          for (int u = 0; u < U; ++u) {
-            const char *rowp = Ab + (uint64_t)cj[u] * ldaB;
-#pragma unroll
-            for (int r = 0; r < R; ++r) {
-              if (col_ok[r]) x[u][r].load(rowp + r * Lg * VW * ES);
-              else x[u][r].zero();
-            }
-          }
-#pragma unroll
-          for (int u = 0; u < U; ++u)
-#pragma unroll
-            for (int r = 0; r < R; ++r) accumulate<AGG, TF, VW>(acc[r], vj[u], x[u][r]);
         }
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+#pragma unroll
+          for (int r = 0; r < R; ++r) accumulate<AGG, TF, VW>(acc[r], vj[u], x[u][r]);
       }
     } else {
       // ---- general path: per-nonzero validity and row-switch procedure
@@ -346,39 +294,18 @@ __device__ __forceinline__ void spmm_body(const SparseArgs &a, const void *__res
           cj[u] = (uint32_t)s_col[jj + u];
           vj[u] = vi ? s_val[jj + u] : 1.f;
         }
-        FeatVec<TF, VW> x[STAGED ? 1 : U][R];
-        if constexpr (STAGED) {
+        FeatVec<TF, VW> x[U][R];
 #pragma unroll
-          for (int u = 0; u < U; ++u) {
-            const char *rowp = Ab + (uint64_t)cj[u] * ldaB;
+        for (int u = 0; u < U; ++u) {
+          const char *rowp = Ab + (uint64_t)cj[u] * ldaB;
 #pragma unroll
-            for (int r = 0; r < R; ++r)
-              if (col_ok[r] && tb + jj + u < n)
-                FeatVec<TF, VW>().stage_issue(stage_slot(u, r), rowp + r * Lg * VW * ES);
-          }
-          cp_async_commit();
-          cp_async_wait<0>();
-        } else {
-#pragma unroll
-          for (int u = 0; u < U; ++u) {
-            const char *rowp = Ab + (uint64_t)cj[u] * ldaB;
-#pragma unroll
-            for (int r = 0; r < R; ++r) {
-              if (col_ok[r] && tb + jj + u < n) x[u][r].load(rowp + r * Lg * VW * ES);
-              else x[u][r].zero();
-            }
+          for (int r = 0; r < R; ++r) {
+            if (col_ok[r] && tb + jj + u < n) x[u][r].load(rowp + r * Lg * VW * ES);
+            else x[u][r].zero();
           }
         }
 #pragma unroll
         for (int u = 0; u < U; ++u) {
-          if constexpr (STAGED) {
-#pragma unroll
-            for (int r = 0; r < R; ++r) {
-              if (col_ok[r] && tb + jj + u < n) x[0][r].stage_read(stage_slot(u, r));
-              else x[0][r].zero();
-            }
-          }
-          FeatVec<TF, VW>(&xu)[R] = x[STAGED ? 0 : u];
           if (tb + jj + u < n) {
             if (rj[u] != cur) {  // row-switch procedure
               if (cur >= 0) {
@@ -392,7 +319,7 @@ __device__ __forceinline__ void spmm_body(const SparseArgs &a, const void *__res
                 for (int v = 0; v < VW; ++v) acc[r][v] = agg_init<AGG>();
             }
 #pragma unroll
-            for (int r = 0; r < R; ++r) accumulate<AGG, TF, VW>(acc[r], vj[u], xu[r]);
+            for (int r = 0; r < R; ++r) accumulate<AGG, TF, VW>(acc[r], vj[u], x[u][r]);
           }
         }
       }
@@ -406,7 +333,7 @@ __device__ __forceinline__ void spmm_body(const SparseArgs &a, const void *__res
 }
 
 template <typename TF, int VW, int L, int R, int VWS, int AGG>
-__global__ void __maxnreg__((SpmmTune<TF, VW, L, R, AGG>::kregs))
+__global__ void __maxnreg__((SpmmTune<TF, VW, L, R, AGG>::regs))
     spmm_kernel(const SparseArgs a, const void *__restrict__ A, const int64_t lda,
                 float *__restrict__ O, const int64_t ldo) {
   spmm_body<TF, VW, L, R, VWS, AGG>(a, A, lda, O, ldo, blockIdx.x);

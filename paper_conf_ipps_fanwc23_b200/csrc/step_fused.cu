@@ -88,8 +88,7 @@ gnn_status_t launch_step_fused(const Plan *p, const gnn_graph_t *g, const float 
   const int64_t per_sd = (int64_t)(32 / lg) * wpb;       // SDDMM chunks per block
   const int64_t nb_sp = (a.num_chunks + per_sp - 1) / per_sp;
   const int64_t nb_sd = (a.num_chunks + per_sd - 1) / per_sd;
-  const int b_sp = spmm_tile_bytes_per_warp(K / 8, vws_sp) +
-                   spmm_stage_bytes_per_warp(4, 8, K / 8, 1, kAggSum);
+  const int b_sp = spmm_tile_bytes_per_warp(K / 8, vws_sp);
   const int b_sd = sddmm_tile_bytes_per_warp(lg, vws_sd);
   const size_t smem = (size_t)wpb * (b_sp > b_sd ? b_sp : b_sd);
   cudaStream_t s = (cudaStream_t)stream;
