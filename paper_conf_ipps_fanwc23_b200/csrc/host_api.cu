@@ -420,12 +420,7 @@ gnn_status_t side_stream(SideStream **out) {
       cudaEventDestroy(t.join);
       t.s = nullptr;
     }
-    // GNN_STEP_SIDE_PRIO=low: the SDDMM's side stream below the caller's (experiment)
-    const char *pr = getenv("GNN_STEP_SIDE_PRIO");
-    int lo = 0, hi = 0;
-    cudaDeviceGetStreamPriorityRange(&lo, &hi);
-    e = cudaStreamCreateWithPriority(&t.s, cudaStreamNonBlocking,
-                                     (pr && pr[0] == 'l') ? lo : 0);
+    e = cudaStreamCreateWithFlags(&t.s, cudaStreamNonBlocking);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&t.fork, cudaEventDisableTiming);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&t.join, cudaEventDisableTiming);
     if (e != cudaSuccess) return cuda_fail(e, "gnn_plan_spmm_sddmm side stream");
@@ -485,20 +480,14 @@ GNN_API gnn_status_t gnn_plan_spmm_sddmm(const gnn_graph_t *g, int32_t K,
     if (e != cudaSuccess) return cuda_fail(e, "gnn_plan_spmm_sddmm fork");
   }
   gnn_status_t st = GNN_OK;
-  // GNN_STEP_SPMM_FIRST=1 enqueues the SpMM (the longer kernel) before the SDDMM (experiment)
-  const char *sf = getenv("GNN_STEP_SPMM_FIRST");
-  const bool spmm_first = sf && sf[0] == '1';
-  auto run_sddmm = [&]() {  // A1 = the graph's own rows of X (row_base), A2T = all of X
-    return launch_sddmm(p, g, X ? X + g->row_base * ldx : nullptr, ldx, X, ldx, out,
-                        fork ? side->s : s, GNN_F32, "gnn_plan_spmm_sddmm sddmm", -1, 0);
-  };
-  auto run_spmm = [&]() {
-    return launch_spmm(p, g, X, ldx, O, ldo, s, GNN_F32, GNN_AGG_SUM, 0,
-                       "gnn_plan_spmm_sddmm spmm", -1, 0);
-  };
-  if (spmm_first && O) st = run_spmm();
-  if (st == GNN_OK && out) st = run_sddmm();
-  if (st == GNN_OK && O && !spmm_first) st = run_spmm();
+  // (the launch order and a low-priority side stream were measured to make no difference,
+  // profiles/r02_s9_c3_fused_ab.txt)
+  if (out)  // A1 = the graph's own rows of X (row_base), A2T = all of X
+    st = launch_sddmm(p, g, X ? X + g->row_base * ldx : nullptr, ldx, X, ldx, out,
+                      fork ? side->s : s, GNN_F32, "gnn_plan_spmm_sddmm sddmm", -1, 0);
+  if (st == GNN_OK && O)
+    st = launch_spmm(p, g, X, ldx, O, ldo, s, GNN_F32, GNN_AGG_SUM, 0,
+                     "gnn_plan_spmm_sddmm spmm", -1, 0);
   if (fork) {  // join even after an error, so `stream` covers everything enqueued
     cudaError_t e = cudaEventRecord(side->join, side->s);
     if (e == cudaSuccess) e = cudaStreamWaitEvent(s, side->join, 0);

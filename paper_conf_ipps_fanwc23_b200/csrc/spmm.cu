@@ -265,13 +265,6 @@ gnn_status_t launch_spmm(const Plan *p, const gnn_graph_t *g, const void *A, int
     vws = effective_vws(in.vw_sparse, g, nullptr);
     if (vws > 2) vws = 2;
   }
-#if GNN_SPMM_VWS_CLAMP
-  {
-    int d = spmm_depth(ES, VW, lanes, vecs, agg) / vecs;
-    if (d < 1) d = 1;
-    while (vws > d) vws >>= 1;
-  }
-#endif
   SpmmFn f = pick_spmm(dtype, VW, lanes, vecs, vws, agg);
   if (!f)
     return fail(GNN_ERR_UNSUPPORTED, "%s: no kernel for vw=%d L=%d agg=%d dtype=%d", who, VW,

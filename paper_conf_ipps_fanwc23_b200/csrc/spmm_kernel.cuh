@@ -39,21 +39,6 @@ struct SpmmTune {
 #endif
 };
 
-// host mirror of SpmmTune::depth (feature vectors in flight per lane) for the launcher
-inline int spmm_depth(int es, int vw, int L, int R, int agg) {
-  const bool wide = vw * es == 32;
-  const bool lean = agg == 0 && R == 1 && wide && (es == 4 || L >= 8);
-#if defined(GNN_SPMM_DEPTH8)
-  (void)lean;
-  return wide ? GNN_SPMM_DEPTH8 : 8;
-#else
-  return R == 2 ? GNN_SPMM_DEPTH_R2 : ((lean || (wide && L <= 2)) ? 4 : 8);
-#endif
-}
-#ifndef GNN_SPMM_VWS_CLAMP
-#define GNN_SPMM_VWS_CLAMP 0  // 1: narrow the sparse copies so a batch is depth/R nonzeros
-#endif
-
 // Aggregators of the node-wise MPP op (Eq. 1): ⊕ = sum (SpMM proper; mean is
 // sum followed by a row scale), max or min of the terms v_i * A[col_i].
 enum : int { kAggSum = 0, kAggMax = 1, kAggMin = 2 };
