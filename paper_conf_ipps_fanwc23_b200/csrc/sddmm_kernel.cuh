@@ -13,12 +13,13 @@ namespace gnn {
 // SDDMM spreads them over Lg = V / Rsd lanes with Rsd vectors per lane, so each dot
 // product is reduced over Lg lanes and 32 / Lg nonzeros are in flight per warp step;
 // U = nonzeros per batch per group, U * Rsd = 8 feature vectors in flight per lane.
-// Measured on the GCR-reordered C4: Rsd = 2 from V = 16 on (round 1, r01_sweep8: K=128
-// 4.82 -> 3.61 ms, K=256 8.85 -> 7.05 ms); at V = 8 (K = 64) round 1 also preferred 2
-// (2.07 -> 1.94 ms), the round-2 kernels prefer 1 (8 lanes x 1 vector, 8 in flight:
-// 1.652 -> 1.544 ms, profiles/r02_s13_sweep_c4_sddmm_r1_k64.txt).
+// Measured on the GCR-reordered C4.  Round 1 (r01_sweep8) preferred Rsd = 2 from V = 8
+// (K=64 2.07 -> 1.94 ms, K=128 4.82 -> 3.61, K=256 8.85 -> 7.05); with the round-2 launch
+// shape one vector per lane wins up to V = 16: fp32 K=64 1.652 -> 1.544 ms, K=128 3.039 ->
+// 2.983, bf16 K=128 1.719 -> 1.662, bf16 K=256 3.211 -> 3.164; at V = 32 (fp32 K=256) the
+// two are equal (profiles/r02_s13_sweep_c4_sddmm_r1_k64.txt, r02_s15_sweep_sddmm_r.txt).
 #ifndef GNN_SDDMM_R2_FROM
-#define GNN_SDDMM_R2_FROM 16  // smallest V that uses Rsd = 2
+#define GNN_SDDMM_R2_FROM 32  // smallest V that uses Rsd = 2
 #endif
 #ifndef GNN_SDDMM_UR
 #define GNN_SDDMM_UR 8       // U * Rsd: feature vectors in flight per lane
