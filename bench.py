@@ -109,6 +109,27 @@ def load_peaks():
     return 6650.0, "fallback (B200_PROFILING.md)"
 
 
+def hbm_copy_in_run(dev, nbytes=1 << 30, reps=5):
+    """SURVEY §8(d) peak #1 re-checked in the same job: torch copy of 1 GiB (read + write
+    bytes / time, best of reps, CUDA events), beside the driver-written MEASURED_PEAKS."""
+    import torch
+    a = torch.empty(nbytes // 4, dtype=torch.float32, device=dev)
+    b = torch.empty_like(a)
+    a.fill_(1.0)
+    best = 1e30
+    for it in range(reps + 1):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        b.copy_(a)
+        e1.record()
+        torch.cuda.synchronize()
+        if it:
+            best = min(best, e0.elapsed_time(e1))
+    del a, b
+    torch.cuda.empty_cache()
+    return round(2 * nbytes / best / 1e6, 1)
+
+
 def probe_own_stream(X, idx, K, chunk=0, reps=3):
     """The gather ceiling of a kernel (SURVEY §8(d) peak #2): gnn_probe_gather -- the
     same 256-bit row loads as the kernels, no arithmetic, no stores -- over THIS
@@ -661,6 +682,9 @@ def run_ours(args):
             "kernels": head["kernels"], "no_reorder": head.get("no_reorder"),
             "bf16": head.get("bf16"), "exchange": exchange,
             "C5": extras.get("C5"), "C3": extras.get("C3"),
+            "peaks_in_run": {"hbm_copy_GBps": hbm_copy_in_run(dev),
+                             "note": "torch copy of 1 GiB, read+write bytes, best of 5; the "
+                                     "roofline's HBM peak is MEASURED_PEAKS.json's"},
             "host": host_info(), "version": git_sha(),
         }
         print(json.dumps(line), flush=True)
