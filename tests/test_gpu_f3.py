@@ -165,12 +165,13 @@ def test_randomized_configurations(seed):
 
 @pytest.mark.parametrize("agg", ["sum", "max", "mean"])
 @pytest.mark.parametrize("C", [0, 8, 64])
-def test_deterministic_spmm_bitwise_reproducible(agg, C):
+@pytest.mark.parametrize("K", [64, 256])
+def test_deterministic_spmm_bitwise_reproducible(agg, C, K):
     """deterministic plans (no atomics: split-row partials summed in chunk order) give the
-    same bits on every run, and match the oracle."""
+    same bits on every run, and match the oracle (K = 256: the widened launch shape, rows
+    of two vectors per lane run on twice the lanes, writes the per-chunk partials too)."""
     for g in graphs():
         dg = upload(g)
-        K = 64
         p = gs.plan(dg, K, force_chunk=C, deterministic=True)
         X = torch.from_numpy(gen.features(70, g.N, K)).to(DEV)
         outs = [gs.spmm(p, dg, X, agg=agg).cpu().numpy() for _ in range(3)]
@@ -257,3 +258,17 @@ def test_extremum_backward_matches_torch_scatter_reduce():
         torch.testing.assert_close(gX, X.grad, rtol=1e-5, atol=1e-5)
         torch.testing.assert_close(gv, v.grad, rtol=1e-5, atol=1e-5)
         X.grad = v.grad = None
+
+
+@pytest.mark.parametrize("K", [32, 256])
+def test_deterministic_bf16_spmm(K):
+    """bf16 features through a deterministic plan (widened launch at K = 256): same bits
+    on every run, within the fp32 bar of the oracle fed the exact bf16 values."""
+    for g in graphs():
+        dg = upload(g)
+        p = gs.plan(dg, K, deterministic=True, feature_dtype="bf16")
+        Xb = torch.from_numpy(gen.features(71, g.N, K)).to(torch.bfloat16).to(DEV)
+        outs = [gs.spmm(p, dg, Xb).cpu().numpy() for _ in range(3)]
+        assert all(np.array_equal(outs[0], o) for o in outs[1:])
+        ref, T = oracle.spmm(g.row_ind, g.col_ind, g.val, Xb.float().cpu().numpy(), M=g.M)
+        assert_within(outs[0], ref, T, what=f"det bf16 K={K}")
