@@ -906,13 +906,16 @@ def run_e2e(args, g, Ks, dev, perm=None, world=1, rank=0):
     r0, r1 = int(b[rank]), int(b[rank + 1])
     e0, e1 = int(g.row_ptr[r0]), int(g.row_ptr[r1])
     M, nnz = r1 - r0, e1 - e0
+    # the shard's CSR offsets go up instead of its RowInd (decoded on the device)
     runner = gs.HostRunner(M, g.N, g.row_ind[e0:e1], g.col_ind[e0:e1],
                            None if g.val is None else g.val[e0:e1], max(Ks), device=dev,
-                           Ks=Ks, row_base=r0).pin()
+                           Ks=Ks, row_base=r0, row_ptr=g.row_ptr[r0:r1 + 1]).pin()
     h_X = {K: feats(K) for K in Ks}
     h_O = {K: torch.empty((M, K), dtype=torch.float32).pin_memory() for K in Ks}
     h_E = {K: torch.empty(nnz, dtype=torch.float32).pin_memory() for K in Ks}
-    h2d = 12 * nnz + sum(4 * g.N * K for K in Ks)      # this rank's copies
+    # this rank's copies: ColInd + Value (8 B per nonzero), the CSR offsets (4 (M + 1) B,
+    # plus one boundary row per piece), X of every width
+    h2d = 8 * nnz + 4 * (M + 1) + sum(4 * g.N * K for K in Ks)
     d2h = sum(4 * M * K for K in Ks) + 4 * nnz * len(Ks)
 
     def step_multi():
@@ -956,6 +959,7 @@ def run_e2e(args, g, Ks, dev, perm=None, world=1, rank=0):
             "ms_per_step": round(ms, 3), "h2d_bytes_per_step": int(h2d),
             "d2h_bytes_per_step": int(d2h), "steps": steps, "api": "gnn_run_host_multi",
             "ranks": world, "sharding": "nnz-balanced row shards (X whole on every rank)",
+            "graph_upload": "CSR offsets + ColInd + Value (RowInd decoded on the device)",
             "per_width_calls": {"api": "gnn_run_host (one call per K)",
                                 "ms_per_step": round(ms_calls, 3),
                                 "value": round(nbytes / (ms_calls * 1e-3) / 1e9, 2)}}

@@ -297,9 +297,12 @@ GNN_API gnn_status_t gnn_permute_rows(const float *X, int64_t ldx, int64_t n, in
  * Deterministic plans run as one piece.  Reads the host row_ind to find the rows each
  * piece completes.  GNN_HOST_TRACE=1 prints a per-piece timeline to stderr (synchronises;
  * a measurement aid).
- * graph_host: host pointers (row_ptr unused), a square N-node graph or a row shard of one
- * (rows [row_base, row_base + M) with row_base + M <= N; SDDMM then uses A1 = those rows
- * of X, O holds the shard's M rows).  fp32 only.
+ * graph_host: host pointers, a square N-node graph or a row shard of one (rows
+ * [row_base, row_base + M) with row_base + M <= N; SDDMM then uses A1 = those rows of X, O
+ * holds the shard's M rows).  If graph_host->row_ptr is given ([M+1], read relative to
+ * row_ptr[0], consistent with row_ind), each piece uploads the CSR offsets of the rows it
+ * spans instead of its RowInd, which is decoded on the device (4 B per nonzero less over
+ * PCIe; row_ind is still read on the host for the piece bookkeeping).  fp32 only.
  * upload_graph = 0 reuses the graph already in this workspace from an earlier call (the
  * graph's offsets do not depend on K, so one workspace sized for the largest K serves all).
  * workspace: gnn_run_host_workspace_bytes(M, N, nnz, K, opts) bytes, 256-B aligned, device. */

@@ -598,11 +598,15 @@ class HostRunner:
     ordered on the current stream (synchronise before reading)."""
 
     def __init__(self, M, N, row_ind, col_ind, val, Kmax, device="cuda", Ks=None, row_base=0,
-                 **opts):
-        """M rows [row_base, row_base + M) of an N-node graph (a row shard when M < N)."""
+                 row_ptr=None, **opts):
+        """M rows [row_base, row_base + M) of an N-node graph (a row shard when M < N).
+        row_ptr (the shard's M + 1 CSR offsets): upload those instead of RowInd."""
         self._keep = [np.ascontiguousarray(row_ind, np.int32),
                       np.ascontiguousarray(col_ind, np.int32),
-                      None if val is None else np.ascontiguousarray(val, np.float32)]
+                      None if val is None else np.ascontiguousarray(val, np.float32),
+                      None if row_ptr is None else np.ascontiguousarray(row_ptr, np.int32)]
+        if row_ptr is not None and self._keep[3].shape[0] != int(M) + 1:
+            raise ValueError("row_ptr must have M + 1 entries")
         self.M, self.N, self.nnz = int(M), int(N), int(row_ind.shape[0] if hasattr(row_ind, "shape") else len(row_ind))
         self.row_base = int(row_base)
         self.opts = _opts(**opts)
@@ -619,17 +623,19 @@ class HostRunner:
             nbytes = max(int(nbytes), int(mb))
         self.ws = torch.empty(max(int(nbytes), 1), dtype=torch.uint8, device=device)
         self.ws_bytes = int(nbytes)
-        self.desc = _Graph(self.M, self.N, self.nnz, None, self._keep[0].ctypes.data,
-                           self._keep[1].ctypes.data,
+        self.desc = _Graph(self.M, self.N, self.nnz,
+                           None if self._keep[3] is None else self._keep[3].ctypes.data,
+                           self._keep[0].ctypes.data, self._keep[1].ctypes.data,
                            None if self._keep[2] is None else self._keep[2].ctypes.data, self.row_base)
 
     def pin(self):
         """Re-point the graph at pinned copies (asynchronous H2D)."""
         pinned = [None if a is None else torch.from_numpy(a).pin_memory() for a in self._keep]
         self._pinned = pinned
-        self.desc = _Graph(self.M, self.N, self.nnz, None, pinned[0].data_ptr(),
-                           pinned[1].data_ptr(), None if pinned[2] is None else pinned[2].data_ptr(),
-                           self.row_base)
+        self.desc = _Graph(self.M, self.N, self.nnz,
+                           None if pinned[3] is None else pinned[3].data_ptr(),
+                           pinned[0].data_ptr(), pinned[1].data_ptr(),
+                           None if pinned[2] is None else pinned[2].data_ptr(), self.row_base)
         return self
 
     def _check_host(self, X_host, K, O_host, out_host):

@@ -21,8 +21,25 @@ constexpr int kMaxPieces = 32;
 constexpr int kMaxK = 16;  // feature widths per gnn_run_host_multi call
 inline size_t a256(size_t b) { return (b + 255) & ~size_t(255); }
 
+// RowInd of nonzeros [b, er) decoded on the device from the CSR offsets of the rows they
+// span (the hybrid format's two row encodings): local rows [ra, ra + nr) with device
+// offsets rp[0..nr] (read relative to base = row_ptr[0]); one warp per row.
+__global__ void csr_range_to_coo_kernel(const int32_t *__restrict__ rp, int64_t nr, int64_t ra,
+                                        int64_t base, int64_t b, int64_t er, int64_t row_base,
+                                        int32_t *__restrict__ row_ind) {
+  const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t r = warp; r < nr; r += nwarps) {
+    int64_t lo = rp[r] - base, hi = rp[r + 1] - base;
+    lo = lo > b ? lo : b;
+    hi = hi < er ? hi : er;
+    for (int64_t i = lo + lane; i < hi; i += 32) row_ind[i] = (int32_t)(ra + r + row_base);
+  }
+}
+
 struct HostLayout {  // offsets inside the workspace; the graph part does not depend on K
-  size_t row_ind, col_ind, val, total;
+  size_t row_ptr, row_ind, col_ind, val, total;
   size_t X[kMaxK], O[kMaxK], out[kMaxK], plan[kMaxK];
 };
 
@@ -31,6 +48,7 @@ struct HostLayout {  // offsets inside the workspace; the graph part does not de
 bool layout(int64_t M, int64_t N, int64_t nnz, int32_t nk, const int32_t *K,
             const gnn_plan_opts_t *opts, HostLayout *l) {
   size_t o = 0;
+  l->row_ptr = o; o += a256(4 * (size_t)(M + 1));
   l->row_ind = o; o += a256(4 * (size_t)nnz);
   l->col_ind = o; o += a256(4 * (size_t)nnz);
   l->val = o;     o += a256(4 * (size_t)nnz);
@@ -328,8 +346,24 @@ GNN_API gnn_status_t gnn_run_host_multi(const gnn_graph_t *gh, int32_t upload_gr
     const int64_t en = p + 1 == P ? nnz : nnz * (p + 1) / P;  // this piece: nonzeros [b, en)
     if (up && en > b) {
       const int64_t er = en < nnz ? en + 1 : nnz;
-      e = cudaMemcpyAsync(w + l.row_ind + 4 * b, gh->row_ind + b, 4 * (er - b),
-                          cudaMemcpyHostToDevice, res.sin);
+      if (gh->row_ptr) {
+        // CSR upload: the offsets of the rows this piece spans (a few bytes) instead of its
+        // RowInd (4 B per nonzero), decoded on the copy-in stream
+        const int64_t ra = gh->row_ind[b] - r0, rb = gh->row_ind[er - 1] - r0;
+        e = cudaMemcpyAsync(w + l.row_ptr + 4 * ra, gh->row_ptr + ra, 4 * (rb - ra + 2),
+                            cudaMemcpyHostToDevice, res.sin);
+        if (e == cudaSuccess) {
+          int64_t blocks = ((rb - ra + 1) * 32 + 255) / 256;
+          if (blocks > 4096) blocks = 4096;
+          csr_range_to_coo_kernel<<<(unsigned)blocks, 256, 0, res.sin>>>(
+              (const int32_t *)(w + l.row_ptr) + ra, rb - ra + 1, ra, gh->row_ptr[0], b, er, r0,
+              (int32_t *)(w + l.row_ind));
+          e = cudaGetLastError();
+        }
+      } else {
+        e = cudaMemcpyAsync(w + l.row_ind + 4 * b, gh->row_ind + b, 4 * (er - b),
+                            cudaMemcpyHostToDevice, res.sin);
+      }
       if (e == cudaSuccess)
         e = cudaMemcpyAsync(w + l.col_ind + 4 * b, gh->col_ind + b, 4 * (en - b),
                             cudaMemcpyHostToDevice, res.sin);

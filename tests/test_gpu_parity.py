@@ -562,14 +562,15 @@ def test_run_host_end_to_end_matches_oracle():
         assert_within(E.numpy(), r2, T2, what=f"run_host sddmm K={K}")
 
 
-def _run_host_check(g, Ks, pieces, seed=900, opts=None):
-    """gnn_run_host with GNN_HOST_PIECES=pieces against the oracle everywhere."""
+def _run_host_check(g, Ks, pieces, seed=900, opts=None, csr=False):
+    """gnn_run_host with GNN_HOST_PIECES=pieces against the oracle everywhere (csr: the
+    graph goes up as CSR offsets, RowInd decoded on the device)."""
     import os
     old = os.environ.get("GNN_HOST_PIECES")
     os.environ["GNN_HOST_PIECES"] = str(pieces)
     try:
         runner = gs.HostRunner(g.M, g.N, g.row_ind, g.col_ind, g.val, max(Ks), device=DEV,
-                               **(opts or {})).pin()
+                               row_ptr=g.row_ptr if csr else None, **(opts or {})).pin()
         for j, K in enumerate(Ks):
             X = torch.from_numpy(_x(seed + K, g.N, K)).pin_memory()
             O = torch.full((g.M, K), float("nan")).pin_memory()
@@ -587,14 +588,16 @@ def _run_host_check(g, Ks, pieces, seed=900, opts=None):
             os.environ["GNN_HOST_PIECES"] = old
 
 
+@pytest.mark.parametrize("csr", [False, True])
 @pytest.mark.parametrize("pieces", [2, 3, 7, 32])
-def test_run_host_pipelined_pieces(pieces):
+def test_run_host_pipelined_pieces(pieces, csr):
     """The copy/compute pipeline of gnn_run_host (pieces of the plan's chunks on two
     compute streams, O rows downloaded as they become final): every output element
     matches the oracle for any piece count, including pieces whose boundaries fall
-    inside a row, before runs of empty rows and inside a hub row."""
+    inside a row, before runs of empty rows and inside a hub row; with the graph uploaded
+    as RowInd or as CSR offsets decoded on the device."""
     g = configs.make_graph("C2")
-    _run_host_check(g, (32, 64, 256), pieces)
+    _run_host_check(g, (32, 64, 256), pieces, csr=csr)
     rng = np.random.default_rng(17)
     M = 3000
     rows = rng.integers(0, M, 60000)
@@ -602,7 +605,7 @@ def test_run_host_pipelined_pieces(pieces):
     rows = np.concatenate([rows, np.full(20000, 1500), [0, M - 1]])  # hub + first/last row
     cols = rng.integers(0, M, rows.size)
     g2 = gen.from_coo(M, M, rows, cols, gen.uniform_values(5, rows.size))
-    _run_host_check(g2, (8, 32, 128), pieces)
+    _run_host_check(g2, (8, 32, 128), pieces, csr=csr)
 
 
 @pytest.mark.parametrize("chunk", [1000, 4096])
@@ -656,7 +659,7 @@ def test_run_host_multi_full_size_bench_config():
     g, perm = full_graph("C4", True)
     Ks = (32, 64, 128, 256)
     runner = gs.HostRunner(g.M, g.N, g.row_ind, g.col_ind, g.val, max(Ks), device=DEV,
-                           Ks=Ks).pin()
+                           Ks=Ks, row_ptr=g.row_ptr).pin()  # CSR upload, as bench.py
     Xs = [torch.from_numpy(_bench_features("C4", g, K, perm)).pin_memory() for K in Ks]
     Os = [torch.full((g.M, K), float("nan")).pin_memory() for K in Ks]
     Es = [torch.full((g.nnz,), float("nan")).pin_memory() for _ in Ks]
@@ -674,7 +677,7 @@ def test_run_host_multi_full_size_bench_config():
         assert_within(Es[j].numpy()[edges], r2, T2, what=f"run_host_multi C4 sddmm K={K}")
 
 
-def _run_multi_check(g, Ks, pieces=None, skip_o=(), seed=950):
+def _run_multi_check(g, Ks, pieces=None, skip_o=(), seed=950, csr=False):
     """gnn_run_host_multi over several widths in one call, every output vs the oracle."""
     import os
     old = os.environ.get("GNN_HOST_PIECES")
@@ -682,7 +685,7 @@ def _run_multi_check(g, Ks, pieces=None, skip_o=(), seed=950):
         os.environ["GNN_HOST_PIECES"] = str(pieces)
     try:
         runner = gs.HostRunner(g.M, g.N, g.row_ind, g.col_ind, g.val, max(Ks), device=DEV,
-                               Ks=Ks).pin()
+                               Ks=Ks, row_ptr=g.row_ptr if csr else None).pin()
         Xs = [torch.from_numpy(_x(seed + K, g.N, K)).pin_memory() for K in Ks]
         Os = [None if j in skip_o else torch.full((g.M, K), float("nan")).pin_memory()
               for j, K in enumerate(Ks)]
@@ -707,19 +710,21 @@ def _run_multi_check(g, Ks, pieces=None, skip_o=(), seed=950):
             os.environ["GNN_HOST_PIECES"] = old
 
 
+@pytest.mark.parametrize("csr", [False, True])
 @pytest.mark.parametrize("pieces", [None, 3, 32])
-def test_run_host_multi_widths(pieces):
+def test_run_host_multi_widths(pieces, csr):
     """Several feature widths in one pipelined gnn_run_host_multi call (per-width plans,
-    pieces alternating over two compute streams across widths, one width's SpMM skipped)."""
+    pieces alternating over two compute streams across widths, one width's SpMM skipped;
+    graph uploaded as RowInd or as CSR offsets)."""
     g = configs.make_graph("C2")
-    _run_multi_check(g, (32, 8, 256, 64), pieces, skip_o=(1,))
+    _run_multi_check(g, (32, 8, 256, 64), pieces, skip_o=(1,), csr=csr)
     rng = np.random.default_rng(23)
     M = 2500
     rows = rng.integers(0, M, 50000)
     rows = rows[(rows % 13) > 3]
     rows = np.concatenate([rows, np.full(15000, 700), [M - 1]])
     g2 = gen.from_coo(M, M, rows, rng.integers(0, M, rows.size), gen.uniform_values(6, rows.size))
-    _run_multi_check(g2, (16, 128), pieces)
+    _run_multi_check(g2, (16, 128), pieces, csr=csr)
 
 
 def test_run_host_multi_rejects_bad_arguments():
@@ -767,7 +772,8 @@ def test_run_host_multi_row_shards():
                 e0, e1 = int(g.row_ptr[r0]), int(g.row_ptr[r1])
                 runner = gs.HostRunner(r1 - r0, g.N, g.row_ind[e0:e1], g.col_ind[e0:e1],
                                        g.val[e0:e1], max(Ks), device=DEV, Ks=Ks,
-                                       row_base=r0).pin()
+                                       row_base=r0,
+                                       row_ptr=g.row_ptr[r0:r1 + 1] if p % 2 else None).pin()
                 Os = [torch.full((r1 - r0, K), float("nan")).pin_memory() for K in Ks]
                 Es = [torch.full((e1 - e0,), float("nan")).pin_memory() for _ in Ks]
                 runner.run_multi(Xs, Ks, Os, Es)
