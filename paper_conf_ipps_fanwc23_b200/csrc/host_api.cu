@@ -495,23 +495,6 @@ GNN_API gnn_status_t gnn_plan_spmm_sddmm(const gnn_graph_t *g, int32_t K,
   Plan *p = reinterpret_cast<Plan *>(plan);
   p->inline_plan = !det;
   cudaStream_t s = (cudaStream_t)stream;
-  // L2 prefetch of the step's inputs by the pre-zero kernel when they fit half of L2
-  // (GNN_STEP_PREFETCH=0: off)
-  {
-    DeviceInfo d;
-    const char *pe = getenv("GNN_STEP_PREFETCH");
-    const int64_t xb = 4 * (int64_t)g->N * ldx, sb = 4 * g->nnz;
-    if (O && X && !(pe && pe[0] == '0') && device_info(&d) == GNN_OK &&
-        xb + 3 * sb <= d.l2_bytes / 2) {
-      const void *ptrs[4] = {X, g->col_ind, g->row_ind, g->val};
-      const int64_t bytes[4] = {xb, sb, sb, sb};
-      for (int i = 0; i < 4; ++i)  // (bulk prefetches need 16-byte aligned ranges)
-        if (ptrs[i] && aligned(ptrs[i], 16)) {
-          p->pf_ptr[i] = ptrs[i];
-          p->pf_bytes[i] = bytes[i];
-        }
-    }
-  }
   // both outputs: one fused launch where the shape has an instance and K <= 32 (measured on
   // 20 C3 subgraphs: K=32 0.0402 -> 0.0367 ms, but K=64 0.0489 -> 0.0523 and K=128 0.0684
   // -> 0.0738: the fused kernel runs the SpMM half at SDDMM's 128-register budget;

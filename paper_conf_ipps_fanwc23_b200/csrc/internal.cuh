@@ -33,16 +33,6 @@ struct Plan {
   int64_t M;
   int64_t row_base;
   bool inline_plan = false;  // kernels recompute the boundary table (gnn_plan_spmm_sddmm)
-  // L2 prefetch of the step's inputs by the pre-zero kernel (gnn_plan_spmm_sddmm): up to 4
-  // byte ranges, each split over the pre-zero grid (cp.async.bulk.prefetch.L2)
-  const void *pf_ptr[4] = {};
-  int64_t pf_bytes[4] = {};
-};
-
-// By-value kernel argument carrying Plan::pf_* (empty: no prefetch).
-struct PrefetchArgs {
-  const char *ptr[4];
-  int64_t bytes[4];
 };
 
 // Kernel parameter block shared by the SpMM / SDDMM launchers.
@@ -101,7 +91,6 @@ int spmm_active_blocks_per_sm(int dtype, int vw, int lanes, int vecs, int warps_
 gnn_status_t check_common(const Plan *p, const gnn_graph_t *g, const char *who);
 int effective_vws(int vws, const gnn_graph_t *g, const void *extra);
 SparseArgs make_args(const Plan *p, const gnn_graph_t *g);
-PrefetchArgs prefetch_args(const Plan *p);
 
 // Launchers (spmm.cu / sddmm.cu); c0 < 0 = every chunk of the plan, else chunks [c0, c1).
 gnn_status_t launch_spmm(const Plan *p, const gnn_graph_t *g, const void *A, int64_t lda,

@@ -31,24 +31,9 @@ namespace gnn {
 // chunk.
 template <int VW>
 __global__ void spmm_prezero_kernel(const SparseArgs a, float *__restrict__ O,
-                                    const int64_t ldo, const float init, const PrefetchArgs pf) {
+                                    const int64_t ldo, const float init) {
   // let a programmatic dependent (the SpMM of gnn_plan_spmm_sddmm) launch right away
   asm volatile("griddepcontrol.launch_dependents;");
-  // one-call step: pull this block's slice of the step's inputs (X, the sparse arrays)
-  // into L2 with one bulk prefetch per range, so the kernels' first gathers do not each
-  // pay a DRAM miss (the inputs of a sampled subgraph fit L2)
-  if (threadIdx.x < 4 && pf.bytes[threadIdx.x] > 0) {
-    const int64_t n = pf.bytes[threadIdx.x];
-    const int64_t per = ((n + gridDim.x - 1) / gridDim.x + 15) & ~int64_t(15);
-    const int64_t b0 = (int64_t)blockIdx.x * per;
-    if (b0 < n) {
-      const int64_t len = b0 + per <= n ? per : ((n - b0) & ~int64_t(15));
-      if (len > 0)
-        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(pf.ptr[threadIdx.x] + b0),
-                     "r"((uint32_t)len)
-                     : "memory");
-    }
-  }
   const int64_t c = a.c_begin + (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5);
   const int lane = threadIdx.x & 31;
   if (c >= a.c_end) return;
@@ -196,15 +181,6 @@ int effective_vws(int vws, const gnn_graph_t *g, const void *extra) {
   return vws;
 }
 
-PrefetchArgs prefetch_args(const Plan *p) {
-  PrefetchArgs f;
-  for (int i = 0; i < 4; ++i) {
-    f.ptr[i] = reinterpret_cast<const char *>(p->pf_ptr[i]);
-    f.bytes[i] = p->pf_ptr[i] ? p->pf_bytes[i] : 0;
-  }
-  return f;
-}
-
 SparseArgs make_args(const Plan *p, const gnn_graph_t *g) {
   SparseArgs a;
   a.row_ind = g->row_ind;
@@ -309,12 +285,11 @@ gnn_status_t launch_spmm(const Plan *p, const gnn_graph_t *g, const void *A, int
   if (!accumulate && !a.carry && c0 < 0) {
     const int64_t blocks = (nch * 32 + 255) / 256;
     const float init = agg == kAggMax ? -INFINITY : agg == kAggMin ? INFINITY : 0.f;
-    const PrefetchArgs pf = prefetch_args(p);
     switch (VO) {
-      case 1: spmm_prezero_kernel<1><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, init, pf); break;
-      case 2: spmm_prezero_kernel<2><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, init, pf); break;
-      case 4: spmm_prezero_kernel<4><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, init, pf); break;
-      default: spmm_prezero_kernel<8><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, init, pf); break;
+      case 1: spmm_prezero_kernel<1><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, init); break;
+      case 2: spmm_prezero_kernel<2><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, init); break;
+      case 4: spmm_prezero_kernel<4><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, init); break;
+      default: spmm_prezero_kernel<8><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, init); break;
     }
   }
   const size_t smem = (size_t)in.warps_per_block * spmm_tile_bytes_per_warp(lanes, vws);
@@ -377,12 +352,11 @@ gnn_status_t launch_spmm_prezero(const Plan *p, const gnn_graph_t *g, float *O, 
   const int VW = p->info.vw_feat, VO = VW < 8 ? VW : 8;
   const int64_t blocks = ((a.c_end - a.c_begin) * 32 + 255) / 256;
   cudaStream_t s = (cudaStream_t)stream;
-  const PrefetchArgs pf = prefetch_args(p);
   switch (VO) {
-    case 1: spmm_prezero_kernel<1><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, 0.f, pf); break;
-    case 2: spmm_prezero_kernel<2><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, 0.f, pf); break;
-    case 4: spmm_prezero_kernel<4><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, 0.f, pf); break;
-    default: spmm_prezero_kernel<8><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, 0.f, pf); break;
+    case 1: spmm_prezero_kernel<1><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, 0.f); break;
+    case 2: spmm_prezero_kernel<2><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, 0.f); break;
+    case 4: spmm_prezero_kernel<4><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, 0.f); break;
+    default: spmm_prezero_kernel<8><<<(unsigned)blocks, 256, 0, s>>>(a, O, ldo, 0.f); break;
   }
   cudaError_t e = cudaGetLastError();
   return e == cudaSuccess ? GNN_OK : cuda_fail(e, "spmm prezero launch");

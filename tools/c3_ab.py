@@ -40,16 +40,13 @@ def main():
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
     stream = torch.cuda.current_stream()
     run = gs.StepRunner(dev)
-    # (GNN_STEP_FUSED, GNN_STEP_PLAN_KERNEL, GNN_STEP_PREFETCH)
-    modes = {"fused": ("1", "0", "1"), "two_kernels": ("0", "0", "1"),
-             "two_kernels_no_prefetch": ("0", "0", "0"), "fused_no_prefetch": ("1", "0", "0"),
-             "plan_kernel": ("0", "1", "0")}
+    # (GNN_STEP_FUSED, GNN_STEP_PLAN_KERNEL)
+    modes = {"fused": ("1", "0"), "two_kernels": ("0", "0"), "plan_kernel": ("0", "1")}
     res = {m: [] for m in modes}
     for rnd in range(a.rounds):
-        for mode, (fz, pk, pf) in modes.items():
+        for mode, (fz, pk) in modes.items():
             os.environ["GNN_STEP_FUSED"] = fz
             os.environ["GNN_STEP_PLAN_KERNEL"] = pk
-            os.environ["GNN_STEP_PREFETCH"] = pf
             for s in subs:
                 run(*s)
             torch.cuda.synchronize()
@@ -64,7 +61,6 @@ def main():
             res[mode].append(statistics.mean(x.elapsed_time(y) for x, y in ev))
     os.environ.pop("GNN_STEP_PLAN_KERNEL", None)
     os.environ.pop("GNN_STEP_FUSED", None)
-    os.environ.pop("GNN_STEP_PREFETCH", None)
     print(json.dumps({"K": K, "graphs": a.graphs, "steps": a.steps,
                       **{f"{m}_ms": [round(x, 4) for x in v] for m, v in res.items()}}))
 
