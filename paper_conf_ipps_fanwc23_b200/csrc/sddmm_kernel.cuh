@@ -200,6 +200,8 @@ __device__ __forceinline__ void sddmm_body(const SparseArgs &a, const void *__re
     cur[sl] = row;
   };
 
+  // (warp-uniform) every lane's columns exist: K is a whole number of slices
+  const bool full = a.K == S * L * VW;
   const int ntiles = (a.chunk + T - 1) / T;
   for (int t = 0; t < ntiles; ++t) {
     const int tb = t * T;
@@ -222,8 +224,9 @@ __device__ __forceinline__ void sddmm_body(const SparseArgs &a, const void *__re
     }
     // The batch loop is instantiated twice: FAST (whole tile in one row, every nonzero
     // valid: no per-nonzero row or bounds logic) and general.
-    auto run_tile = [&](auto fast_tag) {
+    auto run_tile = [&](auto fast_tag, auto full_tag) {
       constexpr bool FAST = decltype(fast_tag)::value;
+      constexpr bool FULL = decltype(full_tag)::value;
 #pragma unroll 1
       for (int jj = 0; jj < T; jj += U) {
         int32_t rj[U];
@@ -250,7 +253,10 @@ __device__ __forceinline__ void sddmm_body(const SparseArgs &a, const void *__re
               const char *rowp = A2l + (uint64_t)cj[u] * ld2B;
 #pragma unroll
               for (int r = 0; r < R; ++r) {
-                if (lane_ok[r] && (FAST || u < valid)) x[u][r].load(rowp + r * Lg * VW * ES);
+                // FULL (no absent columns): no predicate, no zero-fill -- a nonzero past
+                // the chunk end reads row 0 of the zero-filled tile and is not stored
+                if (FULL || (lane_ok[r] && (FAST || u < valid)))
+                  x[u][r].load(rowp + r * Lg * VW * ES);
                 else x[u][r].zero();
               }
             }
@@ -276,7 +282,8 @@ __device__ __forceinline__ void sddmm_body(const SparseArgs &a, const void *__re
     // are requested as soon as this batch's dot products have consumed their registers,
     // BEFORE this batch's shuffle reduction and store, so the memory pipe is not idle
     // while the butterfly runs (same registers: x is dead after the dots).
-    auto run_fast_pipelined = [&]() {
+    auto run_fast_pipelined = [&](auto full_tag) {
+      constexpr bool FULL = decltype(full_tag)::value;
       const char *A2l = A2b + (int64_t)(l * VW) * ES;
       bool lane_ok[R];
 #pragma unroll
@@ -288,7 +295,7 @@ __device__ __forceinline__ void sddmm_body(const SparseArgs &a, const void *__re
           const char *rowp = A2l + (uint64_t)(uint32_t)s_col[jj + u] * ld2B;
 #pragma unroll
           for (int r = 0; r < R; ++r) {
-            if (lane_ok[r]) x[u][r].load(rowp + r * Lg * VW * ES);
+            if (FULL || lane_ok[r]) x[u][r].load(rowp + r * Lg * VW * ES);
             else x[u][r].zero();
           }
         }
@@ -314,7 +321,8 @@ __device__ __forceinline__ void sddmm_body(const SparseArgs &a, const void *__re
 #if GNN_SDDMM_PIPE_GENERAL
     // the same pipelining for tiles with row switches / a partial last tile: the next
     // batch's A2T rows do not depend on the row switches of this one
-    auto run_general_pipelined = [&]() {
+    auto run_general_pipelined = [&](auto full_tag) {
+      constexpr bool FULL = decltype(full_tag)::value;
       const char *A2l = A2b + (int64_t)(l * VW) * ES;
       bool lane_ok[R];
 #pragma unroll
@@ -327,7 +335,7 @@ __device__ __forceinline__ void sddmm_body(const SparseArgs &a, const void *__re
           const char *rowp = A2l + (uint64_t)(uint32_t)s_col[jj + u] * ld2B;
 #pragma unroll
           for (int r = 0; r < R; ++r) {
-            if (lane_ok[r] && u < valid) x[u][r].load(rowp + r * Lg * VW * ES);
+            if (FULL || (lane_ok[r] && u < valid)) x[u][r].load(rowp + r * Lg * VW * ES);
             else x[u][r].zero();
           }
         }
@@ -353,17 +361,24 @@ __device__ __forceinline__ void sddmm_body(const SparseArgs &a, const void *__re
 #endif
     if constexpr (SMAX == 1 && Lg >= 8) {
       if (fast) {
-        run_fast_pipelined();
+        if (full) run_fast_pipelined(std::true_type{});
+        else run_fast_pipelined(std::false_type{});
         continue;
       }
 #if GNN_SDDMM_PIPE_GENERAL
-      run_general_pipelined();
+      if (full) run_general_pipelined(std::true_type{});
+      else run_general_pipelined(std::false_type{});
       continue;
 #endif
     }
 #endif
-    if (fast) run_tile(std::true_type{});
-    else run_tile(std::false_type{});
+    if (fast) {
+      if (full) run_tile(std::true_type{}, std::true_type{});
+      else run_tile(std::true_type{}, std::false_type{});
+    } else {
+      if (full) run_tile(std::false_type{}, std::true_type{});
+      else run_tile(std::false_type{}, std::false_type{});
+    }
   }
 }
 
