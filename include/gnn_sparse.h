@@ -76,7 +76,7 @@ typedef struct {
 /* Plan options; zero-initialised fields take defaults. */
 typedef struct {
   int32_t alpha;           /* InEq. (5) scale factor; default 2             */
-  int32_t warps_per_block; /* WarpsPerBlock; 1..16, default 4               */
+  int32_t warps_per_block; /* WarpsPerBlock; 1..16, default 2               */
   int32_t force_chunk;     /* 0 = DTP choice; >0 forces NnzPerWarp (ablation/tests) */
   int32_t force_vw;        /* 0 = from K; 1/2/4/8 forces the feature vector width   */
   int32_t deterministic;   /* 1: SpMM sums rows split across chunks in chunk order

@@ -45,7 +45,7 @@ class _Graph(ctypes.Structure):
 
 
 class PlanOpts(ctypes.Structure):
-    """gnn_plan_opts_t; zero fields take the library defaults (alpha 2, 4 warps/block)."""
+    """gnn_plan_opts_t; zero fields take the library defaults (alpha 2, 2 warps/block)."""
     _fields_ = [("alpha", ctypes.c_int32), ("warps_per_block", ctypes.c_int32),
                 ("force_chunk", ctypes.c_int32), ("force_vw", ctypes.c_int32),
                 ("deterministic", ctypes.c_int32), ("feature_dtype", ctypes.c_int32),

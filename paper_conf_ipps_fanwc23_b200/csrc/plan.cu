@@ -31,9 +31,10 @@ gnn_status_t make_info(int64_t M, int64_t nnz, int32_t K, const gnn_plan_opts_t 
   gnn_plan_opts_t o{};
   if (opts) o = *opts;
   const int32_t alpha = o.alpha ? o.alpha : 2;
-  // WarpsPerBlock (no value given; DESIGN reading 13): 4 -- measured against 8 at
-  // the same resident warps per SM, 1-3% faster on every C4 kernel (profiles/r02_s1)
-  const int32_t wpb = o.warps_per_block ? o.warps_per_block : 4;
+  // WarpsPerBlock (no value given; DESIGN reading 13): 2 -- at the same resident
+  // warps per SM, 4-warp blocks measured 1-3% faster than 8 (profiles/r02_s1) and 2-warp
+  // blocks 0-1.6% faster than 4 (C4 fp32 / bf16, C5 bf16; C5 fp32 equal; r02_s22/s23)
+  const int32_t wpb = o.warps_per_block ? o.warps_per_block : 2;
   if (M < 0 || nnz < 0 || nnz >= (int64_t(1) << 31) || K < 1 || alpha < 1 || wpb < 1 ||
       wpb * 32 > kMaxThreads || o.force_chunk < 0 || o.deterministic < 0 ||
       o.deterministic > 1 || o.no_locality < 0 || o.no_locality > 1)

@@ -122,7 +122,7 @@ def oracle_plan_checked(p, g, K, **kw):
     assert (info["num_sms"], info["active_blocks_per_sm"], info["l2_bytes"]) == (nsm, abs_, l2)
     dt = kw.get("feature_dtype", 0)
     ref = oracle.plan(g.row_ind, K, nsm, abs_, alpha=kw.get("alpha", 2) or 2,
-                      warps_per_block=kw.get("warps_per_block") or 4,  # library default
+                      warps_per_block=kw.get("warps_per_block") or 2,  # library default
                       force_chunk=kw.get("force_chunk", 0), force_vw=kw.get("force_vw", 0),
                       feature_dtype=1 if dt in (1, "bf16") else 0, M=g.M, l2_bytes=l2)
     assert info == ref.info, (info, ref.info)
