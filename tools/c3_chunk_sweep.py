@@ -26,6 +26,7 @@ def main():
     ap.add_argument("--reps", type=int, default=50)
     ap.add_argument("--K", type=int, default=128)
     ap.add_argument("--alphas", default="0", help="DTP alpha values (0 = library default 2)")
+    ap.add_argument("--wpb", type=int, default=0, help="warps per block (0 = library default)")
     a = ap.parse_args()
     dev = torch.device("cuda:0")
     K = a.K
@@ -44,6 +45,7 @@ def main():
         run = gs.StepRunner(dev)
         run.opts.force_chunk = fc
         run.opts.alpha = al
+        run.opts.warps_per_block = a.wpb
         for s in subs:
             run(s[1], s[2], s[3], s[4])
         torch.cuda.synchronize()
@@ -60,7 +62,7 @@ def main():
         ms = statistics.mean(x.elapsed_time(y) for x, y in per)
         # kernels alone (plan built once, outside the events)
         for (g, dg, X, O, E) in subs:
-            p = gs.plan(dg, K, force_chunk=fc, alpha=al)
+            p = gs.plan(dg, K, force_chunk=fc, alpha=al, warps_per_block=a.wpb)
             chunks.append(p.info()["chunk"])
             for fn, acc in ((lambda: gs.spmm(p, dg, X, out=O), spm),
                             (lambda: gs.sddmm(p, dg, X, X, out=E), sdd)):
@@ -74,7 +76,7 @@ def main():
                     ts.append((e0, e1))
                 torch.cuda.synchronize()
                 acc.append(statistics.median(x.elapsed_time(y) for x, y in ts))
-        print(json.dumps({"force_chunk": fc, "alpha": al or 2, "step_ms": round(ms, 4),
+        print(json.dumps({"force_chunk": fc, "alpha": al or 2, "wpb": a.wpb, "step_ms": round(ms, 4),
                           "spmm_ms_mean": round(statistics.mean(spm), 4),
                           "sddmm_ms_mean": round(statistics.mean(sdd), 4),
                           "chunks": sorted(set(chunks))}), flush=True)
