@@ -281,49 +281,49 @@ __device__ __forceinline__ void spmm_body(const SparseArgs &a, const void *__res
     } else {
       // ---- general path: per-nonzero validity and row-switch procedure
       auto general_tile = [&](auto full_tag) {
-      constexpr bool FULL = decltype(full_tag)::value;
+        constexpr bool FULL = decltype(full_tag)::value;
 #pragma unroll 1
-      for (int jj = 0; jj < T; jj += U) {
-        int32_t rj[U];
-        uint32_t cj[U];
-        float vj[U];
+        for (int jj = 0; jj < T; jj += U) {
+          int32_t rj[U];
+          uint32_t cj[U];
+          float vj[U];
 #pragma unroll
-        for (int u = 0; u < U; ++u) {
-          rj[u] = s_row[jj + u];
-          cj[u] = (uint32_t)s_col[jj + u];
-          vj[u] = vi ? s_val[jj + u] : 1.f;
-        }
-        FeatVec<TF, VW> x[U][R];
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-          const char *rowp = Ab + (uint64_t)cj[u] * ldaB;
-#pragma unroll
-          for (int r = 0; r < R; ++r) {
-            // (FULL: entries past the chunk end read row 0 of the zero-filled tile and are
-            // not accumulated)
-            if (FULL || (col_ok[r] && tb + jj + u < n)) x[u][r].load(rowp + r * Lg * VW * ES);
-            else x[u][r].zero();
+          for (int u = 0; u < U; ++u) {
+            rj[u] = s_row[jj + u];
+            cj[u] = (uint32_t)s_col[jj + u];
+            vj[u] = vi ? s_val[jj + u] : 1.f;
           }
-        }
+          FeatVec<TF, VW> x[U][R];
 #pragma unroll
-        for (int u = 0; u < U; ++u) {
-          if (tb + jj + u < n) {
-            if (rj[u] != cur) {  // row-switch procedure
-              if (cur >= 0) {
-                flush(cur);
-                for (int64_t r = (int64_t)cur + 1; r < rj[u]; ++r) zero_row(r);
-              }
-              cur = rj[u];
+          for (int u = 0; u < U; ++u) {
+            const char *rowp = Ab + (uint64_t)cj[u] * ldaB;
 #pragma unroll
-              for (int r = 0; r < R; ++r)
-#pragma unroll
-                for (int v = 0; v < VW; ++v) acc[r][v] = agg_init<AGG>();
+            for (int r = 0; r < R; ++r) {
+              // (FULL: entries past the chunk end read row 0 of the zero-filled tile and are
+              // not accumulated)
+              if (FULL || (col_ok[r] && tb + jj + u < n)) x[u][r].load(rowp + r * Lg * VW * ES);
+              else x[u][r].zero();
             }
+          }
 #pragma unroll
-            for (int r = 0; r < R; ++r) accumulate<AGG, TF, VW>(acc[r], vj[u], x[u][r]);
+          for (int u = 0; u < U; ++u) {
+            if (tb + jj + u < n) {
+              if (rj[u] != cur) {  // row-switch procedure
+                if (cur >= 0) {
+                  flush(cur);
+                  for (int64_t r = (int64_t)cur + 1; r < rj[u]; ++r) zero_row(r);
+                }
+                cur = rj[u];
+#pragma unroll
+                for (int r = 0; r < R; ++r)
+#pragma unroll
+                  for (int v = 0; v < VW; ++v) acc[r][v] = agg_init<AGG>();
+              }
+#pragma unroll
+              for (int r = 0; r < R; ++r) accumulate<AGG, TF, VW>(acc[r], vj[u], x[u][r]);
+            }
           }
         }
-      }
       };
       if (full) general_tile(std::true_type{});
       else general_tile(std::false_type{});
