@@ -56,7 +56,13 @@ variants/libgnnexp.so: tools/spmm_interleaved.cu $(PKG)/csrc/device.cuh
 	@mkdir -p variants
 	$(NVCC) $(ARCH) -O3 -std=c++17 -shared -Xcompiler -fPIC -Iinclude -o $@ $<
 
+# SM-local traversal experiment (tools/locality_probe.py), not part of the product
+locprobe: variants/liblocprobe.so
+variants/liblocprobe.so: tools/locality_probe.cu
+	@mkdir -p variants
+	$(NVCC) $(ARCH) -O3 -lineinfo -shared -Xcompiler -fPIC -Xptxas -v -o $@ $<
+
 clean:
 	rm -rf gen/libgnngen.so oracle/liboracle.so $(PKG)/libgnnsparse.so build/obj*
 
-.PHONY: all clean variant micro exp
+.PHONY: all clean variant micro exp locprobe

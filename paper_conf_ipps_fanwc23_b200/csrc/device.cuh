@@ -43,6 +43,16 @@ __device__ __forceinline__ uint64_t l2_evict_last() {
 #endif
 
 // ------------------------------------------------------------ features ----
+// address of feature row c: base + c * ldB as ONE mad.wide.u32 (IMAD.WIDE.U32 with the
+// 64-bit base as addend); written as C++ the compiler splits it into IMAD.WIDE + IADD3 +
+// IADD3.X and, under the tight register budgets, reloads the base from the constant bank
+// inside the gather loop
+__device__ __forceinline__ const char *row_addr(const char *base, uint32_t c, uint32_t ldB) {
+  const char *p;
+  asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(p) : "r"(c), "r"(ldB), "l"(base));
+  return p;
+}
+
 template <int VW>
 __device__ __forceinline__ void ld_feat(const float *p, float (&x)[VW]);
 
@@ -530,6 +540,8 @@ struct TmaTiles {
         src[q] = (a == 0 ? ri0 : a == 1 ? ci0 : reinterpret_cast<const int32_t *>(vi0)) + cs;
       }
     }
+    if (!vi0)  // v = 1: value slots hold 1.0 for good (never copied), as AsyncTiles
+      for (int e = lane; e < WORDS; e += 32) vals(0, 0)[e] = vals(1, 0)[e] = 1.f;
     if (lane == 0) {
       mbar_init(bar(0), 1);
       mbar_init(bar(1), 1);
@@ -586,6 +598,13 @@ struct AsyncTiles : SparseTiles<L, VWS> {
     ri = ri0 + own_cs;
     ci = ci0 + own_cs;
     vi = vi0 ? vi0 + own_cs : nullptr;
+    if (!vi0) fill_ones(this->vals(0, g) + l * VWS, this->vals(1, g) + l * VWS);
+  }
+  // val == NULL (v = 1): the value slots of both stages hold 1.0 for good (load() never
+  // writes them), so the kernels read s_val unconditionally -- no select per nonzero
+  __device__ __forceinline__ static void fill_ones(float *a, float *b) {
+#pragma unroll
+    for (int v = 0; v < VWS; ++v) a[v] = b[v] = 1.f;
   }
   __device__ __forceinline__ void issue(int st, int tb, int) const {
     Base::load(st, g, l, ri, ci, vi, tb, cnt);

@@ -250,7 +250,7 @@ __device__ __forceinline__ void sddmm_body(const SparseArgs &a, const void *__re
             FeatVec<TF, VW> x[U][R];
 #pragma unroll
             for (int u = 0; u < U; ++u) {
-              const char *rowp = A2l + (uint64_t)cj[u] * ld2B;
+              const char *rowp = row_addr(A2l, cj[u], ld2B);
 #pragma unroll
               for (int r = 0; r < R; ++r) {
                 // FULL (no absent columns): no predicate, no zero-fill -- a nonzero past
@@ -292,7 +292,7 @@ __device__ __forceinline__ void sddmm_body(const SparseArgs &a, const void *__re
       auto load_batch = [&](int jj) {
 #pragma unroll
         for (int u = 0; u < U; ++u) {
-          const char *rowp = A2l + (uint64_t)(uint32_t)s_col[jj + u] * ld2B;
+          const char *rowp = row_addr(A2l, (uint32_t)s_col[jj + u], ld2B);
 #pragma unroll
           for (int r = 0; r < R; ++r) {
             if (FULL || lane_ok[r]) x[u][r].load(rowp + r * Lg * VW * ES);
@@ -332,7 +332,7 @@ __device__ __forceinline__ void sddmm_body(const SparseArgs &a, const void *__re
         const int valid = n - (tb + jj);
 #pragma unroll
         for (int u = 0; u < U; ++u) {
-          const char *rowp = A2l + (uint64_t)(uint32_t)s_col[jj + u] * ld2B;
+          const char *rowp = row_addr(A2l, (uint32_t)s_col[jj + u], ld2B);
 #pragma unroll
           for (int r = 0; r < R; ++r) {
             if (FULL || (lane_ok[r] && u < valid)) x[u][r].load(rowp + r * Lg * VW * ES);

@@ -145,7 +145,7 @@ __device__ __forceinline__ void spmm_body(const SparseArgs &a, const void *__res
   int32_t rf = 0, rl = 0;
   uint32_t fl = 0;
   if (item_ok) chunk_rows(a, c, rf, rl, fl);
-  // feature row c of A starts at Ab + c * ldaB (IMAD.WIDE.U32 per gather)
+  // feature row c of A starts at Ab + c * ldaB (one IMAD.WIDE.U32 per gather, row_addr)
   const char *__restrict__ Ab = reinterpret_cast<const char *>(A) + (int64_t)k0 * ES;
   const uint32_t ldaB = (uint32_t)lda * (uint32_t)ES;
   float *__restrict__ Ok = O + k0;  // row r at Ok + (r - row_base) * ldo
@@ -196,7 +196,6 @@ __device__ __forceinline__ void spmm_body(const SparseArgs &a, const void *__res
     for (int v = 0; v < VW; ++v) acc[r][v] = agg_init<AGG>();
   int32_t cur = -1;
 
-  const float *__restrict__ vi = a.val ? a.val + cs : nullptr;
   // sparse tiles: per-warp double-buffered shared-memory ring (TMA bulk copies, or
   // cp.async for narrow sparse vectors), one tile ahead of use
   extern __shared__ int32_t gnn_smem[];
@@ -258,12 +257,12 @@ __device__ __forceinline__ void spmm_body(const SparseArgs &a, const void *__res
 #pragma unroll
           for (int u = 0; u < U; ++u) {
             cj[u] = (uint32_t)s_col[jj + u];
-            vj[u] = vi ? s_val[jj + u] : 1.f;
+            vj[u] = s_val[jj + u];  // (1.0 when val == NULL: tiles.init)
           }
           FeatVec<TF, VW> x[U][R];
 #pragma unroll
           for (int u = 0; u < U; ++u) {
-            const char *rowp = Ab + (uint64_t)cj[u] * ldaB;
+            const char *rowp = row_addr(Ab, cj[u], ldaB);
 #pragma unroll
             for (int r = 0; r < R; ++r) {
               if (FULL || col_ok[r]) x[u][r].load(rowp + r * Lg * VW * ES);
@@ -291,12 +290,12 @@ __device__ __forceinline__ void spmm_body(const SparseArgs &a, const void *__res
           for (int u = 0; u < U; ++u) {
             rj[u] = s_row[jj + u];
             cj[u] = (uint32_t)s_col[jj + u];
-            vj[u] = vi ? s_val[jj + u] : 1.f;
+            vj[u] = s_val[jj + u];  // (1.0 when val == NULL: tiles.init)
           }
           FeatVec<TF, VW> x[U][R];
 #pragma unroll
           for (int u = 0; u < U; ++u) {
-            const char *rowp = Ab + (uint64_t)cj[u] * ldaB;
+            const char *rowp = row_addr(Ab, cj[u], ldaB);
 #pragma unroll
             for (int r = 0; r < R; ++r) {
               // (FULL: entries past the chunk end read row 0 of the zero-filled tile and are
