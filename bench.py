@@ -646,6 +646,13 @@ def run_ours(args):
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
         cpu = cpu_baseline(g, Ks, args.cpu_seconds, name)
+    paper_ctx = None
+    if rank == 0 and world == 1 and args.cusparse:
+        torch.cuda.empty_cache()
+        try:
+            paper_ctx = vs_cusparse_block(g, perm, Ks, name, dev)
+        except Exception as ex:  # context only: never lose the main line
+            paper_ctx = {"error": f"{type(ex).__name__}: {ex}"[:300]}
     del g, g0
     extras = {}
     if args.extras and name == "C4" and not args.K:
@@ -681,7 +688,7 @@ def run_ours(args):
             "gpu_launches": head["gpu_launches"], "clocks": head["clocks"],
             "kernels": head["kernels"], "no_reorder": head.get("no_reorder"),
             "bf16": head.get("bf16"), "exchange": exchange,
-            "C5": extras.get("C5"), "C3": extras.get("C3"),
+            "C5": extras.get("C5"), "C3": extras.get("C3"), "paper_context": paper_ctx,
             "peaks_in_run": {"hbm_copy_GBps": hbm_copy_in_run(dev),
                              "note": "torch copy of 1 GiB, read+write bytes, best of 5; the "
                                      "roofline's HBM peak is MEASURED_PEAKS.json's"},
@@ -691,6 +698,76 @@ def run_ours(args):
     if world > 1:
         dist.barrier()
         dist.destroy_process_group()
+
+
+def vs_cusparse_block(g, perm, Ks, name, dev, reps=3):
+    """North star: the paper's own speedups quoted alongside.  The paper's headline numbers
+    are speedups over cuSPARSE (Table III: HP-SpMM vs cuSPARSE CSR ALG2 1.90x / 2.53x
+    full-graph on V100 / A30; HP-SDDMM vs cuSPARSE CSR SDDMM 10.90x / 11.17x).
+    The B200 analogue: our SpMM / SDDMM vs cuSPARSE through torch.sparse (CSR SpMM =
+    torch.sparse.mm, CSR SDDMM = torch.sparse.sampled_addmm, default algorithms) on the same
+    device graph and features, kernel time only, L2 flushed before each launch, the two
+    alternated, medians.  Outside the timed region; context, not the metric
+    (tools/vs_cusparse.py is the standalone version)."""
+    import warnings
+
+    import torch
+
+    import paper_conf_ipps_fanwc23_b200 as gs
+    from gen import configs
+
+    with warnings.catch_warnings():
+        warnings.simplefilter("ignore")
+        S = torch.sparse_csr_tensor(torch.from_numpy(g.row_ptr).to(dev),
+                                    torch.from_numpy(g.col_ind).to(dev),
+                                    torch.from_numpy(g.val).to(dev), size=(g.M, g.N))
+    dg = gs.DeviceGraph.from_arrays(g.M, g.N, g.row_ind, g.col_ind, g.val, g.row_ptr,
+                                    device=dev)
+    flush = torch.empty(256 * 1024 * 1024 // 4, device=dev)
+
+    def once(fn):
+        flush.fill_(1.0)
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        fn()
+        b.record()
+        torch.cuda.synchronize()
+        return a.elapsed_time(b)
+
+    out = {}
+    for K in Ks:
+        X = torch.from_numpy(configs.make_features(name, g.N, K)).to(dev)
+        if perm is not None:
+            X = gs.permute_rows(X, torch.from_numpy(perm))
+        O = torch.empty((g.M, K), device=dev)
+        E = torch.empty(g.nnz, device=dev)
+        p = gs.plan(dg, K)
+        fns = {"ours_spmm": lambda: gs.spmm(p, dg, X, out=O),
+               "cusparse_spmm": lambda: torch.sparse.mm(S, X),
+               "ours_sddmm": lambda: gs.sddmm(p, dg, X, X, out=E),
+               "cusparse_sddmm": lambda: torch.sparse.sampled_addmm(S, X, X.t(), beta=0.0)}
+        for fn in fns.values():
+            fn()
+        t = {k: [] for k in fns}
+        for _ in range(reps):
+            for k, fn in fns.items():
+                t[k].append(once(fn))
+        med = {k: statistics.median(v) for k, v in t.items()}
+        out[f"K{K}"] = {**{k + "_ms": round(v, 4) for k, v in med.items()},
+                        "spmm_speedup": round(med["cusparse_spmm"] / med["ours_spmm"], 2),
+                        "sddmm_speedup": round(med["cusparse_sddmm"] / med["ours_sddmm"], 2)}
+        del X, O, E, p
+    return {"vs_cusparse": out,
+            "workload": f"{name} (the headline graph and features, same layout)",
+            "cusparse": f"torch {torch.__version__} torch.sparse CSR (int32 indices), "
+                        "default algorithms; its SDDMM omits the v_i scaling",
+            "paper": {"hp_spmm_vs_cusparse_csr_alg2": {"V100": 1.90, "A30": 2.53,
+                                                       "source": "Table III, P:367"},
+                      "hp_sddmm_vs_cusparse_csr_sddmm": {"V100": 10.90, "A30": 11.17,
+                                                         "source": "P:373"},
+                      "note": "full-graph averages over 19 graphs at K = 32/64/128 on the "
+                              "paper's GPUs and cuSPARSE of CUDA 11.8 (P:321-323): context, "
+                              "not a like-for-like target"}}
 
 
 def c3_block(args, dev, world, rank):
@@ -1090,6 +1167,8 @@ def main():
     ap.add_argument("--c3-graphs", type=int, default=20)
     ap.add_argument("--no-c3-cuda-graphs", dest="c3_cuda_graphs", action="store_false")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-cusparse", dest="cusparse", action="store_false",
+                    help="skip the paper-context block (our kernels vs cuSPARSE)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-reorder", dest="reorder", action="store_false",
                     help="time the graph as generated (default: GCR-reordered offline first, "
