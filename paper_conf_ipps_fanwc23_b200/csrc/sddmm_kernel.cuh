@@ -321,35 +321,39 @@ __device__ __forceinline__ void sddmm_body(const SparseArgs &a, const void *__re
 #if GNN_SDDMM_PIPE_GENERAL
     // the same pipelining for tiles with row switches / a partial last tile: the next
     // batch's A2T rows do not depend on the row switches of this one
-    auto run_general_pipelined = [&](auto full_tag) {
+    auto run_general_pipelined = [&](auto full_tag, auto whole_tag) {
       constexpr bool FULL = decltype(full_tag)::value;
+      constexpr bool WHOLE = decltype(whole_tag)::value;  // tile inside every chunk
       const char *A2l = A2b + (int64_t)(l * VW) * ES;
       bool lane_ok[R];
 #pragma unroll
       for (int r = 0; r < R; ++r) lane_ok[r] = item_ok && (r * Lg + l) * VW < a.K;
       FeatVec<TF, VW> x[U][R];
       auto load_batch = [&](int jj) {
-        const int valid = n - (tb + jj);
+        const int valid = WHOLE ? U : n - (tb + jj);
 #pragma unroll
         for (int u = 0; u < U; ++u) {
           const char *rowp = row_addr(A2l, (uint32_t)s_col[jj + u], ld2B);
 #pragma unroll
           for (int r = 0; r < R; ++r) {
-            if (FULL || (lane_ok[r] && u < valid)) x[u][r].load(rowp + r * Lg * VW * ES);
-            else x[u][r].zero();
+            if (FULL || (lane_ok[r] && (WHOLE || u < valid)))
+              x[u][r].load(rowp + r * Lg * VW * ES);
+            else
+              x[u][r].zero();
           }
         }
       };
       load_batch(0);
 #pragma unroll 1
       for (int jj = 0; jj < T; jj += U) {
-        const int valid = n - (tb + jj);
+        const int valid = WHOLE ? U : n - (tb + jj);
         float part[U];
 #pragma unroll
         for (int u = 0; u < U; ++u) {
           part[u] = 0.f;
           const int32_t rj = s_row[jj + u];
-          if (item_ok && u < valid && rj != cur[0]) load_a1_slice(0, rj);  // Algo 4 l. 8-11
+          if (item_ok && (WHOLE || u < valid) && rj != cur[0])
+            load_a1_slice(0, rj);  // Algo 4 l. 8-11
 #pragma unroll
           for (int r = 0; r < R; ++r) part[u] = dot_f<TF, VW>(part[u], a1[0][r], x[u][r]);
         }
@@ -366,8 +370,14 @@ __device__ __forceinline__ void sddmm_body(const SparseArgs &a, const void *__re
         continue;
       }
 #if GNN_SDDMM_PIPE_GENERAL
-      if (full) run_general_pipelined(std::true_type{});
-      else run_general_pipelined(std::false_type{});
+      // (warp-uniform) every group's tile lies inside its chunk: no per-nonzero bounds test
+      if (__all_sync(kFull, tb + T <= n || !item_ok)) {
+        if (full) run_general_pipelined(std::true_type{}, std::true_type{});
+        else run_general_pipelined(std::false_type{}, std::true_type{});
+      } else {
+        if (full) run_general_pipelined(std::true_type{}, std::false_type{});
+        else run_general_pipelined(std::false_type{}, std::false_type{});
+      }
       continue;
 #endif
     }

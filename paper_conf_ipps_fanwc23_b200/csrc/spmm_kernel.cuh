@@ -278,9 +278,14 @@ __device__ __forceinline__ void spmm_body(const SparseArgs &a, const void *__res
       if (full) fast_tile(std::true_type{});
       else fast_tile(std::false_type{});
     } else {
-      // ---- general path: per-nonzero validity and row-switch procedure
-      auto general_tile = [&](auto full_tag) {
+      // ---- general path: per-nonzero row-switch procedure
+      // WHOLE (warp-uniform): every group's tile lies inside its chunk, so no per-nonzero
+      // validity test (a group past the last chunk reads the zero-filled tile -- row 0 --
+      // and never flushes: its first row switch starts from cur = -1 and the final flush
+      // below is guarded by item_ok)
+      auto general_tile = [&](auto full_tag, auto whole_tag) {
         constexpr bool FULL = decltype(full_tag)::value;
+        constexpr bool WHOLE = decltype(whole_tag)::value;
 #pragma unroll 1
         for (int jj = 0; jj < T; jj += U) {
           int32_t rj[U];
@@ -300,13 +305,24 @@ __device__ __forceinline__ void spmm_body(const SparseArgs &a, const void *__res
             for (int r = 0; r < R; ++r) {
               // (FULL: entries past the chunk end read row 0 of the zero-filled tile and are
               // not accumulated)
-              if (FULL || (col_ok[r] && tb + jj + u < n)) x[u][r].load(rowp + r * Lg * VW * ES);
-              else x[u][r].zero();
+              if (FULL || (col_ok[r] && (WHOLE || tb + jj + u < n)))
+                x[u][r].load(rowp + r * Lg * VW * ES);
+              else
+                x[u][r].zero();
             }
+          }
+          // (warp-uniform) no group switches rows within this batch (rows are sorted, so
+          // the batch's last row decides): plain accumulation, no per-nonzero tests
+          if (WHOLE && __all_sync(kFull, rj[U - 1] == cur || !item_ok)) {
+#pragma unroll
+            for (int u = 0; u < U; ++u)
+#pragma unroll
+              for (int r = 0; r < R; ++r) accumulate<AGG, TF, VW>(acc[r], vj[u], x[u][r]);
+            continue;
           }
 #pragma unroll
           for (int u = 0; u < U; ++u) {
-            if (tb + jj + u < n) {
+            if (WHOLE || tb + jj + u < n) {
               if (rj[u] != cur) {  // row-switch procedure
                 if (cur >= 0) {
                   flush(cur);
@@ -324,11 +340,16 @@ __device__ __forceinline__ void spmm_body(const SparseArgs &a, const void *__res
           }
         }
       };
-      if (full) general_tile(std::true_type{});
-      else general_tile(std::false_type{});
+      if (__all_sync(kFull, tb + T <= n || !item_ok)) {
+        if (full) general_tile(std::true_type{}, std::true_type{});
+        else general_tile(std::false_type{}, std::true_type{});
+      } else {
+        if (full) general_tile(std::true_type{}, std::false_type{});
+        else general_tile(std::false_type{}, std::false_type{});
+      }
     }
   }
-  if (cur >= 0) flush(cur);
+  if (cur >= 0 && item_ok) flush(cur);
   // trailing empty rows after the last chunk
   if (item_ok && c == a.num_chunks - 1) {
     for (int64_t r = (int64_t)rl + 1; r < a.row_base + a.M; ++r) zero_row(r);
