@@ -348,14 +348,25 @@ __device__ __forceinline__ void sddmm_body(const SparseArgs &a, const void *__re
       for (int jj = 0; jj < T; jj += U) {
         const int valid = WHOLE ? U : n - (tb + jj);
         float part[U];
+        if (WHOLE && __all_sync(kFull, s_row[jj + U - 1] == cur[0] || !item_ok)) {
+          // no group switches rows within this batch (rows are sorted): no per-nonzero
+          // row test, the cached A1 row serves all U dot products
 #pragma unroll
-        for (int u = 0; u < U; ++u) {
-          part[u] = 0.f;
-          const int32_t rj = s_row[jj + u];
-          if (item_ok && (WHOLE || u < valid) && rj != cur[0])
-            load_a1_slice(0, rj);  // Algo 4 l. 8-11
+          for (int u = 0; u < U; ++u) {
+            part[u] = 0.f;
 #pragma unroll
-          for (int r = 0; r < R; ++r) part[u] = dot_f<TF, VW>(part[u], a1[0][r], x[u][r]);
+            for (int r = 0; r < R; ++r) part[u] = dot_f<TF, VW>(part[u], a1[0][r], x[u][r]);
+          }
+        } else {
+#pragma unroll
+          for (int u = 0; u < U; ++u) {
+            part[u] = 0.f;
+            const int32_t rj = s_row[jj + u];
+            if (item_ok && (WHOLE || u < valid) && rj != cur[0])
+              load_a1_slice(0, rj);  // Algo 4 l. 8-11
+#pragma unroll
+            for (int r = 0; r < R; ++r) part[u] = dot_f<TF, VW>(part[u], a1[0][r], x[u][r]);
+          }
         }
         if (jj + U < T) load_batch(jj + U);
         reduce_scale_store<U, Lg>(part, vi ? s_val + jj : nullptr, l, oc + tb + jj,
