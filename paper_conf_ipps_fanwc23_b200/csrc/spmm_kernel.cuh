@@ -142,6 +142,27 @@ __device__ __forceinline__ void spmm_body(const SparseArgs &a, const void *__res
   for (int r = 0; r < R; ++r) col_ok[r] = item_ok && k0 + r * Lg * VW < a.K;
   const int64_t cs = c * a.chunk;
   const int n = item_ok ? (int)(min(cs + (int64_t)a.chunk, a.nnz) - cs) : 0;  // nnz here
+  // sparse tiles: per-warp double-buffered shared-memory ring (TMA bulk copies, or
+  // cp.async for narrow sparse vectors), one tile ahead of use -- the first tile is
+  // requested before the chunk's boundary rows are read, so the two latencies overlap
+  extern __shared__ int32_t gnn_smem[];
+  Tiles tiles;
+  {
+    const int64_t item0 =
+        a.c_begin * a.slices + (bid * (blockDim.x >> 5) + (threadIdx.x >> 5)) * G;
+    tiles.init(gnn_smem + (threadIdx.x >> 5) * Tiles::WARP_WORDS, lane, a.row_ind, a.col_ind,
+               a.val, [&](int gg, int64_t &cs_, int &n_) {
+                 const int64_t it = item0 + gg;
+                 cs_ = 0;
+                 n_ = 0;
+                 if (it < a.c_end * a.slices) {
+                   cs_ = (it / a.slices) * a.chunk;
+                   n_ = (int)(min(cs_ + (int64_t)a.chunk, a.nnz) - cs_);
+                 }
+               },
+               cs, n);
+  }
+  tiles.issue(0, 0, lane);
   int32_t rf = 0, rl = 0;
   uint32_t fl = 0;
   if (item_ok) chunk_rows(a, c, rf, rl, fl);
@@ -196,26 +217,6 @@ __device__ __forceinline__ void spmm_body(const SparseArgs &a, const void *__res
     for (int v = 0; v < VW; ++v) acc[r][v] = agg_init<AGG>();
   int32_t cur = -1;
 
-  // sparse tiles: per-warp double-buffered shared-memory ring (TMA bulk copies, or
-  // cp.async for narrow sparse vectors), one tile ahead of use
-  extern __shared__ int32_t gnn_smem[];
-  Tiles tiles;
-  {
-    const int64_t item0 =
-        a.c_begin * a.slices + (bid * (blockDim.x >> 5) + (threadIdx.x >> 5)) * G;
-    tiles.init(gnn_smem + (threadIdx.x >> 5) * Tiles::WARP_WORDS, lane, a.row_ind, a.col_ind,
-               a.val, [&](int gg, int64_t &cs_, int &n_) {
-                 const int64_t it = item0 + gg;
-                 cs_ = 0;
-                 n_ = 0;
-                 if (it < a.c_end * a.slices) {
-                   cs_ = (it / a.slices) * a.chunk;
-                   n_ = (int)(min(cs_ + (int64_t)a.chunk, a.nnz) - cs_);
-                 }
-               },
-               cs, n);
-  }
-  tiles.issue(0, 0, lane);
 
   const int ntiles = (a.chunk + T - 1) / T;  // warp-uniform trip count
   for (int t = 0; t < ntiles; ++t) {
