@@ -330,13 +330,25 @@ __device__ __forceinline__ void spmm_body(const SparseArgs &a, const void *__res
                   for (int64_t r = (int64_t)cur + 1; r < rj[u]; ++r) zero_row(r);
                 }
                 cur = rj[u];
+                if constexpr (AGG == kAggSum) {
+                  // the new row starts at its first term (v*x, = 0 + v*x): both branches
+                  // write the accumulator in place, no merge copies per nonzero
 #pragma unroll
-                for (int r = 0; r < R; ++r)
+                  for (int r = 0; r < R; ++r)
 #pragma unroll
-                  for (int v = 0; v < VW; ++v) acc[r][v] = agg_init<AGG>();
+                    for (int v = 0; v < VW; ++v) acc[r][v] = vj[u] * x[u][r].get(v);
+                } else {
+#pragma unroll
+                  for (int r = 0; r < R; ++r) {
+#pragma unroll
+                    for (int v = 0; v < VW; ++v) acc[r][v] = agg_init<AGG>();
+                    accumulate<AGG, TF, VW>(acc[r], vj[u], x[u][r]);
+                  }
+                }
+              } else {
+#pragma unroll
+                for (int r = 0; r < R; ++r) accumulate<AGG, TF, VW>(acc[r], vj[u], x[u][r]);
               }
-#pragma unroll
-              for (int r = 0; r < R; ++r) accumulate<AGG, TF, VW>(acc[r], vj[u], x[u][r]);
             }
           }
         }
