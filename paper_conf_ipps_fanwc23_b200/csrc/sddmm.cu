@@ -51,6 +51,15 @@ gnn_status_t launch_sddmm(const Plan *p, const gnn_graph_t *g, const void *A1, i
     V = 4;
   }
 #endif
+#if GNN_SDDMM_NARROW_LG8
+  // single-slice rows of four 32-byte vectors (fp32 K = 32, bf16 K = 64): a 4-lane dot
+  // product takes the unpipelined path; as eight 16-byte vectors (8-lane dot products) the
+  // next batch's gathers are issued before this batch's butterfly (run_fast_pipelined)
+  if (in.slices == 1 && V == 4 && VWk * ES == 32) {
+    VWk /= 2;
+    V = 8;
+  }
+#endif
   SddmmFn f = dtype == GNN_BF16 ? pick_sddmm_bf16(VWk, V, vws, in.slices)
                                 : pick_sddmm_f32(VWk, V, vws, in.slices);
   if (!f)
