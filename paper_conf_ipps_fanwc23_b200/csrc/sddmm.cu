@@ -55,7 +55,7 @@ gnn_status_t launch_sddmm(const Plan *p, const gnn_graph_t *g, const void *A1, i
   // single-slice rows of four 32-byte vectors (fp32 K = 32, bf16 K = 64): a 4-lane dot
   // product takes the unpipelined path; as eight 16-byte vectors (8-lane dot products) the
   // next batch's gathers are issued before this batch's butterfly (run_fast_pipelined)
-  if (in.slices == 1 && V == 4 && VWk * ES == 32) {
+  if (in.slices == 1 && V == 4 && VWk * ES >= GNN_SDDMM_NARROW_MIN_BYTES) {
     VWk /= 2;
     V = 8;
   }

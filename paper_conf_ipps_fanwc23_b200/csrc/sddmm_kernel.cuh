@@ -30,6 +30,10 @@ namespace gnn {
 #ifndef GNN_SDDMM_PIPE
 #define GNN_SDDMM_PIPE 1     // next batch's loads issued before this batch's reduction
 #endif
+#ifndef GNN_SDDMM_NARROW_MIN_BYTES
+#define GNN_SDDMM_NARROW_MIN_BYTES 32  // ... only vectors of at least this many bytes (16:
+                                       // bf16 K=32 as 8-byte vectors, 3% slower on C4, r02_s41)
+#endif
 #ifndef GNN_SDDMM_NARROW_LG8
 #define GNN_SDDMM_NARROW_LG8 1  // 4 x 32-byte single-slice rows run as 8 x 16-byte (sddmm.cu;
                                 // C4 fp32 K=32 0.924 -> 0.891 ms, bf16 K=64 0.984 -> 0.964, r02_s38)
