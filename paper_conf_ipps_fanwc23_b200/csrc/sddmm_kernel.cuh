@@ -47,16 +47,26 @@ struct SddmmShape {
   static constexpr int Lg = V / R;
   static constexpr int depth = GNN_SDDMM_UR / R > 1 ? GNN_SDDMM_UR / R : 1;
 };
-// Register budget per thread: 128 = 2 resident blocks of 8 warps per SM, 80 = 3, 64 = 4.
+// Register budget per thread: 128 = 8 resident 2-warp blocks per SM, 96 = 10.  Rows of
+// one vector per lane (R = 1: fp32 K <= 128, bf16 K <= 256) fit 96 without spilling and
+// gain from the extra warps (fp32 C4 K=32 0.891 -> 0.859 ms, K=64 1.496 -> 1.461, K=128
+// 2.860 -> 2.773, C5 K=64 2.154 -> 2.063, C3 step 0.0599 -> 0.0590; bf16 C4 K=128 1.592
+// -> 1.513, K=256 3.009 -> 2.866); two-vector rows (R = 2, fp32 K = 256) lose 7-9% at 96
+// and keep 128 (profiles/r02_s47_sweep_sddmm_regs.txt, r02_s48_sweep_sddmm_regs_r1.txt).
 #ifndef GNN_SDDMM_REGS
 #define GNN_SDDMM_REGS 128
+#endif
+#ifndef GNN_SDDMM_REGS_R1
+#define GNN_SDDMM_REGS_R1 96
 #endif
 #ifndef GNN_SDDMM_REGS_BF16
 #define GNN_SDDMM_REGS_BF16 GNN_SDDMM_REGS
 #endif
-template <typename TF>
+template <typename TF, int VW, int V, int SMAX>
 struct SddmmRegs {
-  static constexpr int value = TF::bytes == 2 ? GNN_SDDMM_REGS_BF16 : GNN_SDDMM_REGS;
+  static constexpr int value = (SddmmShape<VW, V, SMAX>::R == 1 && SMAX == 1)
+                                   ? GNN_SDDMM_REGS_R1
+                                   : (TF::bytes == 2 ? GNN_SDDMM_REGS_BF16 : GNN_SDDMM_REGS);
 };
 
 // WarpReduce (Algo 4 line 12) of U partial dot products at once over the group's L
@@ -412,7 +422,7 @@ __device__ __forceinline__ void sddmm_body(const SparseArgs &a, const void *__re
 }
 
 template <typename TF, int VW, int L, int VWS, int SMAX>
-__global__ void __maxnreg__(SddmmRegs<TF>::value)
+__global__ void __maxnreg__((SddmmRegs<TF, VW, L, SMAX>::value))
     sddmm_kernel(const SparseArgs a, const void *__restrict__ A1, const int64_t lda1,
                  const void *__restrict__ A2T, const int64_t lda2, float *__restrict__ out) {
   sddmm_body<TF, VW, L, VWS, SMAX>(a, A1, lda1, A2T, lda2, out, blockIdx.x);
