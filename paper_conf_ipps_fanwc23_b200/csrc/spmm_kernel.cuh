@@ -21,6 +21,16 @@ namespace gnn {
 //   K=256 3.91 -> 3.75 ms; everything else (narrow bf16 rows, max / min, two-vector rows
 //   that stay so) keeps 128 registers and the round-1 depths (r01_sweep4 / 12 / 19).
 // GNN_SPMM_REGS / GNN_SPMM_DEPTH8 / GNN_SPMM_DEPTH_R2 override the table (build sweeps).
+#ifndef GNN_SPMM_REGS_F32
+#define GNN_SPMM_REGS_F32 80  // lean fp32 rows (one 256-bit vector per lane), L <= 8 lanes
+#endif
+// ... rows of >= 16 lanes (K >= 128): 72 registers (14 resident 2-warp blocks instead of 12,
+// 8 B of spill in a cold path): C4 K=128 2.820 -> 2.745 ms, K=256 5.62-5.69 -> 5.54-5.55,
+// C5 K=256 -1%; at L <= 8 it measured 0.1-0.5% slower and 64 registers lose 4-11%
+// everywhere (profiles/r02_s49_sweep_spmm_regs.txt)
+#ifndef GNN_SPMM_REGS_F32_WIDE
+#define GNN_SPMM_REGS_F32_WIDE 72
+#endif
 #ifndef GNN_SPMM_DEPTH_R2
 #define GNN_SPMM_DEPTH_R2 4
 #endif
@@ -32,7 +42,8 @@ struct SpmmTune {
 #if defined(GNN_SPMM_REGS)
   static constexpr int regs = GNN_SPMM_REGS;
 #else
-  static constexpr int regs = lean ? (f32 ? 80 : 96) : 128;
+  static constexpr int regs =
+      lean ? (f32 ? (L >= 16 ? GNN_SPMM_REGS_F32_WIDE : GNN_SPMM_REGS_F32) : 96) : 128;
 #endif
 #if defined(GNN_SPMM_DEPTH8)
   static constexpr int depth = wide ? GNN_SPMM_DEPTH8 : 8;
