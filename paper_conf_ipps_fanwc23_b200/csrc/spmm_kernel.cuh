@@ -31,6 +31,10 @@ namespace gnn {
 #ifndef GNN_SPMM_REGS_F32_WIDE
 #define GNN_SPMM_REGS_F32_WIDE 72
 #endif
+#ifndef GNN_SPMM_REGS_BF16
+#define GNN_SPMM_REGS_BF16 96  // lean bf16 rows of >= 8 lanes (88: 84 used, no spill, but
+                               // K=256 2% slower, r02_s51)
+#endif
 #ifndef GNN_SPMM_DEPTH_R2
 #define GNN_SPMM_DEPTH_R2 4
 #endif
@@ -43,7 +47,8 @@ struct SpmmTune {
   static constexpr int regs = GNN_SPMM_REGS;
 #else
   static constexpr int regs =
-      lean ? (f32 ? (L >= 16 ? GNN_SPMM_REGS_F32_WIDE : GNN_SPMM_REGS_F32) : 96) : 128;
+      lean ? (f32 ? (L >= 16 ? GNN_SPMM_REGS_F32_WIDE : GNN_SPMM_REGS_F32) : GNN_SPMM_REGS_BF16)
+           : 128;
 #endif
 #if defined(GNN_SPMM_DEPTH8)
   static constexpr int depth = wide ? GNN_SPMM_DEPTH8 : 8;
